@@ -1,0 +1,104 @@
+// Internal structures shared by the host planner (plan.cpp, run.cu) and the device kernels.
+// Not part of the C ABI (include/brickdl.h is).
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/brickdl.h"
+
+namespace bdl {
+
+constexpr int kMaxLayers = 16;   // layers per merged subgraph handled by one kernel
+
+// Bricked tensor view (device side).  Dimension order everywhere: 0=n, 1=d, 2=h, 3=w.
+struct TView {
+    void *ptr;
+    int ext[4];          // logical extents (N, D, H, W)
+    int C, Cp;           // channels, padded channels
+    int B[4];            // brick extents
+    int nb[4];           // bricks per dim
+    const int32_t *bmap; // logical -> physical, or null
+    long long brick_elems;
+};
+
+// One layer as the CUDA-core brick kernels see it.
+struct GLayer {
+    int kind;            // bdl_opkind
+    int cin, cout;
+    int k[4], s[4], p[4];   // index 0 (batch) always k=1, s=1, p=0
+    int in_ext[4], out_ext[4];
+    int relu;
+    int res_ext;         // 1: add the external residual view `res` (same extents as output)
+    const float *w;      // packed [taps][cin][cout] fp32 (workspace)
+    const float *bias;   // [cout] fp32 (workspace) or null
+    TView res;
+    TView out;           // memo buffer / subgraph output (bricked) for this layer's output
+};
+
+enum KernelKind { KERNEL_BRICK = 0, KERNEL_TC_BAND = 1 };
+
+struct Layer {
+    bdl_layer L;               // as given
+    int in_ext[4], out_ext[4]; // (n, d, h, w)
+    int64_t w_off = -1, b_off = -1;  // workspace offsets of packed weights / bias
+    int64_t tc_w_off = -1;           // tcgen05 packed weights
+};
+
+struct Tensor {                 // materialized tensor between subgraphs
+    int producer;               // layer index, -1 = graph input
+    bdl_layout layout;
+    int64_t ws_off;             // -1: user buffer (graph input / output)
+};
+
+struct Subgraph {
+    int first, last;
+    int mode;                   // bdl_mode (resolved)
+    int mode_model;             // what the Delta rule chose
+    int model_brick;            // rho/tau choice (edge)
+    int64_t rho;
+    double delta, delta_first;
+    int kernel;                 // KernelKind
+    int in_tensor;              // index into Plan::tensors
+    int out_tensor;
+    std::vector<int> res_tensor;   // per layer in subgraph: tensor index of external residual, or -1
+    // memoized mode
+    std::vector<int64_t> memo_off; // per layer (except last): bricked intermediate buffer offsets
+    int64_t status_off = -1;       // int32 [L][tasks]
+    std::vector<int64_t> task_base;// per layer offset into the status table (in words)
+    int64_t ntasks_total = 0;
+    int64_t counter_off = -1;      // uint64 [4] + ticket counter
+    // padded mode scratch (CUDA-core kernel)
+    int64_t scratch_off = -1;
+    int64_t scratch_slot_floats = 0;
+    int grid = 0;                  // persistent grid size
+    uint64_t ticket_base = 0;      // memo ticket counter offset for the next run
+    unsigned epoch = 0;            // memo tag epoch (bumped every run; tags of older epochs read as state 0)
+    // tcgen05 band kernel parameters
+    int tc_band = 0;               // band rows
+    int tc_smem = 0;
+    std::vector<int64_t> tc_inter_off;
+};
+
+}  // namespace bdl
+
+struct bdl_plan {
+    std::vector<bdl::Layer> layers;
+    std::vector<bdl::Subgraph> sgs;
+    std::vector<bdl::Tensor> tensors;
+    bdl_layout in_layout, out_layout;
+    bdl_plan_opts opts;
+    int64_t ws_bytes = 0;
+    uint32_t epoch = 0;
+    int num_sms = 148;
+    int64_t l2_bytes = 0;
+    bool prepared = false;
+    void *prepared_ws = nullptr;
+};
+
+namespace bdl {
+void set_error(const std::string &msg);
+bdl_status fail(bdl_status s, const std::string &msg);
+bool layout_valid(const bdl_layout *l);
+TView make_view(const bdl_layout &l, void *ptr);
+}  // namespace bdl

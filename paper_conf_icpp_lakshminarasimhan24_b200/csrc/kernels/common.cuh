@@ -1,0 +1,54 @@
+// Device helpers shared by the BrickDL kernels (product path only).
+#pragma once
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+
+#include "../internal.h"
+
+namespace bdl {
+
+__device__ __forceinline__ float to_f(float v) { return v; }
+__device__ __forceinline__ float to_f(__nv_bfloat16 v) { return __bfloat162float(v); }
+template <typename T> __device__ __forceinline__ T from_f(float v);
+template <> __device__ __forceinline__ float from_f<float>(float v) { return v; }
+template <> __device__ __forceinline__ __nv_bfloat16 from_f<__nv_bfloat16>(float v) { return __float2bfloat16_rn(v); }
+// value after storage rounding, kept in fp32
+template <typename T> __device__ __forceinline__ float store_round(float v) { return to_f(from_f<T>(v)); }
+
+// Physical brick index of a logical brick (BrickMap, Fig 6b).
+__device__ __forceinline__ long long tv_phys(const TView &v, long long logical) {
+    return v.bmap ? (long long)v.bmap[logical] : logical;
+}
+
+// Element offset of channel 0 at logical position (n, d, h, w) (must be inside the bricked grid).
+__device__ __forceinline__ long long tv_off(const TView &v, int n, int d, int h, int w) {
+    int bn = n / v.B[0], bd = d / v.B[1], bh = h / v.B[2], bw = w / v.B[3];
+    long long logical = (((long long)bn * v.nb[1] + bd) * v.nb[2] + bh) * v.nb[3] + bw;
+    long long phys = tv_phys(v, logical);
+    int in = (((n - bn * v.B[0]) * v.B[1] + (d - bd * v.B[1])) * v.B[2] + (h - bh * v.B[2])) * v.B[3] + (w - bw * v.B[3]);
+    return phys * v.brick_elems + (long long)in * v.Cp;
+}
+
+__device__ __forceinline__ bool tv_inside(const TView &v, int n, int d, int h, int w) {
+    return n >= 0 && n < v.ext[0] && d >= 0 && d < v.ext[1] && h >= 0 && h < v.ext[2] && w >= 0 && w < v.ext[3];
+}
+
+// ---- memory-model helpers for the memo table (release/acquire at GPU scope)
+__device__ __forceinline__ int ld_acquire(const int *p) {
+    int v;
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(int *p, int v) {
+    asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+}  // namespace bdl
+
+#define BDL_CUDA_CHECK_LAUNCH(name)                                                  \
+    do {                                                                             \
+        cudaError_t e__ = cudaGetLastError();                                        \
+        if (e__ != cudaSuccess)                                                      \
+            return ::bdl::fail(BDL_ECUDA, std::string(name) + ": " + cudaGetErrorString(e__)); \
+    } while (0)

@@ -1,0 +1,484 @@
+// Static analysis (§3.3): graph partitioning (L603-626), padded-vs-memoized mode choice
+// by padding data growth Delta (L628-647), brick-size model rho/tau (L649-662), and the
+// workspace layout of a plan.  Host-only C++.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "internal.h"
+
+namespace bdl {
+
+// Output extent of a layer along one dim: floor((I + 2p - (k-1) - 1)/s) + 1.
+static int out_extent(int I, int k, int s, int p) { return (I + 2 * p - (k - 1) - 1) / s + 1; }
+
+static int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+
+// ---------------------------------------------------------------------------------------------
+// Region analysis (Fig 4): reverse traversal from an output brick region [a, b) of the
+// subgraph's last layer; returns per layer the INPUT region of that layer (unclipped) along one dim.
+// in_lo[j], in_hi[j] for j = 0..L-1 (layer first+j).
+static void regions_1d(const std::vector<Layer> &ly, int first, int last, int dim, int64_t a, int64_t b,
+                       std::vector<int64_t> &in_lo, std::vector<int64_t> &in_hi) {
+    int L = last - first + 1;
+    in_lo.assign(L, 0);
+    in_hi.assign(L, 0);
+    for (int j = L - 1; j >= 0; j--) {
+        const bdl_layer &l = ly[first + j].L;
+        int k = dim == 0 ? 1 : l.k[dim - 1], s = dim == 0 ? 1 : l.stride[dim - 1], p = dim == 0 ? 0 : l.pad[dim - 1];
+        int64_t lo = a * s - p, hi = (b - 1) * s - p + k;  // input extent I = s(O-1) + k (Q19)
+        in_lo[j] = lo;
+        in_hi[j] = hi;
+        a = lo;
+        b = hi;
+    }
+}
+
+// Delta: sum over layers and bricks of the padded input region (clipped at the feature
+// map) over the halo-free region, minus 1.  `first_only` gives the alternative reading (first
+// layer's input only).  Brick extents B[4] over (n, d, h, w) of the last layer's output.
+double compute_delta(const std::vector<Layer> &ly, int first, int last, const int B[4], bool first_only) {
+    int L = last - first + 1;
+    const Layer &lastL = ly[last];
+    std::vector<double> pad_sum(L, 1.0), exact_sum(L, 1.0);
+    for (int dim = 0; dim < 4; dim++) {
+        int64_t ext_out = lastL.out_ext[dim];
+        int64_t nb = (ext_out + B[dim] - 1) / B[dim];
+        std::vector<double> ps(L, 0.0), es(L, 0.0);
+        for (int64_t i = 0; i < nb; i++) {
+            int64_t a = i * B[dim], b = std::min<int64_t>(a + B[dim], ext_out);
+            std::vector<int64_t> lo, hi;
+            regions_1d(ly, first, last, dim, a, b, lo, hi);
+            // halo-free region: strides only
+            int64_t ea = a, eb = b;
+            std::vector<int64_t> elo(L), ehi(L);
+            for (int j = L - 1; j >= 0; j--) {
+                const bdl_layer &l = ly[first + j].L;
+                int s = dim == 0 ? 1 : l.stride[dim - 1];
+                ea *= s;
+                eb *= s;
+                elo[j] = ea;
+                ehi[j] = eb;
+            }
+            for (int j = 0; j < L; j++) {
+                int64_t I = ly[first + j].in_ext[dim];
+                ps[j] += (double)std::max<int64_t>(0, std::min(hi[j], I) - std::max<int64_t>(lo[j], 0));
+                es[j] += (double)std::max<int64_t>(0, std::min(ehi[j], I) - std::max<int64_t>(elo[j], 0));
+            }
+        }
+        for (int j = 0; j < L; j++) {
+            pad_sum[j] *= ps[j];
+            exact_sum[j] *= es[j];
+        }
+    }
+    double P = 0, E = 0;
+    for (int j = 0; j < (first_only ? 1 : L); j++) {
+        double c = ly[first + j].L.cin;
+        P += c * pad_sum[j];
+        E += c * exact_sum[j];
+    }
+    return E > 0 ? P / E - 1.0 : 0.0;
+}
+
+// rho/tau brick-size model (L649-658): rho(B) = prod(blocked dims) / B^n over the candidate set,
+// pick the largest rho <= tau (the batch counts as a blocked dim, so rho = #bricks).
+int model_brick(const bdl_plan_opts &o, int nsp, const int ext[4], int64_t *rho_out) {
+    int best = -1;
+    double best_rho = -1;
+    int largest = 0;
+    for (int i = 0; i < 4; i++) {
+        int Bc = o.bcand[i];
+        if (Bc <= 0) continue;
+        largest = std::max(largest, Bc);
+        double rho = (double)ext[0];
+        for (int d = 4 - nsp; d < 4; d++) rho *= (double)ext[d] / Bc;
+        if (rho <= (double)o.tau && rho > best_rho) {
+            best_rho = rho;
+            best = Bc;
+        }
+    }
+    if (best < 0) {  // every candidate exceeds tau: the coarsest brick
+        best = largest;
+        best_rho = (double)ext[0];
+        for (int d = 4 - nsp; d < 4; d++) best_rho *= (double)ext[d] / best;
+    }
+    if (rho_out) *rho_out = (int64_t)std::llround(best_rho);
+    return best;
+}
+
+static bool is_pool(const Layer &l) { return l.L.kind == BDL_OP_MAXPOOL; }
+
+}  // namespace bdl
+
+namespace bdl {
+int tc_band_rows(const bdl_plan *p, const Subgraph &sg, int *smem_out);
+}
+using namespace bdl;
+
+// ---------------------------------------------------------------------------------------------
+// tcgen05 band-kernel eligibility (3x3 stride-1 pad-1 2-D convs, Cin = Cout = C,
+// C in {16, 32, 64, 128}, batch brick 1, residual only from the subgraph input at the last layer).
+
+static bool tc_eligible(const bdl_plan *p, const Subgraph &sg) {
+    if (p->in_layout.dtype != BDL_BF16) return false;
+    if (p->in_layout.Bn != 1) return false;
+    const Layer &f = p->layers[sg.first];
+    int C = f.L.cin;
+    if (!(C == 16 || C == 32 || C == 64 || C == 128)) return false;
+    int nsp = p->in_layout.nsp;
+    for (int j = sg.first; j <= sg.last; j++) {
+        const bdl_layer &l = p->layers[j].L;
+        if (l.kind != BDL_OP_CONV || l.cin != C || l.cout != C) return false;
+        for (int d = 0; d < 3; d++) {
+            bool spatial = (nsp == 3) || d > 0;
+            int k = spatial ? 3 : 1, pp = spatial ? 1 : 0;
+            if (l.k[d] != k || l.stride[d] != 1 || l.pad[d] != pp) return false;
+        }
+        int jj = j - sg.first;
+        int rt = sg.res_tensor[jj];
+        if (rt >= 0 && !(j == sg.last && rt == sg.in_tensor)) return false;
+        if (l.residual != BDL_NO_RESIDUAL && rt < 0) return false;
+    }
+    int smem = 0;
+    return tc_band_rows(p, sg, &smem) > 0;
+}
+
+extern "C" {
+
+bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const bdl_layout *in,
+                               const bdl_plan_opts *opts_in, bdl_plan **out) {
+    if (!layers || nlayers <= 0 || !out) return fail(BDL_EINVAL, "bdl_graph_partition: bad arguments");
+    if (!layout_valid(in)) return fail(BDL_EINVAL, "bdl_graph_partition: bad input layout");
+    *out = nullptr;
+    bdl_plan *p = new (std::nothrow) bdl_plan();
+    if (!p) return fail(BDL_ENOMEM, "bdl_graph_partition: out of host memory");
+    if (opts_in) p->opts = *opts_in; else bdl_plan_opts_default(&p->opts);
+    p->in_layout = *in;
+
+    // device facts (the planner also runs on hosts without a GPU: B200 defaults)
+    p->num_sms = 148;
+    p->l2_bytes = 126LL << 20;
+    int dev_count = 0;
+    if (cudaGetDeviceCount(&dev_count) == cudaSuccess && dev_count > 0) {
+        int dev = 0, v = 0;
+        cudaGetDevice(&dev);
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0) p->num_sms = v;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrL2CacheSize, dev) == cudaSuccess && v > 0) p->l2_bytes = v;
+    } else {
+        cudaGetLastError();
+    }
+    if (p->opts.num_sms > 0) p->num_sms = p->opts.num_sms;
+    int64_t budget = p->opts.onchip_budget > 0 ? p->opts.onchip_budget : p->l2_bytes;
+
+    // ---- layer shapes
+    const int nsp = in->nsp;
+    p->layers.resize(nlayers);
+    for (int i = 0; i < nlayers; i++) {
+        Layer &L = p->layers[i];
+        L.L = layers[i];
+        const bdl_layer &l = layers[i];
+        if (l.kind != BDL_OP_CONV && l.kind != BDL_OP_MAXPOOL) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EUNSUPPORTED, "layer " + std::to_string(i) + ": unknown op kind");
+        }
+        if (l.input < -1 || l.input >= i) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": input must be an earlier layer or -1");
+        }
+        int cin_expected = l.input == -1 ? (int)in->C : layers[l.input].cout;
+        if (l.cin != cin_expected || l.cout <= 0 || (l.kind == BDL_OP_MAXPOOL && l.cout != l.cin)) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": channel count mismatch");
+        }
+        if (l.kind == BDL_OP_CONV && !l.w) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": conv without weights");
+        }
+        const int *src = nullptr;
+        int gin[4] = {(int)in->N, (int)in->D, (int)in->H, (int)in->W};
+        src = l.input == -1 ? gin : p->layers[l.input].out_ext;
+        for (int d = 0; d < 4; d++) L.in_ext[d] = src[d];
+        L.out_ext[0] = L.in_ext[0];
+        for (int d = 0; d < 3; d++) {
+            if (l.k[d] <= 0 || l.stride[d] <= 0 || l.pad[d] < 0 || (nsp == 2 && d == 0 && (l.k[0] != 1 || l.stride[0] != 1 || l.pad[0] != 0))) {
+                bdl_plan_destroy(p);
+                return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": bad kernel/stride/pad");
+            }
+            L.out_ext[d + 1] = out_extent(L.in_ext[d + 1], l.k[d], l.stride[d], l.pad[d]);
+            if (L.out_ext[d + 1] <= 0) {
+                bdl_plan_destroy(p);
+                return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": empty output");
+            }
+        }
+        if (l.residual != BDL_NO_RESIDUAL) {
+            if (l.residual < -1 || l.residual >= i) {
+                bdl_plan_destroy(p);
+                return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": bad residual index");
+            }
+            const int *rs = l.residual == -1 ? gin : p->layers[l.residual].out_ext;
+            int rc = l.residual == -1 ? (int)in->C : layers[l.residual].cout;
+            bool same = rc == l.cout;
+            for (int d = 0; d < 4; d++) same = same && rs[d] == L.out_ext[d];
+            if (!same) {
+                bdl_plan_destroy(p);
+                return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": residual shape mismatch");
+            }
+        }
+    }
+    const int Bx[4] = {in->Bn, in->Bd, in->Bh, in->Bw};
+    // Q8: a brick must be at least the kernel's extent (L741) for the layers of a merged subgraph.
+    auto fits_brick = [&](int j) {
+        const bdl_layer &l = p->layers[j].L;
+        for (int d = 0; d < 3; d++)
+            if (l.k[d] > Bx[d + 1] || l.pad[d] > Bx[d + 1]) return false;
+        return true;
+    };
+    auto consumed_after = [&](int m, int end) {
+        for (int j = end + 1; j < nlayers; j++)
+            if (p->layers[j].L.input == m || p->layers[j].L.residual == m) return true;
+        return false;
+    };
+    auto range_ok = [&](int first, int end) {
+        if (p->opts.max_subgraph_layers > 0 && end - first + 1 > p->opts.max_subgraph_layers) return false;
+        if (end - first + 1 > kMaxLayers) return false;
+        for (int j = first; j <= end; j++) {
+            if (!fits_brick(j)) return false;
+            if (j > first && p->layers[j].L.input != j - 1) return false;      // a chain
+            if (j < end && is_pool(p->layers[j])) return false;                 // pool ends a subgraph (L620-626)
+            int r = p->layers[j].L.residual;
+            if (r != BDL_NO_RESIDUAL && r >= first) return false;                // residual must be materialized
+            if (j < end && consumed_after(j, end)) return false;               // no live-out inside
+        }
+        // footprint (L605-614): concurrently resident bricks x padded regions (+ memo tags)
+        int nconc = 2 * p->num_sms;
+        int64_t fp = 0;
+        std::vector<int64_t> lo, hi;
+        int64_t vol_sum = 0;
+        {
+            std::vector<int64_t> ext(end - first + 1, 1);
+            for (int d = 0; d < 4; d++) {
+                regions_1d(p->layers, first, end, d, 0, Bx[d], lo, hi);
+                for (int j = 0; j <= end - first; j++) ext[j] *= (hi[j] - lo[j]);
+            }
+            for (int j = 0; j <= end - first; j++) vol_sum += ext[j] * p->layers[first + j].L.cin;
+        }
+        fp = (int64_t)nconc * vol_sum * in->elem_bytes;
+        for (int j = first; j <= end; j++) {
+            const bdl_layer &l = p->layers[j].L;
+            fp += (int64_t)l.cout * l.cin * l.k[0] * l.k[1] * l.k[2] * in->elem_bytes;
+        }
+        return fp <= budget;
+    };
+
+    // ---- reverse traversal partition (L605-614)
+    std::vector<std::pair<int, int>> ranges;
+    int end = nlayers - 1;
+    while (end >= 0) {
+        int first = end;
+        while (first - 1 >= 0 && !is_pool(p->layers[first - 1]) && range_ok(first - 1, end)) first--;
+        ranges.push_back({first, end});
+        end = first - 1;
+    }
+    std::reverse(ranges.begin(), ranges.end());
+
+    // ---- tensors: graph input, every subgraph output
+    Tensor tin;
+    tin.producer = -1;
+    tin.layout = *in;
+    tin.ws_off = -1;
+    p->tensors.push_back(tin);
+    auto tensor_of = [&](int producer) {
+        for (size_t t = 0; t < p->tensors.size(); t++)
+            if (p->tensors[t].producer == producer) return (int)t;
+        return -1;
+    };
+    for (auto &r : ranges) {
+        Subgraph sg;
+        sg.first = r.first;
+        sg.last = r.second;
+        const Layer &fl = p->layers[sg.first];
+        sg.in_tensor = tensor_of(fl.L.input);
+        if (sg.in_tensor < 0) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EINVAL, "partition: subgraph input is not materialized (internal error)");
+        }
+        const Layer &ll = p->layers[sg.last];
+        Tensor t;
+        t.producer = sg.last;
+        bdl_layout_init(&t.layout, nsp, ll.out_ext[0], ll.L.cout, ll.out_ext[1], ll.out_ext[2], ll.out_ext[3],
+                        in->Bn, in->Bd, in->Bh, in->Bw, in->dtype);
+        t.ws_off = 0;
+        if (t.layout.N == in->N && t.layout.D == in->D && t.layout.H == in->H && t.layout.W == in->W)
+            t.layout.brickmap = in->brickmap;  // same grid: keep the caller's BrickMap
+        p->tensors.push_back(t);
+        sg.out_tensor = (int)p->tensors.size() - 1;
+        for (int j = sg.first; j <= sg.last; j++) {
+            int r2 = p->layers[j].L.residual;
+            if (r2 == BDL_NO_RESIDUAL) {
+                sg.res_tensor.push_back(-1);
+            } else {
+                int t2 = tensor_of(r2);
+                if (t2 < 0) {
+                    bdl_plan_destroy(p);
+                    return fail(BDL_EUNSUPPORTED, "layer " + std::to_string(j) + ": residual source is not a subgraph output");
+                }
+                sg.res_tensor.push_back(t2);
+            }
+        }
+        // ---- models
+        int ext_in[4];
+        for (int d = 0; d < 4; d++) ext_in[d] = fl.in_ext[d];
+        sg.model_brick = model_brick(p->opts, nsp, ext_in, &sg.rho);
+        sg.delta = compute_delta(p->layers, sg.first, sg.last, Bx, false);
+        sg.delta_first = compute_delta(p->layers, sg.first, sg.last, Bx, true);
+        // executed brick = the layout's; the tiny-layer rule (L659-662) uses it
+        double rho_exec = (double)ext_in[0];
+        int64_t bn = 1;
+        for (int d = 4 - nsp; d < 4; d++) {
+            rho_exec *= (double)ext_in[d] / Bx[d];
+            bn *= Bx[d];
+        }
+        if (sg.last == sg.first) sg.mode_model = BDL_MODE_UNMERGED;
+        else if (rho_exec < (double)bn) sg.mode_model = BDL_MODE_UNMERGED;
+        else sg.mode_model = sg.delta > p->opts.delta_threshold ? BDL_MODE_MEMOIZED : BDL_MODE_PADDED;
+        sg.mode = p->opts.force_mode != BDL_MODE_AUTO ? p->opts.force_mode : sg.mode_model;
+        p->sgs.push_back(sg);
+    }
+    p->tensors.back().ws_off = -1;  // graph output is the user's buffer
+    p->out_layout = p->tensors.back().layout;
+    for (auto &sg : p->sgs) sg.kernel = tc_eligible(p, sg) ? KERNEL_TC_BAND : KERNEL_BRICK;
+
+    // ---- workspace layout
+    int64_t off = 0;
+    auto take = [&](int64_t bytes) {
+        int64_t o = align_up(off, 256);
+        off = o + align_up(bytes, 256);
+        return o;
+    };
+    for (auto &L : p->layers) {
+        if (L.L.kind != BDL_OP_CONV) continue;
+        int64_t taps = (int64_t)L.L.k[0] * L.L.k[1] * L.L.k[2];
+        L.w_off = take(taps * L.L.cin * L.L.cout * 4);
+        L.b_off = take((int64_t)L.L.cout * 4);
+    }
+    for (auto &sg : p->sgs)
+        if (sg.kernel == KERNEL_TC_BAND)
+            for (int j = sg.first; j <= sg.last; j++) {
+                Layer &L = p->layers[j];
+                int64_t taps = (int64_t)L.L.k[0] * L.L.k[1] * L.L.k[2];
+                L.tc_w_off = take(taps * L.L.cin * L.L.cout * 2);
+            }
+    for (size_t t = 1; t + 1 < p->tensors.size(); t++) p->tensors[t].ws_off = take(p->tensors[t].layout.total_bytes);
+    for (auto &sg : p->sgs) {
+        int L = sg.last - sg.first + 1;
+        sg.memo_off.assign(L, -1);
+        sg.task_base.assign(L, 0);
+        int64_t words = 0;
+        for (int j = 0; j < L; j++) {
+            const Layer &ly = p->layers[sg.first + j];
+            bdl_layout lo;
+            bdl_layout_init(&lo, nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
+                            in->Bn, in->Bd, in->Bh, in->Bw, in->dtype);
+            if (j < L - 1) sg.memo_off[j] = take(lo.total_bytes);
+            sg.task_base[j] = words;
+            words += lo.nbricks;
+        }
+        sg.ntasks_total = words;
+        sg.status_off = take(words * 4);
+        sg.counter_off = take(8 * 8);
+        // padded-mode scratch for the CUDA-core kernel: two ping-pong region buffers per CTA
+        int64_t maxvol = 1;
+        {
+            std::vector<int64_t> ext(L, 1);
+            std::vector<int64_t> lo, hi;
+            for (int d = 0; d < 4; d++) {
+                regions_1d(p->layers, sg.first, sg.last, d, 0, Bx[d], lo, hi);
+                for (int j = 0; j < L; j++) ext[j] *= (hi[j] - lo[j]);
+            }
+            // output region of layer j (j < L-1) == input region of layer j+1
+            for (int j = 1; j < L; j++) maxvol = std::max(maxvol, ext[j] * (int64_t)p->layers[sg.first + j].L.cin);
+        }
+        sg.grid = 4 * p->num_sms;
+        sg.scratch_slot_floats = align_up(maxvol, 64);
+        sg.scratch_off = L > 1 ? take((int64_t)sg.grid * 2 * sg.scratch_slot_floats * 4) : -1;
+        if (sg.kernel == KERNEL_TC_BAND) sg.tc_band = tc_band_rows(p, sg, &sg.tc_smem);
+    }
+    p->ws_bytes = align_up(off, 256);
+    *out = p;
+    return BDL_OK;
+}
+
+int32_t bdl_plan_num_subgraphs(const bdl_plan *p) { return p ? (int32_t)p->sgs.size() : 0; }
+
+bdl_status bdl_plan_subgraph(const bdl_plan *p, int32_t i, int32_t *first, int32_t *last, int32_t *mode,
+                             int32_t *mbrick, double *delta, int32_t *kernel) {
+    if (!p || i < 0 || i >= (int)p->sgs.size()) return fail(BDL_EINVAL, "bdl_plan_subgraph: bad index");
+    const Subgraph &s = p->sgs[i];
+    if (first) *first = s.first;
+    if (last) *last = s.last;
+    if (mode) *mode = s.mode;
+    if (mbrick) *mbrick = s.model_brick;
+    if (delta) *delta = s.delta;
+    if (kernel) *kernel = s.kernel;
+    return BDL_OK;
+}
+
+bdl_status bdl_plan_set_mode(bdl_plan *p, int32_t i, int32_t mode) {
+    if (!p || i < 0 || i >= (int)p->sgs.size()) return fail(BDL_EINVAL, "bdl_plan_set_mode: bad index");
+    if (mode == BDL_MODE_AUTO) mode = p->sgs[i].mode_model;
+    if (mode < BDL_MODE_PADDED || mode > BDL_MODE_UNMERGED) return fail(BDL_EINVAL, "bdl_plan_set_mode: bad mode");
+    p->sgs[i].mode = mode;
+    p->prepared = false;
+    return BDL_OK;
+}
+
+bdl_status bdl_plan_out_layout(const bdl_plan *p, bdl_layout *out) {
+    if (!p || !out) return fail(BDL_EINVAL, "bdl_plan_out_layout: NULL");
+    *out = p->out_layout;
+    return BDL_OK;
+}
+
+int64_t bdl_plan_workspace_bytes(const bdl_plan *p) { return p ? p->ws_bytes : 0; }
+
+void bdl_plan_destroy(bdl_plan *p) { delete p; }
+
+// Extra host-side introspection used by tests (not in the header's required set, but C ABI):
+// Delta alternative reading and rho of subgraph i.
+bdl_status bdl_plan_subgraph_model(const bdl_plan *p, int32_t i, double *delta_first, int64_t *rho,
+                                   int32_t *mode_model, int32_t *tc_band) {
+    if (!p || i < 0 || i >= (int)p->sgs.size()) return fail(BDL_EINVAL, "bad index");
+    const Subgraph &s = p->sgs[i];
+    if (delta_first) *delta_first = s.delta_first;
+    if (rho) *rho = s.rho;
+    if (mode_model) *mode_model = s.mode_model;
+    if (tc_band) *tc_band = s.tc_band;
+    return BDL_OK;
+}
+
+// Region table (Fig 4): input-region extent of each layer of layers [first, last] for an output
+// brick of edge `b` along one spatial dim (d = 1..3), interior brick (unclipped).
+bdl_status bdl_region_extents(const bdl_layer *layers, int32_t first, int32_t last, int32_t dim, int32_t b,
+                              int64_t *ext_out) {
+    if (!layers || first < 0 || last < first || dim < 1 || dim > 3 || !ext_out) return fail(BDL_EINVAL, "bad args");
+    std::vector<Layer> ly(last + 1);
+    for (int j = 0; j <= last; j++) ly[j].L = layers[j];
+    std::vector<int64_t> lo, hi;
+    regions_1d(ly, first, last, dim, 0, b, lo, hi);
+    for (int j = 0; j <= last - first; j++) ext_out[j] = hi[j] - lo[j];
+    return BDL_OK;
+}
+
+// rho/tau model exposed for tests (A-2 pins).
+int32_t bdl_model_brick(const bdl_plan_opts *o, int32_t nsp, int64_t N, int64_t D, int64_t H, int64_t W,
+                        int64_t *rho) {
+    bdl_plan_opts d;
+    bdl_plan_opts_default(&d);
+    int ext[4] = {(int)N, (int)D, (int)H, (int)W};
+    return model_brick(o ? *o : d, nsp, ext, rho);
+}
+
+}  // extern "C"

@@ -1,0 +1,118 @@
+// Execution entry points of the C ABI: prepare (weight packing, memo-table reset), run a subgraph,
+// run the whole graph, memo counters.  Host code; every step of the path runs in our kernels.
+#include <cuda_runtime.h>
+
+#include <string>
+#include <vector>
+
+#include "internal.h"
+#include "kernels/common.cuh"
+
+namespace bdl {
+bdl_status launch_pack_f32(const bdl_layer &l, int dtype, float *w_out, float *b_out, cudaStream_t s);
+bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &in, const TView &out,
+                                 const std::vector<TView> &res_views, unsigned char *ws, cudaStream_t s,
+                                 int *launches);
+bdl_status launch_pack_tc(const bdl_layer &l, void *w_out, cudaStream_t s);
+bdl_status launch_tc_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out,
+                              const TView *res, unsigned char *ws, cudaStream_t s, int *launches);
+int tc_launches(const bdl_plan *p, const Subgraph &sg);
+
+static void *tensor_ptr(const bdl_plan *p, int t, const void *in_b, void *out_b, unsigned char *ws) {
+    const Tensor &T = p->tensors[t];
+    if (T.ws_off >= 0) return ws + T.ws_off;
+    if (T.producer == -1) return const_cast<void *>(in_b);
+    return out_b;
+}
+}  // namespace bdl
+
+using namespace bdl;
+
+extern "C" {
+
+bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream) {
+    if (!p) return fail(BDL_EINVAL, "bdl_plan_prepare: plan is NULL");
+    if (!workspace && p->ws_bytes > 0) return fail(BDL_EINVAL, "bdl_plan_prepare: workspace is NULL");
+    if (((uintptr_t)workspace) % 256) return fail(BDL_EINVAL, "bdl_plan_prepare: workspace must be 256-byte aligned");
+    unsigned char *ws = (unsigned char *)workspace;
+    cudaStream_t s = (cudaStream_t)stream;
+    for (auto &L : p->layers) {
+        if (L.L.kind != BDL_OP_CONV) continue;
+        bdl_status st = launch_pack_f32(L.L, p->in_layout.dtype, (float *)(ws + L.w_off), (float *)(ws + L.b_off), s);
+        if (st != BDL_OK) return st;
+        if (L.tc_w_off >= 0) {
+            st = launch_pack_tc(L.L, ws + L.tc_w_off, s);
+            if (st != BDL_OK) return st;
+        }
+    }
+    for (auto &sg : p->sgs) {
+        cudaMemsetAsync(ws + sg.status_off, 0, sg.ntasks_total * 4, s);
+        cudaMemsetAsync(ws + sg.counter_off, 0, 64, s);
+        sg.ticket_base = 0;
+        sg.epoch = 0;
+    }
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return fail(BDL_ECUDA, std::string("bdl_plan_prepare: ") + cudaGetErrorString(e));
+    p->prepared = true;
+    p->prepared_ws = workspace;
+    return BDL_OK;
+}
+
+bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void *out_bricked, void *workspace,
+                            void *stream) {
+    if (!p || i < 0 || i >= (int)p->sgs.size()) return fail(BDL_EINVAL, "bdl_run_subgraph: bad plan or index");
+    if (!p->prepared || p->prepared_ws != workspace)
+        return fail(BDL_EINVAL, "bdl_run_subgraph: call bdl_plan_prepare with this workspace first");
+    if (!in_bricked || !out_bricked) return fail(BDL_EINVAL, "bdl_run_subgraph: NULL tensor");
+    unsigned char *ws = (unsigned char *)workspace;
+    cudaStream_t s = (cudaStream_t)stream;
+    Subgraph &sg = p->sgs[i];
+    sg.epoch++;
+    const Tensor &tin = p->tensors[sg.in_tensor];
+    const Tensor &tout = p->tensors[sg.out_tensor];
+    TView vin = make_view(tin.layout, tensor_ptr(p, sg.in_tensor, in_bricked, out_bricked, ws));
+    TView vout = make_view(tout.layout, tensor_ptr(p, sg.out_tensor, in_bricked, out_bricked, ws));
+    std::vector<TView> res(sg.last - sg.first + 1);
+    const TView *tc_res = nullptr;
+    for (size_t j = 0; j < res.size(); j++) {
+        int t = sg.res_tensor[j];
+        if (t < 0) continue;
+        res[j] = make_view(p->tensors[t].layout, tensor_ptr(p, t, in_bricked, out_bricked, ws));
+        tc_res = &res[j];
+    }
+    int launches = 0;
+    if (sg.kernel == KERNEL_TC_BAND) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
+    return launch_brick_subgraph(p, sg, vin, vout, res, ws, s, &launches);
+}
+
+bdl_status bdl_run(bdl_plan *p, const void *in_bricked, void *out_bricked, void *workspace, void *stream) {
+    if (!p) return fail(BDL_EINVAL, "bdl_run: plan is NULL");
+    for (int i = 0; i < (int)p->sgs.size(); i++) {
+        bdl_status st = bdl_run_subgraph(p, i, in_bricked, out_bricked, workspace, stream);
+        if (st != BDL_OK) return st;
+    }
+    return BDL_OK;
+}
+
+int32_t bdl_plan_launches_per_run(const bdl_plan *p) {
+    if (!p) return 0;
+    int n = 0;
+    for (auto &sg : p->sgs) {
+        int L = sg.last - sg.first + 1;
+        if (sg.kernel == KERNEL_TC_BAND) n += tc_launches(p, sg);
+        else n += (sg.mode == BDL_MODE_UNMERGED || L == 1) ? L : 1;
+    }
+    return n;
+}
+
+bdl_status bdl_plan_counters(const bdl_plan *p, int32_t i, const void *workspace, void *stream, uint64_t out[4]) {
+    if (!p || i < 0 || i >= (int)p->sgs.size() || !workspace || !out) return fail(BDL_EINVAL, "bdl_plan_counters: bad args");
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = cudaMemcpyAsync(out, (const unsigned char *)workspace + p->sgs[i].counter_off, 32,
+                                    cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return fail(BDL_ECUDA, std::string("bdl_plan_counters: ") + cudaGetErrorString(e));
+    return BDL_OK;
+}
+
+}  // extern "C"

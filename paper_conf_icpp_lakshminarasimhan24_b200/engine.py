@@ -1,0 +1,178 @@
+"""High-level Python API over the C ABI: build a plan for a layer graph, own the device workspace,
+brickify -> merged execution -> unbrickify.  PyTorch provides device memory and streams only;
+all computation happens in libbrickdl.so's kernels.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+
+from . import (BDL_BF16, BDL_F32, BDL_MODE_AUTO, BDL_NO_RESIDUAL, BDL_OP_CONV, BDL_OP_MAXPOOL, KERNEL_NAMES,
+               MODE_NAMES, bdl_layer, bdl_layout, bdl_plan_opts, check, lib)
+
+_TORCH_DTYPE = {BDL_F32: torch.float32, BDL_BF16: torch.bfloat16}
+
+
+def make_layout(nsp, N, C, D, H, W, brick, dtype):
+    lo = bdl_layout()
+    Bn, Bd, Bh, Bw = brick
+    check(lib().bdl_layout_init(ctypes.byref(lo), nsp, N, C, D, H, W, Bn, Bd, Bh, Bw, dtype))
+    return lo
+
+
+def default_opts(**kw):
+    o = bdl_plan_opts()
+    lib().bdl_plan_opts_default(ctypes.byref(o))
+    for k, v in kw.items():
+        if k == "bcand":
+            for i, b in enumerate(v):
+                o.bcand[i] = b
+        else:
+            setattr(o, k, v)
+    return o
+
+
+def _stream_handle(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+class Plan:
+    """A partitioned, prepared layer graph (workloads.make_layers format).
+
+    weights: list of float tensors [Co, Ci, kd, kh, kw] (or None for pools); biases: list of [Co].
+    With device=None the plan is built host-only (static analysis without a GPU; run() unavailable).
+    """
+
+    def __init__(self, layers, weights, biases, N, C, D, H, W, nsp, dtype, brick, opts=None,
+                 device="cuda", brickmap=None):
+        self.dtype = BDL_BF16 if dtype in ("bf16", BDL_BF16) else BDL_F32
+        self.tdtype = _TORCH_DTYPE[self.dtype]
+        self.nsp = nsp
+        self.device = device
+        self.in_layout = make_layout(nsp, N, C, D, H, W, brick, self.dtype)
+        self._keep = []
+        if brickmap is not None and device is not None:
+            bm = torch.as_tensor(brickmap, dtype=torch.int32).to(device).contiguous()
+            self._keep.append(bm)
+            self.in_layout.brickmap = bm.data_ptr()
+        arr = (bdl_layer * len(layers))()
+        for i, l in enumerate(layers):
+            a = arr[i]
+            a.kind = BDL_OP_CONV if l["kind"] == "conv" else BDL_OP_MAXPOOL
+            a.cin, a.cout = l["cin"], l["cout"]
+            for d in range(3):
+                a.k[d], a.stride[d], a.pad[d] = l["k"][d], l["stride"][d], l["pad"][d]
+            a.relu = int(l["relu"])
+            a.input = l["input"]
+            a.residual = BDL_NO_RESIDUAL if l["residual"] is None else l["residual"]
+            if a.kind == BDL_OP_CONV:
+                if device is None:
+                    a.w, a.bias = 1, 1   # host-only planning: pointers are not dereferenced
+                else:
+                    w = weights[i].permute(0, 2, 3, 4, 1).contiguous().to(device=device, dtype=self.tdtype)
+                    b = biases[i].to(device=device, dtype=torch.float32).contiguous()
+                    self._keep += [w, b]
+                    a.w, a.bias = w.data_ptr(), b.data_ptr()
+        self._layers = arr
+        self.opts = opts if opts is not None else default_opts()
+        h = ctypes.c_void_p()
+        check(lib().bdl_graph_partition(arr, len(layers), ctypes.byref(self.in_layout), ctypes.byref(self.opts),
+                                        ctypes.byref(h)))
+        self.h = h
+        self.out_layout = bdl_layout()
+        check(lib().bdl_plan_out_layout(h, ctypes.byref(self.out_layout)))
+        self.ws = None
+        if device is not None:
+            nbytes = int(lib().bdl_plan_workspace_bytes(h))
+            self.ws = torch.empty(max(nbytes, 256) + 256, dtype=torch.uint8, device=device)
+            self.ws_ptr = (self.ws.data_ptr() + 255) // 256 * 256
+            self.prepare()
+
+    # ---------------------------------------------------------------- plan introspection
+    def __del__(self):
+        try:
+            if getattr(self, "h", None):
+                lib().bdl_plan_destroy(self.h)
+                self.h = None
+        except Exception:
+            pass
+
+    def prepare(self, stream=None):
+        # (re)packs weights from the staged device copies kept in self._keep
+        check(lib().bdl_plan_prepare(self.h, ctypes.c_void_p(self.ws_ptr), _stream_handle(stream)))
+
+    @property
+    def num_subgraphs(self):
+        return lib().bdl_plan_num_subgraphs(self.h)
+
+    def subgraphs(self):
+        out = []
+        for i in range(self.num_subgraphs):
+            f, la, m, b, k = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+            d = ctypes.c_double()
+            check(lib().bdl_plan_subgraph(self.h, i, ctypes.byref(f), ctypes.byref(la), ctypes.byref(m),
+                                          ctypes.byref(b), ctypes.byref(d), ctypes.byref(k)))
+            df, rho, mm, tb = ctypes.c_double(), ctypes.c_int64(), ctypes.c_int32(), ctypes.c_int32()
+            check(lib().bdl_plan_subgraph_model(self.h, i, ctypes.byref(df), ctypes.byref(rho), ctypes.byref(mm),
+                                                ctypes.byref(tb)))
+            out.append(dict(first=f.value, last=la.value, mode=MODE_NAMES.get(m.value, m.value),
+                            mode_id=m.value, model_brick=b.value, delta=d.value, delta_first=df.value,
+                            rho=rho.value, mode_model=MODE_NAMES.get(mm.value, mm.value),
+                            kernel=KERNEL_NAMES[k.value], tc_band=tb.value))
+        return out
+
+    def set_mode(self, mode, i=None):
+        """mode: 'padded' | 'memoized' | 'unmerged' | 'auto' (all subgraphs, or subgraph i)."""
+        ids = {"auto": 0, "padded": 1, "memoized": 2, "unmerged": 3}
+        m = ids[mode] if isinstance(mode, str) else mode
+        for j in ([i] if i is not None else range(self.num_subgraphs)):
+            check(lib().bdl_plan_set_mode(self.h, j, m))
+        if self.ws is not None:
+            self.prepare()
+
+    @property
+    def launches_per_run(self):
+        return lib().bdl_plan_launches_per_run(self.h)
+
+    # ---------------------------------------------------------------- execution
+    def alloc_bricked(self, layout):
+        return torch.empty(int(layout.total_bytes), dtype=torch.uint8, device=self.device)
+
+    def brickify(self, x, out=None, stream=None):
+        x = x.to(device=self.device, dtype=self.tdtype).contiguous()
+        out = out if out is not None else self.alloc_bricked(self.in_layout)
+        check(lib().bdl_brickify(ctypes.byref(self.in_layout), ctypes.c_void_p(x.data_ptr()),
+                                 ctypes.c_void_p(out.data_ptr()), _stream_handle(stream)))
+        return out
+
+    def unbrickify(self, b, layout=None, out=None, stream=None):
+        layout = layout if layout is not None else self.out_layout
+        shape = (layout.N, layout.C, layout.D, layout.H, layout.W)
+        out = out if out is not None else torch.empty(shape, dtype=self.tdtype, device=self.device)
+        check(lib().bdl_unbrickify(ctypes.byref(layout), ctypes.c_void_p(b.data_ptr()),
+                                   ctypes.c_void_p(out.data_ptr()), _stream_handle(stream)))
+        return out
+
+    def run(self, bricked_in, bricked_out=None, stream=None):
+        bricked_out = bricked_out if bricked_out is not None else self.alloc_bricked(self.out_layout)
+        check(lib().bdl_run(self.h, ctypes.c_void_p(bricked_in.data_ptr()), ctypes.c_void_p(bricked_out.data_ptr()),
+                            ctypes.c_void_p(self.ws_ptr), _stream_handle(stream)))
+        return bricked_out
+
+    def forward(self, x, stream=None):
+        """Dense NC(D)HW -> dense output: brickify, every merged subgraph, unbrickify."""
+        return self.unbrickify(self.run(self.brickify(x, stream=stream), stream=stream), stream=stream)
+
+    def counters(self, i=0, stream=None):
+        arr = (ctypes.c_uint64 * 4)()
+        check(lib().bdl_plan_counters(self.h, i, ctypes.c_void_p(self.ws_ptr), _stream_handle(stream), arr))
+        return dict(computed=arr[0], cas_ok=arr[1], cas_fail=arr[2], spins=arr[3])
+
+
+def plan_from_workload(wl, device="cuda", **opt_kw):
+    """Plan for a workloads.make_workload(...) dict."""
+    opts = default_opts(**opt_kw) if opt_kw else None
+    return Plan(wl["layers"], wl["weights"], wl["biases"], wl["N"], wl["C"], wl["D"], wl["H"], wl["W"],
+                wl["nsp"], wl["dtype"], wl["brick"], opts=opts, device=device)
