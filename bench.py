@@ -1,0 +1,381 @@
+"""Benchmark: merged conv-chain inference throughput (images/s) on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config cfg2] [--mode auto|padded|memoized|unmerged]
+    python bench.py --impl reference ...        # the CPU oracle arm (tier rule: the reference arm is the oracle)
+
+Workload (BASELINE.json configs[1]): ResNet-18 conv2_x basic block, bf16, N=64 per GPU, 56x56x64,
+8x8 bricks; one step = brickify (dense NCHW -> bricks) + every merged subgraph of the plan
+(static-analysis mode choice) + unbrickify, inputs resident in HBM.  L2 is flushed (256 MiB
+write) between timed steps, outside the timed events.  Multi-GPU: one process per GPU (torchrun),
+each rank runs its own 64-image shard ("weak" scaling, no data-path collective); the timed region
+is bracketed by barrier + synchronize, and the time is the max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK_PEAKS = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="native", choices=["native", "reference"])
+    ap.add_argument("--config", default="cfg2")
+    ap.add_argument("--mode", default="auto")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-cudnn", action="store_true")
+    return ap.parse_args()
+
+
+def load_peaks():
+    try:
+        with open(PEAKS_PATH) as f:
+            p = json.load(f)
+        return p, "measured"
+    except Exception:
+        return dict(FALLBACK_PEAKS), "fallback"
+
+
+def workload_desc(wl):
+    return (f"{wl['cfg']}: ResNet-18 conv2_x basic block (conv3x3+b+ReLU -> conv3x3+b, +x, ReLU), "
+            f"N={wl['N']} C={wl['C']} {wl['H']}x{wl['W']}, {wl['brick'][2]}x{wl['brick'][3]} bricks"
+            if wl["cfg"] == "cfg2" else f"{wl['cfg']} N={wl['N']} C={wl['C']} D={wl['D']} H={wl['H']} W={wl['W']}")
+
+
+def useful_flops(wl):
+    """2*MACs of plain layer-by-layer execution (padded-mode recompute not credited)."""
+    from paper_conf_icpp_lakshminarasimhan24_b200 import workloads
+    f = 0
+    D, H, W = wl["D"], wl["H"], wl["W"]
+    for l in wl["layers"]:
+        Do, Ho, Wo = workloads.layer_out_shape(l, D, H, W)
+        if l["kind"] == "conv":
+            kd, kh, kw = l["k"]
+            f += 2 * wl["N"] * Do * Ho * Wo * l["cout"] * l["cin"] * kd * kh * kw
+        D, H, W = Do, Ho, Wo
+    return f
+
+
+# ------------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index=0):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 8:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for nm, v in zip(names, r[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+# ------------------------------------------------------------------------------------------ oracle arms
+def oracle_images_per_s(wl, n_images, threads):
+    import oracle
+    os.environ["OMP_NUM_THREADS"] = str(threads)
+    x = wl["x"].numpy()[:n_images]
+    t = time.perf_counter()
+    oracle.run_graph(wl["layers"], x, wl["weights"], wl["biases"], dtype=wl["dtype"])
+    return n_images / (time.perf_counter() - t)
+
+
+def cpu_baseline(wl, budget_s=12.0):
+    """The oracle as it stands, on this host's cores, on a bounded sample of the same workload."""
+    import oracle
+    threads = os.cpu_count() or 1
+    os.environ["OMP_NUM_THREADS"] = str(threads)
+    oracle.lib()
+    x = wl["x"].numpy()
+    t = time.perf_counter()
+    oracle.run_graph(wl["layers"], x[:1], wl["weights"], wl["biases"], dtype=wl["dtype"])
+    t1 = time.perf_counter() - t
+    n = int(max(1, min(wl["N"], budget_s / max(t1, 1e-3))))
+    ips = oracle_images_per_s(wl, n, threads)
+    return {"value": ips, "unit": "images/s", "cores": threads, "kind": "oracle",
+            "sample": f"{n} of {wl['N']} images of the same workload, fp64 direct conv, OpenMP {threads} threads"}
+
+
+def run_reference(args):
+    from paper_conf_icpp_lakshminarasimhan24_b200 import workloads
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    wl = workloads.make_workload(args.config)
+    import oracle
+    threads = os.cpu_count() or 1
+    os.environ["OMP_NUM_THREADS"] = str(threads)
+    oracle.lib()
+    per_step = 4  # images per step: a bounded sample of the workload
+    x = wl["x"].numpy()
+    for _ in range(args.warmup):
+        oracle.run_graph(wl["layers"], x[:per_step], wl["weights"], wl["biases"], dtype=wl["dtype"])
+    t = time.perf_counter()
+    for s in range(args.steps):
+        i0 = (s * per_step) % wl["N"]
+        oracle.run_graph(wl["layers"], x[i0:i0 + per_step], wl["weights"], wl["biases"], dtype=wl["dtype"])
+    dt = time.perf_counter() - t
+    v = per_step * args.steps / dt
+    line = {"impl": "reference", "metric": "images/sec merged conv chain per B200", "value": v, "unit": "images/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": workload_desc(wl), "sample_per_step": f"{per_step} of {wl['N']} images"},
+            "cpu_baseline": {"value": v, "unit": "images/s", "cores": threads, "kind": "oracle",
+                             "sample": f"{per_step} images per step x {args.steps} steps"},
+            "e2e": {"value": v, "unit": "images/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+# ------------------------------------------------------------------------------------------ native arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_lakshminarasimhan24_b200 import engine, workloads
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    wl = workloads.make_workload(args.config, input_seed_offset=rank)
+    plan = engine.plan_from_workload(wl, device=dev)
+    if args.mode != "auto":
+        plan.set_mode(args.mode)
+    sg = plan.subgraphs()
+    stream = torch.cuda.current_stream(dev)
+
+    x_dense = wl["x"].to(device=dev, dtype=plan.tdtype).contiguous()
+    xb = plan.alloc_bricked(plan.in_layout)
+    yb = plan.alloc_bricked(plan.out_layout)
+    y_dense = torch.empty((plan.out_layout.N, plan.out_layout.C, plan.out_layout.D, plan.out_layout.H,
+                           plan.out_layout.W), dtype=plan.tdtype, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def step():
+        plan.brickify(x_dense, out=xb)
+        plan.run(xb, yb)
+        plan.unbrickify(yb, out=y_dense)
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+
+    K = args.steps
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(K)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for k in range(K):
+            flush.zero_()                      # L2 flush, outside the timed events
+            e = ev[k]
+            e[0].record(stream)
+            plan.brickify(x_dense, out=xb)
+            e[1].record(stream)
+            plan.run(xb, yb)
+            e[2].record(stream)
+            plan.unbrickify(yb, out=y_dense)
+            e[3].record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    step_ms = [e[0].elapsed_time(e[3]) for e in ev]
+    run_ms = [e[1].elapsed_time(e[2]) for e in ev]
+    total_ms = sum(step_ms)
+    t_local = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t_local, op=dist.ReduceOp.MAX)
+    total_ms = float(t_local.item())
+    images = wl["N"] * world * K
+    value = images / (total_ms / 1e3)
+
+    # ---- end to end through the public API: pinned host input -> device -> ... -> pinned host output
+    x_host = wl["x"].to(plan.tdtype).contiguous().pin_memory()
+    y_host = torch.empty(y_dense.shape, dtype=plan.tdtype).pin_memory()
+    x_dev2 = torch.empty_like(x_dense)
+    for _ in range(3):
+        x_dev2.copy_(x_host, non_blocking=True)
+        plan.unbrickify(plan.run(plan.brickify(x_dev2, out=xb), yb), out=y_dense)
+        y_host.copy_(y_dense, non_blocking=True)
+    torch.cuda.synchronize()
+    e2e_ms = 0.0
+    for k in range(K):
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        x_dev2.copy_(x_host, non_blocking=True)
+        plan.brickify(x_dev2, out=xb)
+        plan.run(xb, yb)
+        plan.unbrickify(yb, out=y_dense)
+        y_host.copy_(y_dense, non_blocking=True)
+        b.record(stream)
+        b.synchronize()
+        e2e_ms += a.elapsed_time(b)
+    t2 = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t2, op=dist.ReduceOp.MAX)
+    e2e_value = images / (float(t2.item()) / 1e3)
+
+    # ---- roofline of the dominant kernel (the merged subgraph launch)
+    peaks, peak_src = load_peaks()
+    flops = useful_flops(wl)
+    kernel_ms = statistics.mean(run_ms)
+    achieved = flops / (kernel_ms / 1e3) / 1e12
+    peak = float(peaks["bf16_tflops"])
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_summary_latest.json")
+    if os.path.exists(tp):
+        try:
+            with open(tp) as f:
+                traffic = json.load(f).get("dram_bytes_per_launch", {}).get(sg[0]["kernel"])
+        except Exception:
+            traffic = None
+    roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                "traffic": traffic, "peak_source": f"{peak_src} bf16_tflops (burst, cuBLAS 8192^3)",
+                "kernel": f"{sg[0]['kernel']} ({sg[0]['mode']})", "algorithmic_flops_per_launch": flops,
+                "kernel_ms_mean": kernel_ms, "hbm_frac_of_step_bytes": None}
+    # step bytes: brickify (read+write) + merged subgraph (in, out, weights) + unbrickify (read+write)
+    act = wl["N"] * wl["C"] * wl["H"] * wl["W"] * 2
+    step_bytes = 2 * act + 2 * act + 2 * act
+    roofline["hbm_frac_of_step_bytes"] = step_bytes / (statistics.mean(step_ms) / 1e3) / 1e9 / float(peaks["hbm_gbs"])
+
+    # ---- layer-by-layer cuDNN reference (context): torch conv2d, channels_last bf16
+    cudnn = None
+    if not args.no_cudnn and rank == 0:
+        cudnn = cudnn_lbl(wl, dev, K, flush)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(wl)
+
+    if rank == 0:
+        launches = K * (2 + plan.launches_per_run)
+        line = {
+            "metric": "images/sec merged conv chain per B200", "value": value, "unit": "images/s",
+            "n_gpus": world, "steps": K, "warmup": max(3, args.warmup), "ms_per_step": total_ms / K,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
+            "data": "synthetic (seeded N(0,1) inputs, He-normal weights; workloads.py)",
+            "config": {"workload": workload_desc(wl), "images_per_gpu": wl["N"], "global_batch": wl["N"] * world,
+                       "mode": sg[0]["mode"], "mode_model": sg[0]["mode_model"], "delta": round(sg[0]["delta"], 4),
+                       "kernel": sg[0]["kernel"], "step": "brickify + merged subgraph + unbrickify",
+                       "l2": "flushed between timed steps (256 MiB write outside the events)",
+                       "parallelism": f"batch-sharded x{world}, no data-path collective"},
+            "clocks": clk.summary(),
+            "e2e": {"value": e2e_value, "unit": "images/s", "h2d_bytes_per_step": x_host.numel() * x_host.element_size(),
+                    "d2h_bytes_per_step": y_host.numel() * y_host.element_size()},
+            "gpu_launches": launches,
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "breakdown_ms": {"brickify": statistics.mean(e[0].elapsed_time(e[1]) for e in ev),
+                             "merged_subgraph": kernel_ms,
+                             "unbrickify": statistics.mean(e[2].elapsed_time(e[3]) for e in ev)},
+            "cudnn_layer_by_layer": cudnn,
+        }
+        print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def cudnn_lbl(wl, dev, K, flush):
+    """Layer-by-layer torch/cuDNN run of the same graph (context only, not our product)."""
+    import torch
+    import torch.nn.functional as F
+    try:
+        x = wl["x"][:, :, 0].to(device=dev, dtype=torch.bfloat16).contiguous(memory_format=torch.channels_last)
+        ws = [w[:, :, 0].to(device=dev, dtype=torch.bfloat16).contiguous(memory_format=torch.channels_last)
+              for w in wl["weights"]]
+        bs = [b.to(device=dev, dtype=torch.bfloat16) for b in wl["biases"]]
+
+        def fwd():
+            outs = []
+            for l, w, b in zip(wl["layers"], ws, bs):
+                src = x if l["input"] == -1 else outs[l["input"]]
+                y = F.conv2d(src, w, b, stride=l["stride"][1:], padding=l["pad"][1:])
+                if l["residual"] is not None:
+                    y = y + (x if l["residual"] == -1 else outs[l["residual"]])
+                if l["relu"]:
+                    y = torch.relu(y)
+                outs.append(y)
+            return outs[-1]
+        with torch.no_grad():
+            for _ in range(5):
+                fwd()
+            torch.cuda.synchronize()
+            tot = 0.0
+            for _ in range(K):
+                flush.zero_()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record()
+                fwd()
+                b.record()
+                b.synchronize()
+                tot += a.elapsed_time(b)
+        return {"ms_per_step": tot / K, "images_per_s": wl["N"] * K / (tot / 1e3),
+                "what": "torch conv2d (cuDNN) bf16 channels_last, separate add/ReLU, dense NHWC in/out"}
+    except Exception as e:  # context measurement only
+        return {"error": str(e)[:200]}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

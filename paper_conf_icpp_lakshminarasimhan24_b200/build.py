@@ -23,6 +23,7 @@ SOURCES = [
     "kernels/brickify.cu",
     "kernels/chain_brick.cu",
     "kernels/chain_tc.cu",
+    "kernels/chain_tc_ws.cu",
 ]
 FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",

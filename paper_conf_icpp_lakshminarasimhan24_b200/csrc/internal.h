@@ -78,6 +78,10 @@ struct Subgraph {
     int tc_band = 0;               // band rows
     int tc_smem = 0;
     std::vector<int64_t> tc_inter_off;
+    // warp-specialized memo kernel: locality-aware task order (uploaded at prepare)
+    int64_t order_off = -1;
+    int64_t norder = 0;
+    std::vector<int> order_host;
 };
 
 }  // namespace bdl

@@ -21,6 +21,7 @@
 //   unmerged : one launch per layer over all tiles (the memo kernel with dependency checks off).
 // Epilogue order: + bias -> + residual -> ReLU -> bf16 RNE.
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -28,6 +29,8 @@
 #include "tc_ptx.cuh"
 
 namespace bdl {
+
+static unsigned long long *trace_buf = nullptr;  // debug task trace (BDL_TRACE=<capacity>)
 
 constexpr int kNS = 3;          // weight ring stages (one tap each)
 constexpr int kTcThreads = 128; // 4 warps: warp w owns TMEM lanes [32w, 32w+32)
@@ -57,7 +60,20 @@ struct TcParams {
     unsigned long long ticket_base;
     long long ntiles;              // tiles per layer = N * nty * ntx
     int only_layer;                // >= 0: unmerged launch of that layer
+    unsigned long long *trace;     // debug: per task [smid|l, tile, t0..t4] (globaltimer ns), or null
+    int trace_cap;
 };
+
+__device__ __forceinline__ unsigned long long gtime() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ unsigned smid() {
+    unsigned r;
+    asm volatile("mov.u32 %0, %smid;" : "=r"(r));
+    return r;
+}
 
 struct TcShared {   // static shared state
     uint64_t full[kNS], empty[kNS], mma_done;
@@ -344,6 +360,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) tc_memo_kernel(const __grid_con
         __syncthreads();
         if (sh.task >= p.ntiles) break;
         for (;;) {
+            unsigned long long t0 = gtime();
             if (threadIdx.x == 0) {
                 sh.cmd_l = -1;
                 unsigned long long spins = 0, fails = 0, oks = 0;
@@ -392,17 +409,30 @@ __global__ void __launch_bounds__(kTcThreads, 1) tc_memo_kernel(const __grid_con
             decode_tile(p, tt, n, ty, tx);
             const int y0 = ty * p.Tb, x0 = tx * p.Tw;
             const TView &src = l == 0 ? p.in : p.layer[l - 1].out;
+            unsigned long long t1 = gtime();
             load_tile<C>(src, n, y0 - 1, x0 - 1, p.Tb + 2, p.Wt, bufA, p.rowsA);
             ptx::tc_fence_before();
             __syncthreads();
             ptx::tc_fence_after();
+            unsigned long long t2 = gtime();
             if (threadIdx.x == 0) issue_layer<C>(p, sh, p.layer[l].w, bufA, p.rowsA, ntl, wst, wq);
             ptx::mbar_wait(&sh.mma_done, done_phase);
             done_phase ^= 1;
             ptx::tc_fence_after();
+            unsigned long long t3 = gtime();
             epilogue_global<C>(p, sh, p.layer[l], ntl, n, y0, x0, p.layer[l].res);
             ptx::tc_fence_before();
             __syncthreads();
+            if (threadIdx.x == 0 && p.trace) {
+                unsigned long long t4 = gtime();
+                unsigned long long k = atomicAdd(&p.counters[5], 1ULL);
+                if (k < (unsigned long long)p.trace_cap) {
+                    unsigned long long *r = p.trace + k * 7;
+                    r[0] = ((unsigned long long)smid() << 32) | ((unsigned)blockIdx.x << 8) | (unsigned)l;
+                    r[1] = (unsigned long long)tt;
+                    r[2] = t0; r[3] = t1; r[4] = t2; r[5] = t3; r[6] = t4;
+                }
+            }
             if (threadIdx.x == 0) {
                 if (!unmerged) {
                     __threadfence();
@@ -581,6 +611,14 @@ bdl_status launch_tc_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
     P.epoch = sg.epoch;
     P.counters = (unsigned long long *)(ws + sg.counter_off);
     P.ntiles = (long long)P.N * P.nty * P.ntx;
+    {
+        const char *e = getenv("BDL_TRACE");
+        if (e && atoi(e) > 0) {
+            P.trace_cap = atoi(e);
+            if (!trace_buf) cudaMalloc(&trace_buf, (size_t)P.trace_cap * 7 * 8);
+            P.trace = trace_buf;
+        }
+    }
     switch (P.C) {
         case 16: return launch_tc_C<16>(p, sg, P, g, mode, s, launches);
         case 32: return launch_tc_C<32>(p, sg, P, g, mode, s, launches);
@@ -591,3 +629,11 @@ bdl_status launch_tc_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
 }
 
 }  // namespace bdl
+
+// Debug: copy the task trace (7 x u64 per task) to host; returns records copied.
+extern "C" int bdl_debug_trace_copy(unsigned long long *host, int max_records) {
+    if (!bdl::trace_buf || max_records <= 0) return 0;
+    cudaDeviceSynchronize();
+    cudaMemcpy(host, bdl::trace_buf, (size_t)max_records * 7 * 8, cudaMemcpyDeviceToHost);
+    return max_records;
+}

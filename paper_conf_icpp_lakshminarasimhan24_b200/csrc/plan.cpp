@@ -116,6 +116,7 @@ static bool is_pool(const Layer &l) { return l.L.kind == BDL_OP_MAXPOOL; }
 
 namespace bdl {
 int tc_band_rows(const bdl_plan *p, const Subgraph &sg, int *smem_out);
+std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg);
 }
 using namespace bdl;
 
@@ -405,7 +406,12 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
         sg.grid = 4 * p->num_sms;
         sg.scratch_slot_floats = align_up(maxvol, 64);
         sg.scratch_off = L > 1 ? take((int64_t)sg.grid * 2 * sg.scratch_slot_floats * 4) : -1;
-        if (sg.kernel == KERNEL_TC_BAND) sg.tc_band = tc_band_rows(p, sg, &sg.tc_smem);
+        if (sg.kernel == KERNEL_TC_BAND) {
+            sg.tc_band = tc_band_rows(p, sg, &sg.tc_smem);
+            sg.order_host = ws_task_order(p, sg);
+            sg.norder = (int64_t)sg.order_host.size();
+            sg.order_off = sg.norder ? take(sg.norder * 4) : -1;
+        }
     }
     p->ws_bytes = align_up(off, 256);
     *out = p;

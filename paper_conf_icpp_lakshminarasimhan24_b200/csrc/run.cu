@@ -2,6 +2,7 @@
 // run the whole graph, memo counters.  Host code; every step of the path runs in our kernels.
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <string>
 #include <vector>
 
@@ -16,6 +17,8 @@ bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &i
 bdl_status launch_pack_tc(const bdl_layer &l, void *w_out, cudaStream_t s);
 bdl_status launch_tc_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out,
                               const TView *res, unsigned char *ws, cudaStream_t s, int *launches);
+bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out, const TView *res,
+                              unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged);
 int tc_launches(const bdl_plan *p, const Subgraph &sg);
 
 static void *tensor_ptr(const bdl_plan *p, int t, const void *in_b, void *out_b, unsigned char *ws) {
@@ -46,6 +49,8 @@ bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream) {
         }
     }
     for (auto &sg : p->sgs) {
+        if (sg.order_off >= 0)
+            cudaMemcpyAsync(ws + sg.order_off, sg.order_host.data(), sg.norder * 4, cudaMemcpyHostToDevice, s);
         cudaMemsetAsync(ws + sg.status_off, 0, sg.ntasks_total * 4, s);
         cudaMemsetAsync(ws + sg.counter_off, 0, 64, s);
         sg.ticket_base = 0;
@@ -81,7 +86,14 @@ bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void
         tc_res = &res[j];
     }
     int launches = 0;
-    if (sg.kernel == KERNEL_TC_BAND) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
+    if (sg.kernel == KERNEL_TC_BAND) {
+        const bool single = sg.first == sg.last;
+        if (sg.mode == BDL_MODE_PADDED && !single) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
+        static const bool legacy = getenv("BDL_TC_LEGACY") != nullptr;  // A/B against the synchronous kernel
+        if (legacy) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
+        return launch_ws_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches,
+                                  sg.mode == BDL_MODE_UNMERGED || single);
+    }
     return launch_brick_subgraph(p, sg, vin, vout, res, ws, s, &launches);
 }
 

@@ -113,7 +113,8 @@ def layer_out_shape(layer, D, H, W):
     return tuple(out)
 
 
-def make_workload(cfg: str, N=None, C=None, D=None, H=None, W=None, nlayers=None, seed_offset=0):
+def make_workload(cfg: str, N=None, C=None, D=None, H=None, W=None, nlayers=None, seed_offset=0,
+                  input_seed_offset=0):
     """Seeded synthetic input, weights and biases for a configuration (optionally resized).
 
     Returns dict(cfg, nsp, dtype, N, C, D, H, W, brick, layers, x, weights, biases) where
@@ -129,7 +130,7 @@ def make_workload(cfg: str, N=None, C=None, D=None, H=None, W=None, nlayers=None
     layers = make_layers(cfg, C=c["C"], nlayers=nlayers)
     bf16 = c["dtype"] == "bf16"
 
-    g = torch.Generator().manual_seed(1000 + num)
+    g = torch.Generator().manual_seed(1000 + num + 100 * input_seed_offset)  # per-shard inputs (ranks)
     x = torch.randn(c["N"], c["C"], c["D"], c["H"], c["W"], generator=g, dtype=torch.float32)
     if bf16:
         x = x.to(torch.bfloat16).to(torch.float32)
