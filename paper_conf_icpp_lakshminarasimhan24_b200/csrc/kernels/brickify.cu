@@ -1,12 +1,12 @@
 // Brick creation ("the cost of creating bricks, which is minimal") and its inverse.
 // NC(D)HW dense  <->  bricked [phys][Bn][Bd][Bh][Bw][Cp] (include/brickdl.h).
 //
-// HBM-bound transposes.  One CTA owns a (sample n, brick-row bd/bh, channel group) tile spanning the
-// full width W, staged in shared memory as [pixel][CGP] (channels innermost, CGP = CG + 1 elements):
-//   dense side : every warp moves whole rows of one channel plane with 16-byte vectors (coalesced);
-//   brick side : lanes walk the 16-byte channel vectors of consecutive pixels, so a warp writes or
-//                reads 512 contiguous bytes of a brick per instruction.
-// Index arithmetic is per 16-byte vector, never per element.
+// HBM-bound transposes without shared memory.  A thread owns a V x V block (V = 16 B / element: 8 bf16
+// or 4 fp32): V channels x V consecutive pixels of one row.  It loads V 16-byte row vectors (one per
+// channel) from the dense tensor, transposes the block in registers, and stores V 16-byte channel
+// vectors (one per pixel) into the bricks -- and the reverse for unbrickify.  Lanes are ordered with
+// the channel group fastest, so a warp's brick-side accesses are whole 128-byte pixel rows (C = 64
+// bf16) and its dense-side accesses are 64-byte runs of each channel plane.
 #include <algorithm>
 #include <string>
 
@@ -14,161 +14,110 @@
 
 namespace bdl {
 
-struct ConvGeom {
-    int CG, CGP, G;        // channels per tile, padded stride (elements), 16-B vectors per pixel
-    int ngroups;
-    int rows;              // Bd * Bh
-    int Wfull;             // nb[3] * Bw
-    int vec_ok;            // dense rows are 16-byte aligned (W * elem % 16 == 0)
+template <typename T>
+struct Vec {
+    static constexpr int V = 16 / sizeof(T);
+    union {
+        uint4 u;
+        T e[V];
+    };
 };
+
+struct ConvGeom {
+    int G;         // channel groups (Cp / V)
+    int XG;        // pixel groups per brick-grid row (ceil((nb3*Bw) / V))
+    int rows;      // rows of the brick grid: nb0*Bn (samples, padded) x nb1*Bd x nb2*Bh
+    int vec_ok;    // dense rows are 16-byte aligned and W % V == 0
+};
+
+// Element offset of the channel-0 slot of pixel (n, d, h, w) in the bricked tensor.
+__device__ __forceinline__ long long brick_px(const TView &v, int n, int d, int h, int w) {
+    const int bn = n / v.B[0], bd = d / v.B[1], bh = h / v.B[2], bw = w / v.B[3];
+    const long long logical = (((long long)bn * v.nb[1] + bd) * v.nb[2] + bh) * v.nb[3] + bw;
+    const int inner = (((n - bn * v.B[0]) * v.B[1] + (d - bd * v.B[1])) * v.B[2] + (h - bh * v.B[2])) * v.B[3] + (w - bw * v.B[3]);
+    return tv_phys(v, logical) * v.brick_elems + (long long)inner * v.Cp;
+}
 
 template <typename T>
 __global__ void __launch_bounds__(256) brickify_kernel(TView v, const T *__restrict__ src, ConvGeom cg) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    T *tile = reinterpret_cast<T *>(smem_raw);
-    constexpr int V = 16 / sizeof(T);
-    const int g = blockIdx.x % cg.ngroups;
-    int rest = blockIdx.x / cg.ngroups;
-    const int bh = rest % v.nb[2];
-    rest /= v.nb[2];
-    const int bd = rest % v.nb[1];
-    const int n = rest / v.nb[1];  // 0 .. nb[0]*Bn - 1
-    const int Bd = v.B[1], Bh = v.B[2], W = v.ext[3], Wfull = cg.Wfull;
-    const int c0 = g * cg.CG;
-    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32, nwarps = blockDim.x / 32;
-    const long long plane = (long long)v.ext[1] * v.ext[2] * W;
-    // ---- phase 1: dense rows (channel c, depth z, row y) -> tile[pixel][c]; 4 vectors in flight/thread
-    const int nrows = cg.CG * cg.rows;
-    if (cg.vec_ok) {
-        const int nvec = (Wfull + V - 1) / V;
-        const int total = nrows * nvec;
-        for (int i0 = threadIdx.x; i0 < total; i0 += 4 * blockDim.x) {
-            uint4 u[4];
-            int row_i[4], x_i[4];
-#pragma unroll
-            for (int q = 0; q < 4; q++) {
-                const int i = i0 + q * blockDim.x;
-                row_i[q] = -1;
-                u[q] = make_uint4(0, 0, 0, 0);
-                if (i < total) {
-                    const int r = i / nvec, x0 = (i - r * nvec) * V;
-                    const int c = r / cg.rows, zy = r - c * cg.rows;
-                    const int z = zy / Bh, y = zy - z * Bh;
-                    const int d = bd * Bd + z, h = bh * Bh + y, cc = c0 + c;
-                    row_i[q] = r;
-                    x_i[q] = x0;
-                    if (n < v.ext[0] && cc < v.C && d < v.ext[1] && h < v.ext[2] && x0 < W)
-                        u[q] = __ldg(reinterpret_cast<const uint4 *>(src + ((long long)n * v.C + cc) * plane +
-                                                                     ((long long)d * v.ext[2] + h) * W + x0));
-                }
-            }
-#pragma unroll
-            for (int q = 0; q < 4; q++) {
-                if (row_i[q] < 0) continue;
-                const int r = row_i[q], c = r / cg.rows, zy = r - c * cg.rows;
-                T *trow = tile + (size_t)zy * Wfull * cg.CGP + c;
-                const T *e = reinterpret_cast<const T *>(&u[q]);
-#pragma unroll
-                for (int k = 0; k < V; k++)
-                    if (x_i[q] + k < Wfull) trow[(size_t)(x_i[q] + k) * cg.CGP] = e[k];
-            }
-        }
-    } else {
-        for (int r = warp; r < nrows; r += nwarps) {
-            const int c = r / cg.rows, zy = r - c * cg.rows;
-            const int z = zy / Bh, y = zy - z * Bh;
-            const int d = bd * Bd + z, h = bh * Bh + y, cc = c0 + c;
-            const bool rok = n < v.ext[0] && cc < v.C && d < v.ext[1] && h < v.ext[2];
-            const T *row = src + ((long long)n * v.C + cc) * plane + ((long long)d * v.ext[2] + h) * W;
-            T *trow = tile + (size_t)zy * Wfull * cg.CGP + c;
-            for (int x = lane; x < Wfull; x += 32) trow[(size_t)x * cg.CGP] = (rok && x < W) ? row[x] : from_f<T>(0.f);
-        }
-    }
-    __syncthreads();
-    // ---- phase 2: brick pixels, 16-byte channel vectors, lanes fastest over the vectors of a pixel
+    constexpr int V = Vec<T>::V;
+    const long long units = (long long)cg.rows * cg.XG * cg.G;
+    const int Dg = v.nb[1] * v.B[1], Hg = v.nb[2] * v.B[2], Wg = v.nb[3] * v.B[3];
+    const long long plane = (long long)v.ext[1] * v.ext[2] * v.ext[3];
     T *dst = reinterpret_cast<T *>(v.ptr);
-    const int bn = n / v.B[0], nin = n - bn * v.B[0];
-    const int npix = cg.rows * Wfull;
-    const int gv = cg.CG / V;  // vectors of this group per pixel
-    for (int i = threadIdx.x; i < npix * gv; i += blockDim.x) {
-        const int q = i % gv, p = i / gv;
-        const int zy = p / Wfull, x = p - zy * Wfull;
-        const int z = zy / Bh, y = zy - z * Bh;
-        const int bw = x / v.B[3], xi = x - bw * v.B[3];
-        const long long logical = (((long long)bn * v.nb[1] + bd) * v.nb[2] + bh) * v.nb[3] + bw;
-        const int inner = ((nin * Bd + z) * Bh + y) * v.B[3] + xi;
-        const T *s = tile + (size_t)p * cg.CGP + q * V;
-        union { uint4 u; T e[V]; } pk;
+    for (long long u = blockIdx.x * (long long)blockDim.x + threadIdx.x; u < units; u += (long long)gridDim.x * blockDim.x) {
+        const int g = (int)(u % cg.G);
+        long long r = u / cg.G;
+        const int xg = (int)(r % cg.XG);
+        r /= cg.XG;
+        const int h = (int)(r % Hg);
+        r /= Hg;
+        const int d = (int)(r % Dg);
+        const int n = (int)(r / Dg);
+        const int x0 = xg * V, c0 = g * V;
+        const bool row_ok = n < v.ext[0] && d < v.ext[1] && h < v.ext[2];
+        Vec<T> in[V];
 #pragma unroll
-        for (int e = 0; e < V; e++) pk.e[e] = s[e];
-        *reinterpret_cast<uint4 *>(dst + tv_phys(v, logical) * v.brick_elems + (long long)inner * v.Cp + c0 + q * V) = pk.u;
+        for (int k = 0; k < V; k++) {
+            const int c = c0 + k;
+            const T *row = src + ((long long)n * v.C + c) * plane + ((long long)d * v.ext[2] + h) * v.ext[3];
+            if (cg.vec_ok) {
+                in[k].u = (row_ok && c < v.C && x0 < v.ext[3]) ? __ldg(reinterpret_cast<const uint4 *>(row + x0))
+                                                              : make_uint4(0, 0, 0, 0);
+            } else {
+#pragma unroll
+                for (int i = 0; i < V; i++)
+                    in[k].e[i] = (row_ok && c < v.C && x0 + i < v.ext[3]) ? row[x0 + i] : from_f<T>(0.f);
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < V; i++) {
+            if (x0 + i >= Wg) break;
+            Vec<T> o;
+#pragma unroll
+            for (int k = 0; k < V; k++) o.e[k] = in[k].e[i];
+            *reinterpret_cast<uint4 *>(dst + brick_px(v, n, d, h, x0 + i) + c0) = o.u;
+        }
     }
 }
 
 template <typename T>
 __global__ void __launch_bounds__(256) unbrickify_kernel(TView v, T *__restrict__ dstd, ConvGeom cg) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    T *tile = reinterpret_cast<T *>(smem_raw);
-    constexpr int V = 16 / sizeof(T);
-    const int g = blockIdx.x % cg.ngroups;
-    int rest = blockIdx.x / cg.ngroups;
-    const int bh = rest % v.nb[2];
-    rest /= v.nb[2];
-    const int bd = rest % v.nb[1];
-    const int n = rest / v.nb[1];
-    if (n >= v.ext[0]) return;
-    const int Bd = v.B[1], Bh = v.B[2], W = v.ext[3], Wfull = cg.Wfull;
-    const int c0 = g * cg.CG;
+    constexpr int V = Vec<T>::V;
+    const int XGd = (v.ext[3] + V - 1) / V;
+    const long long units = (long long)v.ext[0] * v.ext[1] * v.ext[2] * XGd * cg.G;
+    const long long plane = (long long)v.ext[1] * v.ext[2] * v.ext[3];
     const T *src = reinterpret_cast<const T *>(v.ptr);
-    const int bn = n / v.B[0], nin = n - bn * v.B[0];
-    const int npix = cg.rows * Wfull;
-    const int gv = cg.CG / V;
-    const int total = npix * gv;
-    for (int i0 = threadIdx.x; i0 < total; i0 += 4 * blockDim.x) {
-        uint4 u[4];
+    for (long long u = blockIdx.x * (long long)blockDim.x + threadIdx.x; u < units; u += (long long)gridDim.x * blockDim.x) {
+        const int g = (int)(u % cg.G);
+        long long r = u / cg.G;
+        const int xg = (int)(r % XGd);
+        r /= XGd;
+        const int h = (int)(r % v.ext[2]);
+        r /= v.ext[2];
+        const int d = (int)(r % v.ext[1]);
+        const int n = (int)(r / v.ext[1]);
+        const int x0 = xg * V, c0 = g * V;
+        Vec<T> in[V];
 #pragma unroll
-        for (int j = 0; j < 4; j++) {
-            const int i = i0 + j * blockDim.x;
-            if (i >= total) continue;
-            const int q = i % gv, p = i / gv;
-            const int zy = p / Wfull, x = p - zy * Wfull;
-            const int z = zy / Bh, y = zy - z * Bh;
-            const int bw = x / v.B[3], xi = x - bw * v.B[3];
-            const long long logical = (((long long)bn * v.nb[1] + bd) * v.nb[2] + bh) * v.nb[3] + bw;
-            const int inner = ((nin * Bd + z) * Bh + y) * v.B[3] + xi;
-            u[j] = __ldg(reinterpret_cast<const uint4 *>(src + tv_phys(v, logical) * v.brick_elems + (long long)inner * v.Cp + c0 + q * V));
-        }
+        for (int i = 0; i < V; i++)
+            in[i].u = (x0 + i < v.ext[3]) ? __ldg(reinterpret_cast<const uint4 *>(src + brick_px(v, n, d, h, x0 + i) + c0))
+                                          : make_uint4(0, 0, 0, 0);
 #pragma unroll
-        for (int j = 0; j < 4; j++) {
-            const int i = i0 + j * blockDim.x;
-            if (i >= total) continue;
-            const int q = i % gv, p = i / gv;
-            const T *e = reinterpret_cast<const T *>(&u[j]);
-            T *s = tile + (size_t)p * cg.CGP + q * V;
+        for (int k = 0; k < V; k++) {
+            const int c = c0 + k;
+            if (c >= v.C) break;
+            T *row = dstd + ((long long)n * v.C + c) * plane + ((long long)d * v.ext[2] + h) * v.ext[3];
+            Vec<T> o;
 #pragma unroll
-            for (int k = 0; k < V; k++) s[k] = e[k];
-        }
-    }
-    __syncthreads();
-    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32, nwarps = blockDim.x / 32;
-    const long long plane = (long long)v.ext[1] * v.ext[2] * W;
-    const int nrows = cg.CG * cg.rows;
-    for (int r = warp; r < nrows; r += nwarps) {
-        const int c = r / cg.rows, zy = r - c * cg.rows;
-        const int z = zy / Bh, y = zy - z * Bh;
-        const int d = bd * Bd + z, h = bh * Bh + y, cc = c0 + c;
-        if (cc >= v.C || d >= v.ext[1] || h >= v.ext[2]) continue;
-        T *row = dstd + ((long long)n * v.C + cc) * plane + ((long long)d * v.ext[2] + h) * W;
-        const T *trow = tile + (size_t)zy * Wfull * cg.CGP + c;
-        if (cg.vec_ok) {
-            for (int x0 = lane * V; x0 < W; x0 += 32 * V) {
-                union { uint4 u; T e[V]; } pk;
+            for (int i = 0; i < V; i++) o.e[i] = in[i].e[k];
+            if (cg.vec_ok) {
+                *reinterpret_cast<uint4 *>(row + x0) = o.u;
+            } else {
 #pragma unroll
-                for (int i = 0; i < V; i++) pk.e[i] = trow[(size_t)(x0 + i) * cg.CGP];
-                *reinterpret_cast<uint4 *>(row + x0) = pk.u;
+                for (int i = 0; i < V; i++)
+                    if (x0 + i < v.ext[3]) row[x0 + i] = o.e[i];
             }
-        } else {
-            for (int x = lane; x < W; x += 32) row[x] = trow[(size_t)x * cg.CGP];
         }
     }
 }
@@ -178,43 +127,22 @@ static bdl_status launch_convert(const bdl_layout *l, const void *src, void *dst
     TView v = make_view(*l, to_bricks ? dst : const_cast<void *>(src));
     const int E = l->elem_bytes, V = 16 / E;
     ConvGeom cg;
-    cg.rows = l->Bd * l->Bh;
-    cg.Wfull = (int)(l->nb[3] * l->Bw);
-    cg.vec_ok = ((l->W * E) % 16 == 0) && (((uintptr_t)(to_bricks ? src : dst)) % 16 == 0);
-    const size_t budget = 96 * 1024;
-    // channel group: the largest divisor of c_pad that is a multiple of V and fits the budget
-    cg.CG = V;
-    for (int k = 1; k <= l->c_pad / V; k++) {
-        int c = l->c_pad / k;
-        if (l->c_pad % k || c % V) continue;
-        if ((size_t)cg.rows * cg.Wfull * (c + 1) * E <= budget) { cg.CG = c; break; }
-    }
-    cg.CGP = cg.CG + 1;
-    cg.G = cg.CG / V;
-    cg.ngroups = (l->c_pad + cg.CG - 1) / cg.CG;
-    if (l->c_pad % cg.CG) return fail(BDL_EUNSUPPORTED, "brickify: channel grouping");
-    size_t smem = (size_t)cg.rows * cg.Wfull * cg.CGP * E;
-    if (smem > 200 * 1024) return fail(BDL_EUNSUPPORTED, "brickify: brick row tile too large for shared memory");
-    long long nrows = to_bricks ? l->nb[0] * (long long)l->Bn : l->N;
-    long long grid = nrows * l->nb[1] * l->nb[2] * cg.ngroups;
-    if (grid <= 0 || grid > 0x7fffffff) return fail(BDL_EINVAL, "brickify: grid size out of range");
+    cg.G = l->c_pad / V;
+    const long long Wg = l->nb[3] * l->Bw;
+    cg.XG = (int)((Wg + V - 1) / V);
+    cg.rows = (int)(l->nb[0] * l->Bn * l->nb[1] * l->Bd * l->nb[2] * l->Bh);
+    cg.vec_ok = ((l->W % V) == 0) && (((uintptr_t)(to_bricks ? src : dst)) % 16 == 0);
+    const long long units = to_bricks ? (long long)cg.rows * cg.XG * cg.G
+                                      : l->N * l->D * l->H * ((l->W + V - 1) / V) * (long long)cg.G;
+    const int threads = 256;
+    const long long blocks = std::max<long long>(1, std::min<long long>((units + threads - 1) / threads, 148LL * 16));
     cudaStream_t s = (cudaStream_t)stream;
     if (l->dtype == BDL_F32) {
-        if (to_bricks) {
-            cudaFuncSetAttribute(brickify_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-            brickify_kernel<float><<<(unsigned)grid, 256, smem, s>>>(v, (const float *)src, cg);
-        } else {
-            cudaFuncSetAttribute(unbrickify_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-            unbrickify_kernel<float><<<(unsigned)grid, 256, smem, s>>>(v, (float *)dst, cg);
-        }
+        if (to_bricks) brickify_kernel<float><<<(unsigned)blocks, threads, 0, s>>>(v, (const float *)src, cg);
+        else unbrickify_kernel<float><<<(unsigned)blocks, threads, 0, s>>>(v, (float *)dst, cg);
     } else {
-        if (to_bricks) {
-            cudaFuncSetAttribute(brickify_kernel<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-            brickify_kernel<__nv_bfloat16><<<(unsigned)grid, 256, smem, s>>>(v, (const __nv_bfloat16 *)src, cg);
-        } else {
-            cudaFuncSetAttribute(unbrickify_kernel<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-            unbrickify_kernel<__nv_bfloat16><<<(unsigned)grid, 256, smem, s>>>(v, (__nv_bfloat16 *)dst, cg);
-        }
+        if (to_bricks) brickify_kernel<__nv_bfloat16><<<(unsigned)blocks, threads, 0, s>>>(v, (const __nv_bfloat16 *)src, cg);
+        else unbrickify_kernel<__nv_bfloat16><<<(unsigned)blocks, threads, 0, s>>>(v, (__nv_bfloat16 *)dst, cg);
     }
     BDL_CUDA_CHECK_LAUNCH(to_bricks ? "bdl_brickify" : "bdl_unbrickify");
     return BDL_OK;
