@@ -43,7 +43,8 @@ struct Roles {
     static constexpr int LW = TMA ? 1 : 4;                 // loader warps
     static constexpr int WPROD = kLoadWarp0 + LW;          // weight producer warp (TMA bulk copies)
     static constexpr int MMA = WPROD + 1;                  // MMA warp
-    static constexpr int EPI0 = MMA + 1;                   // first epilogue warp
+    static constexpr int STORE = MMA + 1;                  // output store + memo publication warp
+    static constexpr int EPI0 = STORE + 1;                 // first epilogue warp
     static constexpr int THREADS = 32 * (EPI0 + kEpiWarps);
     static constexpr int LOADT = 32 * LW;
 };
@@ -72,6 +73,7 @@ struct Params {
     int nty, ntx;
     int lBh, lBw;            // log2 brick extents
     int rowsA;
+    int stage_off;           // TMA path: byte offset of the epilogue staging tile (Tb x Wt rows x C*2 B)
     int nin, nacc;           // input buffers (1-2), accumulators (1-2)
     int ntl;                 // M tiles per task
     int tmem_cols;
@@ -93,13 +95,14 @@ struct Params {
 
 struct Shared {
     uint64_t q_full[kQ], q_empty[kQ];
-    uint64_t res_full;
+    uint64_t res_full, stg_free;
     uint64_t in_full[2], in_empty[2], acc_full[2], acc_empty[2], wfull[kWS], wempty[kWS];
     uint32_t tmem_base;
     int q_l[kQ];
     long long q_t[kQ];
     int desc_l[kRing];
     long long desc_t[kRing];
+    int desc_seq[kRing];      // seq + 1 once desc_*[slot] holds task seq (polled by the epilogue)
     unsigned long long tr[kRing][4];
     int stk_l[kStack];
     long long stk_t[kStack];
@@ -415,7 +418,8 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
     // warp index via shuffle: provably warp-uniform, so role branches keep the uniform datapath
     const int warp = __shfl_sync(0xffffffff, (int)threadIdx.x / 32, 0), lane = threadIdx.x % 32;
     const size_t in_bytes = (size_t)KC * p.rowsA * 16;
-    uint8_t *wst = smem + in_bytes * p.nin;
+    const size_t stage_bytes = RL::TMA ? (((size_t)(C / 64) * p.Tb * p.Wt * 128 + 1023) / 1024 * 1024) : 0;
+    uint8_t *wst = smem + in_bytes * p.nin + stage_bytes;
     float *bias_s = reinterpret_cast<float *>(wst + kWS * C * C * 2);  // [L][C]
     for (int i = threadIdx.x; i < p.L * C; i += kThreads) bias_s[i] = p.layer[i / C].bias[i % C];
     if (RL::TMA && (ptx::smem_u32(smem) & 1023)) __trap();  // 128-B swizzle atoms need 1024-B alignment
@@ -436,6 +440,8 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
             ptx::mbar_init(&sh.wempty[i], 1);
         }
         ptx::mbar_init(&sh.res_full, 1);
+        ptx::mbar_init(&sh.stg_free, 1);
+        for (int i = 0; i < kRing; i++) sh.desc_seq[i] = 0;
         ptx::fence_barrier_init();
     }
     if (warp == kMmaWarp) {
@@ -500,6 +506,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                 sh.tr[seq % kRing][1] = t_dep;
                 sh.tr[seq % kRing][2] = gtime();
                 __threadfence_block();
+                *reinterpret_cast<volatile int *>(&sh.desc_seq[seq % kRing]) = (int)seq + 1;
                 mbar_arrive(&sh.in_full[b]);
                 mbar_arrive(&sh.q_empty[slot]);
             }
@@ -544,165 +551,187 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
             ptx::tc_fence_after();
             if (lane == 0) sh.tr[seq % kRing][3] = gtime();
             if (!(p.dbg & 1)) issue_task<C>(p, sh, ptx::smem_u32(smem + in_bytes * b), tmem_base + a * acc_cols, wst, 9 * seq);
-            if constexpr (!RL::TMA) ptx::mma_commit_elect(&sh.in_empty[b]);  // TMA path: the epilogue reuses
-            ptx::mma_commit_elect(&sh.acc_full[a]);                            // the buffer, then frees it
+            ptx::mma_commit_elect(&sh.in_empty[b]);
+            ptx::mma_commit_elect(&sh.acc_full[a]);
             __syncwarp();
         }
     } else {
-        // ------------------------------------------------------------------ epilogue
-        // kEpiWarps warps; warp ew reads TMEM lane quadrant warp % 4 of M tiles ew/4, ew/4 + 4, ...
+        // ------------------------------------------------------------------ epilogue + store warps
+        // Epilogue: kEpiWarps warps; warp ew reads TMEM lane quadrant warp % 4 of M tiles ew/4, ew/4+4,..
         // Each thread owns one pixel (TMEM lane) and processes its channels 32 at a time.
-        // TMA path: the task's (now idle) input buffer becomes the output staging tile: the residual
-        // rows are TMA-loaded into it, each thread reads its pixel's residual and writes its result
-        // (128-B swizzled pixel rows, conflict-free), and one thread TMA-stores whole tile rows into the
-        // bricked output, then frees the buffer for the loader.
-        const int ew = warp - kEpiWarp0;
-        const int quad = warp % 4;
-        const int tile0 = ew / 4;
-        const uint32_t acc_cols = (uint32_t)p.ntl * C;
-        constexpr int CB = C < 32 ? C : 32;      // channels per TMEM load batch
-        uint32_t res_phase = 0;
-        for (uint32_t seq = 0;; seq++) {
-            const int a = seq % p.nacc;
-            const int b = seq % p.nin;
-            ptx::mbar_wait(&sh.acc_full[a], (seq / p.nacc) & 1);
-            const int l = sh.desc_l[seq % kRing];
-            if (l < 0) break;
-            const unsigned long long t_acc = gtime();
-            const long long t = sh.desc_t[seq % kRing];
-            ptx::tc_fence_after();
-            const Layer &ly = p.layer[l];
-            int n, ty, tx;
-            decode(p, t, n, ty, tx);
-            const int y0 = ty * p.Tb, x0 = tx * p.Tw;
-            __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(ly.out.ptr);
-            const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(p.res.ptr);
-            const int Hg = ly.out.nb[2] << p.lBh, Wg = ly.out.nb[3] << p.lBw;  // bricked grid extents
-            const float *bl = bias_s + l * C;
-            uint8_t *stg = smem + in_bytes * b;
-            const uint32_t kb_stride = (uint32_t)p.rowsA * 128;
-            const int by = y0 >> p.lBh, bx0 = x0 >> p.lBw, nrows = min(p.Tb, p.H - y0);
-            if constexpr (RL::TMA) {
-                if (ly.res) {
-                    if (ew == 0 && ptx::elect_one()) {
-                        for (int i = 0; i < nrows; i++)
-                            for (int kb = 0; kb < C / 64; kb++) {
-                                ptx::mbar_expect_tx(&sh.res_full, (uint32_t)p.Tw * 128);
-                                ptx::tma_load_5d(stg + kb * kb_stride + (size_t)i * p.Wt * 128, &p.tm_res, kb * 64, 0, bx0, i,
-                                                 n * ly.out.nb[2] + by, &sh.res_full);
-                            }
-                        mbar_arrive(&sh.res_full);
+        // TMA path: a dedicated staging tile (128-B swizzled pixel rows m = i*Wt + j) receives the
+        // residual rows by TMA as soon as the task is known (overlapping its MMAs), each thread reads its
+        // pixel's residual and writes its result there, and the store warp TMA-stores whole tile rows
+        // into the bricked output, frees the staging tile, and publishes the task (memo state 2) once
+        // its global writes are complete.
+        const int Hg = p.layer[0].out.nb[2] << p.lBh;  // all layers share the spatial grid
+        constexpr int CB = C < 32 ? C : 32;            // channels per TMEM load batch
+        uint8_t *stg = smem + p.stage_off;
+        const uint32_t stg_kb = (uint32_t)p.Tb * p.Wt * 128;   // staging bytes per 64-channel block
+        if (warp == RL::STORE) {
+            uint32_t res_phase_unused = 0;
+            (void)res_phase_unused;
+            for (uint32_t seq = 0;; seq++) {
+                while (*reinterpret_cast<volatile int *>(&sh.desc_seq[seq % kRing]) != (int)seq + 1) __nanosleep(20);
+                const int l = sh.desc_l[seq % kRing];
+                const long long t = sh.desc_t[seq % kRing];
+                if (l < 0) break;
+                const Layer &ly = p.layer[l];
+                int n, ty, tx;
+                decode(p, t, n, ty, tx);
+                const int y0 = ty * p.Tb, x0 = tx * p.Tw;
+                const int nrows = min(p.Tb, p.H - y0);
+                if (RL::TMA && ly.res && lane == 0) {  // residual rows -> staging (staging is free here)
+                    for (int i = 0; i < nrows; i++) {
+                        const int y = y0 + i;
+                        for (int kb = 0; kb < C / 64; kb++) {
+                            ptx::mbar_expect_tx(&sh.res_full, (uint32_t)p.Tw * 128);
+                            ptx::tma_load_5d(stg + kb * stg_kb + (size_t)i * p.Wt * 128, &p.tm_res, kb * 64, 0, x0 >> p.lBw,
+                                             y & ((1 << p.lBh) - 1), n * ly.out.nb[2] + (y >> p.lBh), &sh.res_full);
+                        }
                     }
+                    mbar_arrive(&sh.res_full);
+                }
+                // wait until the epilogue warps have written this task's results
+                asm volatile("bar.sync 2, %0;" ::"n"(32 * (kEpiWarps + 1)) : "memory");
+                if (lane == 0) {
+                    if constexpr (RL::TMA) {
+                        for (int i = 0; i < p.Tb && y0 + i < Hg; i++) {
+                            const int y = y0 + i;
+                            for (int kb = 0; kb < C / 64; kb++)
+                                ptx::tma_store_5d(&p.tm_out[l], stg + kb * stg_kb + (size_t)i * p.Wt * 128, kb * 64, 0,
+                                                  x0 >> p.lBw, y & ((1 << p.lBh) - 1), n * ly.out.nb[2] + (y >> p.lBh));
+                        }
+                        ptx::bulk_commit();
+                        ptx::bulk_wait_read0();          // staging read out
+                        mbar_arrive(&sh.stg_free);
+                        ptx::bulk_wait0();               // global writes performed
+                        ptx::fence_proxy_async();
+                    }
+                    if (p.only_layer < 0) {
+                        __threadfence();
+                        st_release(status_word(p, l, t), (int)((p.epoch << 2) | 2));
+                    }
+                    atomicAdd(&p.counters[0], 1ULL);
+                    if (p.trace) {
+                        unsigned long long k = atomicAdd(&p.counters[5], 1ULL);
+                        if (k < (unsigned long long)p.trace_cap) {
+                            unsigned smid;
+                            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+                            unsigned long long *rec = p.trace + k * 8;
+                            rec[0] = ((unsigned long long)smid << 40) | ((unsigned long long)blockIdx.x << 8) | (unsigned)l;
+                            rec[1] = (unsigned long long)t;
+                            rec[2] = sh.tr[seq % kRing][0];
+                            rec[3] = sh.tr[seq % kRing][1];
+                            rec[4] = sh.tr[seq % kRing][2];
+                            rec[5] = sh.tr[seq % kRing][3];
+                            rec[6] = sh.tr[seq % kRing][3];
+                            rec[7] = gtime();
+                        }
+                    }
+                }
+                __syncwarp();
+            }
+        } else {
+            const int ew = warp - kEpiWarp0;
+            const int quad = warp % 4;
+            const int tile0 = ew / 4;
+            const uint32_t acc_cols = (uint32_t)p.ntl * C;
+            uint32_t res_phase = 0;
+            for (uint32_t seq = 0;; seq++) {
+                const int a = seq % p.nacc;
+                while (*reinterpret_cast<volatile int *>(&sh.desc_seq[seq % kRing]) != (int)seq + 1) __nanosleep(20);
+                const int l = sh.desc_l[seq % kRing];
+                const long long t = sh.desc_t[seq % kRing];
+                if (l < 0) break;
+                const Layer &ly = p.layer[l];
+                int n, ty, tx;
+                decode(p, t, n, ty, tx);
+                const int y0 = ty * p.Tb, x0 = tx * p.Tw;
+                if (RL::TMA && seq > 0) ptx::mbar_wait(&sh.stg_free, (seq - 1) & 1);  // last store read out
+                ptx::mbar_wait(&sh.acc_full[a], (seq / p.nacc) & 1);
+                ptx::tc_fence_after();
+                if (RL::TMA && ly.res) {
                     ptx::mbar_wait(&sh.res_full, res_phase);
                     res_phase ^= 1;
                 }
-            }
-            for (int tile = tile0; tile < ((p.dbg & 2) ? 0 : p.ntl); tile += 4) {
-                const int m = tile * 128 + quad * 32 + lane;
-                const int i = m / p.Wt, j = m - i * p.Wt;
-                const int y = y0 + i, x = x0 + j;
-                // 0: skip (garbage column / outside the tile / outside the brick grid), 1: zero (masked), 2: value
-                int kind = 0;
-                if (i < p.Tb && j < p.Tw && y < Hg && x < Wg) kind = (y < p.H && x < p.W) ? 2 : 1;
-                const bool has_res = kind == 2 && ly.res;
-                uint8_t *srow = stg + (size_t)m * 128;                       // TMA path staging row
-                const uint32_t sx = (ptx::smem_u32(srow) >> 7) & 7;        // its swizzle phase
-                uint4 *dst = nullptr;
-                uint4 rv[RL::TMA ? 1 : KC];
-                if constexpr (!RL::TMA) {
-                    dst = reinterpret_cast<uint4 *>(outp + (kind ? pix_off(ly.out, p.lBh, p.lBw, n, y, x) : 0));
-                    if (has_res) {
-                        const uint4 *rs = reinterpret_cast<const uint4 *>(resp + pix_off(p.res, p.lBh, p.lBw, n, y, x));
+                __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(ly.out.ptr);
+                const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(p.res.ptr);
+                const int Wg = ly.out.nb[3] << p.lBw;  // bricked grid extents
+                const float *bl = bias_s + l * C;
+                for (int tile = tile0; tile < ((p.dbg & 2) ? 0 : p.ntl); tile += 4) {
+                    const int m = tile * 128 + quad * 32 + lane;
+                    const int i = m / p.Wt, j = m - i * p.Wt;
+                    const int y = y0 + i, x = x0 + j;
+                    // 0: skip (garbage column / outside the tile / outside the grid), 1: zero (masked), 2: value
+                    int kind = 0;
+                    if (i < p.Tb && j < p.Tw && y < Hg && x < Wg) kind = (y < p.H && x < p.W) ? 2 : 1;
+                    const bool has_res = kind == 2 && ly.res;
+                    uint8_t *srow = stg + (size_t)m * 128;                       // TMA path staging row
+                    const uint32_t sx = (ptx::smem_u32(srow) >> 7) & 7;        // its swizzle phase
+                    uint4 *dst = nullptr;
+                    uint4 rv[RL::TMA ? 1 : KC];
+                    if constexpr (!RL::TMA) {
+                        dst = reinterpret_cast<uint4 *>(outp + (kind ? pix_off(ly.out, p.lBh, p.lBw, n, y, x) : 0));
+                        if (has_res) {
+                            const uint4 *rs = reinterpret_cast<const uint4 *>(resp + pix_off(p.res, p.lBh, p.lBw, n, y, x));
 #pragma unroll
-                        for (int k = 0; k < KC; k++) rv[k] = __ldcg(rs + k);
+                            for (int k = 0; k < KC; k++) rv[k] = __ldcg(rs + k);
+                        }
                     }
-                }
-                const uint32_t taddr = sh.tmem_base + a * acc_cols + ((uint32_t)(quad * 32) << 16) + tile * C;
+                    const uint32_t taddr = sh.tmem_base + a * acc_cols + ((uint32_t)(quad * 32) << 16) + tile * C;
 #pragma unroll
-                for (int cb = 0; cb < C / CB; cb++) {
-                    uint32_t r[CB / 16][16];
+                    for (int cb = 0; cb < C / CB; cb++) {
+                        uint32_t r[CB / 16][16];
 #pragma unroll
-                    for (int cc = 0; cc < CB / 16; cc++) ptx::tmem_ld16(taddr + cb * CB + cc * 16, r[cc]);
-                    ptx::tmem_ld_wait();
+                        for (int cc = 0; cc < CB / 16; cc++) ptx::tmem_ld16(taddr + cb * CB + cc * 16, r[cc]);
+                        ptx::tmem_ld_wait();
 #pragma unroll
-                    for (int cc = 0; cc < CB / 16; cc++) ptx::reg_fence16(r[cc]);
+                        for (int cc = 0; cc < CB / 16; cc++) ptx::reg_fence16(r[cc]);
 #pragma unroll
-                    for (int kq = 0; kq < CB / 8; kq++) {
-                        const int k = cb * (CB / 8) + kq;
-                        uint4 *sp = nullptr;
-                        if constexpr (RL::TMA) sp = reinterpret_cast<uint4 *>(srow + (k / 8) * kb_stride + (((k & 7) ^ sx) << 4));
-                        uint4 o = make_uint4(0, 0, 0, 0);
-                        if (kind == 2) {
-                            float v[8];
-                            const float4 b0 = *reinterpret_cast<const float4 *>(bl + k * 8);
-                            const float4 b1 = *reinterpret_cast<const float4 *>(bl + k * 8 + 4);
-                            const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+                        for (int kq = 0; kq < CB / 8; kq++) {
+                            const int k = cb * (CB / 8) + kq;
+                            uint4 *sp = nullptr;
+                            if constexpr (RL::TMA) sp = reinterpret_cast<uint4 *>(srow + (k / 8) * stg_kb + (((k & 7) ^ sx) << 4));
+                            uint4 o = make_uint4(0, 0, 0, 0);
+                            if (kind == 2) {
+                                float v[8];
+                                const float4 b0 = *reinterpret_cast<const float4 *>(bl + k * 8);
+                                const float4 b1 = *reinterpret_cast<const float4 *>(bl + k * 8 + 4);
+                                const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
-                            for (int e = 0; e < 8; e++) v[e] = __uint_as_float(r[kq / 2][(kq % 2) * 8 + e]) + bb[e];
-                            if (has_res) {
-                                uint4 rr;
-                                if constexpr (RL::TMA) rr = *sp;
-                                else rr = rv[k];
-                                const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr);
+                                for (int e = 0; e < 8; e++) v[e] = __uint_as_float(r[kq / 2][(kq % 2) * 8 + e]) + bb[e];
+                                if (has_res) {
+                                    uint4 rr;
+                                    if constexpr (RL::TMA) rr = *sp;
+                                    else rr = rv[k];
+                                    const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr);
 #pragma unroll
-                                for (int e = 0; e < 4; e++) {
-                                    float2 f = __bfloat1622float2(h2[e]);
-                                    v[2 * e] += f.x;
-                                    v[2 * e + 1] += f.y;
+                                    for (int e = 0; e < 4; e++) {
+                                        float2 f = __bfloat1622float2(h2[e]);
+                                        v[2 * e] += f.x;
+                                        v[2 * e + 1] += f.y;
+                                    }
                                 }
-                            }
-                            if (ly.relu) {
+                                if (ly.relu) {
 #pragma unroll
-                                for (int e = 0; e < 8; e++) v[e] = fmaxf(v[e], 0.f);
+                                    for (int e = 0; e < 8; e++) v[e] = fmaxf(v[e], 0.f);
+                                }
+                                o = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
                             }
-                            o = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
-                        }
-                        if constexpr (RL::TMA) {
-                            if (kind) *sp = o;
-                        } else {
-                            if (kind) dst[k] = o;
+                            if constexpr (RL::TMA) {
+                                if (kind) *sp = o;
+                            } else {
+                                if (kind) dst[k] = o;
+                            }
                         }
                     }
                 }
-            }
-            ptx::tc_fence_before();
-            if (lane == 0) mbar_arrive(&sh.acc_empty[a]);
-            if constexpr (RL::TMA) ptx::fence_proxy_async_smem();
-            // all epilogue threads done with this task (bar.sync: memory ordering for the release below)
-            asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiWarps) : "memory");
-            if (warp == kEpiWarp0 && lane == 0) {
-                if constexpr (RL::TMA) {
-                    for (int i = 0; i < p.Tb && y0 + i < Hg; i++)
-                        for (int kb = 0; kb < C / 64; kb++)
-                            ptx::tma_store_5d(&p.tm_out[l], stg + kb * kb_stride + (size_t)i * p.Wt * 128, kb * 64, 0, bx0, i,
-                                              n * ly.out.nb[2] + by);
-                    ptx::bulk_commit();
-                    ptx::bulk_wait_read0();           // staging tile read out: the loader may refill it
-                    mbar_arrive(&sh.in_empty[b]);
-                    ptx::bulk_wait0();                // global writes performed before the release
-                    ptx::fence_proxy_async();
-                }
-                if (p.only_layer < 0) {
-                    __threadfence();
-                    st_release(status_word(p, l, t), (int)((p.epoch << 2) | 2));
-                }
-                atomicAdd(&p.counters[0], 1ULL);
-                if (p.trace) {
-                    unsigned long long k = atomicAdd(&p.counters[5], 1ULL);
-                    if (k < (unsigned long long)p.trace_cap) {
-                        unsigned smid;
-                        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-                        unsigned long long *rec = p.trace + k * 8;
-                        rec[0] = ((unsigned long long)smid << 40) | ((unsigned long long)blockIdx.x << 8) | (unsigned)l;
-                        rec[1] = (unsigned long long)t;
-                        rec[2] = sh.tr[seq % kRing][0];
-                        rec[3] = sh.tr[seq % kRing][1];
-                        rec[4] = sh.tr[seq % kRing][2];
-                        rec[5] = sh.tr[seq % kRing][3];
-                        rec[6] = t_acc;
-                        rec[7] = gtime();
-                    }
-                }
+                ptx::tc_fence_before();
+                if (lane == 0) mbar_arrive(&sh.acc_empty[a]);
+                if constexpr (RL::TMA) ptx::fence_proxy_async_smem();
+                // hand the task to the store warp (memory ordering of the stores above: bar cumulativity)
+                asm volatile("bar.arrive 2, %0;" ::"n"(32 * (kEpiWarps + 1)) : "memory");
             }
         }
     }
@@ -730,33 +759,51 @@ static int ilog2(int v) {
 bool ws_geometry(const bdl_plan *p, const Subgraph &sg, WsGeom &g) {
     const Layer &f = p->layers[sg.first];
     const int C = f.L.cin;
-    const int W = f.in_ext[3];
+    const int H = f.in_ext[2], W = f.in_ext[3];
     const int Bh = p->in_layout.Bh, Bw = p->in_layout.Bw;
     if (p->in_layout.nsp != 2 || ilog2(Bh) < 0 || ilog2(Bw) < 0) return false;
-    const int limit = 227 * 1024 - 2048;
+    const bool tma = C % 64 == 0;
+    const int limit = 227 * 1024 - 4096;
     const int wbytes = ws::kWS * C * C * 2;
-    const int stage = (sg.last - sg.first + 1) * C * 4;  // bias table
-    int Wfull = (W + Bw - 1) / Bw * Bw;
-    for (int Tw = Wfull; Tw >= Bw; Tw -= Bw) {
-        g.Tb = Bh;
-        g.Tw = Tw;
-        g.Wt = Tw + 2;
-        int M = g.Tb * g.Wt;
-        g.ntl = (M + 127) / 128;
-        g.rowsA = (g.ntl * 128 + 2 * g.Wt + 2 + 7) / 8 * 8;
-        if (C % 64) g.rowsA += 1;  // unswizzled chunk planes: odd 16-B stride, conflict-free cp.async stores
-        int inb = (C / 8) * g.rowsA * 16;
-        int cols = g.ntl * C;
-        if (cols > 512) continue;
-        g.nacc = 2 * cols <= 512 ? 2 : 1;
-        g.tmem_cols = 32;
-        while (g.tmem_cols < cols * g.nacc) g.tmem_cols *= 2;
-        for (g.nin = 2; g.nin >= 1; g.nin--) {
-            g.smem = inb * g.nin + wbytes + stage;
-            if (g.smem <= limit) return true;
+    const int bias = (sg.last - sg.first + 1) * C * 4;
+    const int Wfull = (W + Bw - 1) / Bw * Bw;
+    double best = -1;
+    WsGeom cand;
+    // TMA path: any band height (bands need not align with bricks; a task is a Tb-row band);
+    // cp.async path: one brick row per band.
+    for (int Tb = tma ? std::min(H, 16) : Bh; Tb >= (tma ? 1 : Bh); Tb--) {
+        for (int Tw = Wfull; Tw >= Bw; Tw -= Bw) {
+            cand.Tb = Tb;
+            cand.Tw = Tw;
+            cand.Wt = Tw + 2;
+            const int M = Tb * cand.Wt;
+            cand.ntl = (M + 127) / 128;
+            const int cols = cand.ntl * C;
+            if (cols > 512) continue;
+            cand.rowsA = (cand.ntl * 128 + 2 * cand.Wt + 2 + 7) / 8 * 8;
+            if (!tma) cand.rowsA += 1;  // unswizzled chunk planes: odd 16-B stride, conflict-free cp.async stores
+            const int inb = (C / 8) * cand.rowsA * 16;
+            const int stage = tma ? ((C / 64) * Tb * cand.Wt * 128 + 1023) / 1024 * 1024 : 0;
+            cand.nacc = 2 * cols <= 512 ? 2 : 1;
+            cand.tmem_cols = 32;
+            while (cand.tmem_cols < cols * cand.nacc) cand.tmem_cols *= 2;
+            for (cand.nin = 2; cand.nin >= 1; cand.nin--) {
+                cand.smem = inb * cand.nin + stage + wbytes + bias;
+                if (cand.smem <= limit) break;
+            }
+            if (cand.smem > limit) continue;
+            // score: useful fraction of MMA rows, double-buffering, then taller bands (fewer tasks)
+            const double eff = (double)Tb * Tw / (cand.ntl * 128.0) * (cand.nin == 2 ? 1.0 : 0.7) *
+                               (cand.nacc == 2 ? 1.0 : 0.8);
+            const double score = eff + 1e-3 * Tb;
+            if (score > best) {
+                best = score;
+                g = cand;
+            }
+            break;  // widest fitting Tw for this Tb
         }
     }
-    return false;
+    return best > 0;
 }
 
 // Locality-aware wavefront order (host): step s, image n, layer l -> tile row b = s - lag*l.
@@ -870,6 +917,7 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
     P.lBh = ilog2(p->in_layout.Bh);
     P.lBw = ilog2(p->in_layout.Bw);
     P.rowsA = g.rowsA;
+    P.stage_off = (P.C / 8) * g.rowsA * 16 * g.nin;
     P.nin = g.nin;
     P.nacc = g.nacc;
     P.ntl = g.ntl;
@@ -963,3 +1011,11 @@ extern "C" int bdl_debug_ws_trace(unsigned long long *host, int max_records) {
     cudaMemcpy(host, bdl::ws_trace_buf, (size_t)n * 8 * 8, cudaMemcpyDeviceToHost);
     return n;
 }
+
+namespace bdl {
+// Band height of the warp-specialized kernel for subgraph sg (0 if it cannot run it).
+int ws_band_rows(const bdl_plan *p, const Subgraph &sg) {
+    WsGeom g;
+    return ws_geometry(p, sg, g) ? g.Tb : 0;
+}
+}  // namespace bdl

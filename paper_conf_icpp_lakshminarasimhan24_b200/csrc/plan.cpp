@@ -116,6 +116,7 @@ static bool is_pool(const Layer &l) { return l.L.kind == BDL_OP_MAXPOOL; }
 
 namespace bdl {
 int tc_band_rows(const bdl_plan *p, const Subgraph &sg, int *smem_out);
+int ws_band_rows(const bdl_plan *p, const Subgraph &sg);
 std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg);
 }
 using namespace bdl;
@@ -386,7 +387,8 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
                             in->Bn, in->Bd, in->Bh, in->Bw, in->dtype);
             if (j < L - 1) sg.memo_off[j] = take(lo.total_bytes);
             sg.task_base[j] = words;
-            words += lo.nbricks;
+            // memo tags: one per brick, or per band task of the tcgen05 kernels (bands of >= 1 row)
+            words += std::max<int64_t>(lo.nbricks, lo.N * lo.D * lo.H * lo.nb[3]);
         }
         sg.ntasks_total = words;
         sg.status_off = take(words * 4);
@@ -408,6 +410,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
         sg.scratch_off = L > 1 ? take((int64_t)sg.grid * 2 * sg.scratch_slot_floats * 4) : -1;
         if (sg.kernel == KERNEL_TC_BAND) {
             sg.tc_band = tc_band_rows(p, sg, &sg.tc_smem);
+            if (int wb = ws_band_rows(p, sg)) sg.tc_band = wb;  // memoized/unmerged band height
             sg.order_host = ws_task_order(p, sg);
             sg.norder = (int64_t)sg.order_host.size();
             sg.order_off = sg.norder ? take(sg.norder * 4) : -1;

@@ -132,7 +132,8 @@ def test_cfg2_tc_memo_counters():
     plan.set_mode("memoized")
     plan.forward(wl["x"])
     c = plan.counters(0)
-    tasks = 2 * 4 * 5          # layers x images x 8-row bands (full-width tiles)
+    tb = plan.subgraphs()[0]["tc_band"]
+    tasks = 2 * 4 * -(-40 // tb)   # layers x images x Tb-row bands (full-width tiles)
     assert c["computed"] == tasks and c["cas_ok"] == tasks
 
 
