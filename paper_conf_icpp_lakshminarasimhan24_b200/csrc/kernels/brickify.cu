@@ -41,6 +41,7 @@ __device__ __forceinline__ long long brick_px(const TView &v, int n, int d, int 
 template <typename T>
 __global__ void __launch_bounds__(256) brickify_kernel(TView v, const T *__restrict__ src, ConvGeom cg) {
     constexpr int V = Vec<T>::V;
+    pdl_launch_dependents();  // the merged subgraph kernel may start its prologue
     const long long units = (long long)cg.rows * cg.XG * cg.G;
     const int Dg = v.nb[1] * v.B[1], Hg = v.nb[2] * v.B[2], Wg = v.nb[3] * v.B[3];
     const long long plane = (long long)v.ext[1] * v.ext[2] * v.ext[3];
@@ -84,6 +85,7 @@ __global__ void __launch_bounds__(256) brickify_kernel(TView v, const T *__restr
 template <typename T>
 __global__ void __launch_bounds__(256) unbrickify_kernel(TView v, T *__restrict__ dstd, ConvGeom cg) {
     constexpr int V = Vec<T>::V;
+    pdl_wait();  // launched with PDL after the subgraph kernel: wait for its results
     const int XGd = (v.ext[3] + V - 1) / V;
     const long long units = (long long)v.ext[0] * v.ext[1] * v.ext[2] * XGd * cg.G;
     const long long plane = (long long)v.ext[1] * v.ext[2] * v.ext[3];
@@ -139,10 +141,10 @@ static bdl_status launch_convert(const bdl_layout *l, const void *src, void *dst
     cudaStream_t s = (cudaStream_t)stream;
     if (l->dtype == BDL_F32) {
         if (to_bricks) brickify_kernel<float><<<(unsigned)blocks, threads, 0, s>>>(v, (const float *)src, cg);
-        else unbrickify_kernel<float><<<(unsigned)blocks, threads, 0, s>>>(v, (float *)dst, cg);
+        else launch_pdl(unbrickify_kernel<float>, dim3((unsigned)blocks), dim3(threads), 0, s, v, (float *)dst, cg);
     } else {
         if (to_bricks) brickify_kernel<__nv_bfloat16><<<(unsigned)blocks, threads, 0, s>>>(v, (const __nv_bfloat16 *)src, cg);
-        else unbrickify_kernel<__nv_bfloat16><<<(unsigned)blocks, threads, 0, s>>>(v, (__nv_bfloat16 *)dst, cg);
+        else launch_pdl(unbrickify_kernel<__nv_bfloat16>, dim3((unsigned)blocks), dim3(threads), 0, s, v, (__nv_bfloat16 *)dst, cg);
     }
     BDL_CUDA_CHECK_LAUNCH(to_bricks ? "bdl_brickify" : "bdl_unbrickify");
     return BDL_OK;

@@ -48,7 +48,9 @@ struct Roles {
     static constexpr int THREADS = 32 * (EPI0 + kEpiWarps);
     static constexpr int LOADT = 32 * LW;
 };
-constexpr int kWS = 6;            // weight ring stages (one 3x3 tap each)
+constexpr int kTPS = 2;           // 3x3 taps per weight stage
+constexpr int kSPT = (9 + kTPS - 1) / kTPS;  // weight stages per task
+constexpr int kWS = 3;            // weight ring stages
 constexpr int kQ = 4;             // scheduler -> loader queue
 constexpr int kRing = 8;          // task descriptor ring (loader -> MMA -> epilogue)
 constexpr int kStack = 160;
@@ -103,7 +105,7 @@ struct Shared {
     int desc_l[kRing];
     long long desc_t[kRing];
     int desc_seq[kRing];      // seq + 1 once desc_*[slot] holds task seq (polled by the epilogue)
-    unsigned long long tr[kRing][4];
+    unsigned long long tr[kRing][8];   // debug trace timestamps per task slot
     int stk_l[kStack];
     long long stk_t[kStack];
 };
@@ -291,13 +293,14 @@ __device__ void scheduler(const Params &p, Shared &sh) {
 }
 
 // ---------------------------------------------------------------------------------------------- mma
-// Weight taps stream through a kWS-stage ring (global tap index g = 9*seq + tap -> stage g % kWS),
-// filled by the weight-producer warp and released by tcgen05.commit.  The MMA warp runs converged so
-// that descriptors are warp-uniform (uniform registers); an elected lane issues each MMA.
+// Weights stream through a kWS-stage ring, kTPS taps (kTPS x C x C bf16) per stage; global stage index
+// g = kSPT*seq + j -> ring slot g % kWS; filled by the weight-producer warp, released by tcgen05.commit.
+// The MMA warp runs converged so that descriptors are warp-uniform (uniform registers); an elected lane
+// issues each MMA.
 template <int C>
 __device__ __forceinline__ void issue_task(const Params &p, Shared &sh, uint32_t a_base, uint32_t d_base, uint8_t *wst,
-                                           uint32_t g0) {
-    constexpr uint32_t WB = C * C * 2;
+                                           uint32_t seq) {
+    constexpr uint32_t WB = C * C * 2;   // one tap
     constexpr uint32_t LBO_B = C * 16;
     constexpr uint32_t IDESC = ptx::idesc_bf16_f32(128, C);
     const uint32_t LBO_A = (uint32_t)p.rowsA * 16;
@@ -309,21 +312,24 @@ __device__ __forceinline__ void issue_task(const Params &p, Shared &sh, uint32_t
     const uint64_t bdesc0 = ptx::umma_desc_noswz(0, LBO_B, 128);
     const uint32_t row_u = SW ? 8 : 1;                                     // 16-B units per pixel row
     const uint32_t kb_u = SW ? (uint32_t)p.rowsA * 8 : 0;                  // 16-B units per k-block
-    for (int tap = 0; tap < 9; tap++) {
-        const uint32_t g = g0 + tap;
+    for (int j = 0; j < kSPT; j++) {
+        const uint32_t g = kSPT * seq + j;
         const int st = g % kWS;
         ptx::mbar_wait(&sh.wfull[st], (g / kWS) & 1);
         ptx::tc_fence_after();
-        const uint32_t shift = (uint32_t)((tap / 3) * p.Wt + (tap % 3));
-        const uint32_t b0 = (w_base + st * WB) >> 4;
-        const uint32_t a0 = (a_base >> 4) + shift * row_u;
-        for (int t = 0; t < p.ntl; t++) {
+        for (int tq = 0; tq < kTPS && j * kTPS + tq < 9; tq++) {
+            const int tap = j * kTPS + tq;
+            const uint32_t shift = (uint32_t)((tap / 3) * p.Wt + (tap % 3));
+            const uint32_t b0 = (w_base + st * (kTPS * WB) + tq * WB) >> 4;
+            const uint32_t a0 = (a_base >> 4) + shift * row_u;
+            for (int t = 0; t < p.ntl; t++) {
 #pragma unroll
-            for (int kk = 0; kk < C / 16; kk++) {
-                const uint32_t koff = SW ? (kk / 4) * kb_u + (kk % 4) * 2 : kk * (LBO_A >> 3);
-                const uint64_t ad = adesc0 | (uint64_t)((a0 + t * 128 * row_u + koff) & 0x3FFF);
-                const uint64_t bd = bdesc0 | (uint64_t)((b0 + kk * (LBO_B >> 3)) & 0x3FFF);
-                ptx::mma_bf16_elect(d_base + t * C, ad, bd, IDESC, (tap | kk) != 0);
+                for (int kk = 0; kk < C / 16; kk++) {
+                    const uint32_t koff = SW ? (kk / 4) * kb_u + (kk % 4) * 2 : kk * (LBO_A >> 3);
+                    const uint64_t ad = adesc0 | (uint64_t)((a0 + t * 128 * row_u + koff) & 0x3FFF);
+                    const uint64_t bd = bdesc0 | (uint64_t)((b0 + kk * (LBO_B >> 3)) & 0x3FFF);
+                    ptx::mma_bf16_elect(d_base + t * C, ad, bd, IDESC, (tap | kk) != 0);
+                }
             }
         }
         ptx::mma_commit_elect(&sh.wempty[st]);
@@ -420,7 +426,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
     const size_t in_bytes = (size_t)KC * p.rowsA * 16;
     const size_t stage_bytes = RL::TMA ? (((size_t)(C / 64) * p.Tb * p.Wt * 128 + 1023) / 1024 * 1024) : 0;
     uint8_t *wst = smem + in_bytes * p.nin + stage_bytes;
-    float *bias_s = reinterpret_cast<float *>(wst + kWS * C * C * 2);  // [L][C]
+    float *bias_s = reinterpret_cast<float *>(wst + kWS * kTPS * C * C * 2);  // [L][C]
     for (int i = threadIdx.x; i < p.L * C; i += kThreads) bias_s[i] = p.layer[i / C].bias[i % C];
     if (RL::TMA && (ptx::smem_u32(smem) & 1023)) __trap();  // 128-B swizzle atoms need 1024-B alignment
 
@@ -448,13 +454,14 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
         ptx::tmem_alloc(&sh.tmem_base, p.tmem_cols);
         ptx::tmem_relinquish();
     }
-    // zero the input buffers once (guard rows are never written by the loader)
-    for (size_t i = threadIdx.x * 16; i < in_bytes * p.nin; i += kThreads * 16)
-        *reinterpret_cast<uint4 *>(smem + i) = make_uint4(0, 0, 0, 0);
+    // (guard rows of the input buffers are never written by the loader; they only feed accumulator rows
+    //  that the epilogue discards, and MMA rows are independent, so they need no initialization)
     ptx::fence_proxy_async_smem();
     ptx::tc_fence_before();
     __syncthreads();
     ptx::tc_fence_after();
+    pdl_launch_dependents();  // let the next kernel (unbrickify) get scheduled
+    pdl_wait();               // PDL: the previous kernel's outputs (our inputs) are complete from here on
 
     if (warp == kSchedWarp) {
         scheduler(p, sh);
@@ -524,13 +531,15 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
             if (lane == 0) mbar_arrive(&sh.q_empty[slot]);
             if (l < 0) break;
             const __nv_bfloat16 *w = p.layer[l].w;
-            for (int tap = 0; tap < 9; tap++) {
-                const uint32_t g = 9 * seq + tap;
+            for (int j = 0; j < kSPT; j++) {
+                const uint32_t g = kSPT * seq + j;
                 const int st = g % kWS;
+                const int ntap = min(kTPS, 9 - j * kTPS);
+                const uint32_t bytes = (uint32_t)ntap * C * C * 2;
                 if (g >= (uint32_t)kWS) ptx::mbar_wait(&sh.wempty[st], ((g / kWS) - 1) & 1);
                 if (ptx::elect_one()) {
-                    ptx::mbar_arrive_expect_tx(&sh.wfull[st], C * C * 2);
-                    ptx::bulk_g2s(wst + st * (C * C * 2), w + (size_t)tap * C * C, C * C * 2, &sh.wfull[st]);
+                    ptx::mbar_arrive_expect_tx(&sh.wfull[st], bytes);
+                    ptx::bulk_g2s(wst + st * (kTPS * C * C * 2), w + (size_t)j * kTPS * C * C, bytes, &sh.wfull[st]);
                 }
                 __syncwarp();
             }
@@ -550,7 +559,8 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
             }
             ptx::tc_fence_after();
             if (lane == 0) sh.tr[seq % kRing][3] = gtime();
-            if (!(p.dbg & 1)) issue_task<C>(p, sh, ptx::smem_u32(smem + in_bytes * b), tmem_base + a * acc_cols, wst, 9 * seq);
+            if (!(p.dbg & 1)) issue_task<C>(p, sh, ptx::smem_u32(smem + in_bytes * b), tmem_base + a * acc_cols, wst, seq);
+            if (lane == 0) sh.tr[seq % kRing][4] = gtime();
             ptx::mma_commit_elect(&sh.in_empty[b]);
             ptx::mma_commit_elect(&sh.acc_full[a]);
             __syncwarp();
@@ -569,67 +579,105 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
         uint8_t *stg = smem + p.stage_off;
         const uint32_t stg_kb = (uint32_t)p.Tb * p.Wt * 128;   // staging bytes per 64-channel block
         if (warp == RL::STORE) {
-            uint32_t res_phase_unused = 0;
-            (void)res_phase_unused;
+            // Per task i: wait for its descriptor; once the previous task's TMA store has read the
+            // staging tile, free it and immediately prefetch task i's residual rows into it; then
+            // publish the previous task after its global writes complete; then wait for the epilogue
+            // and issue task i's row stores.
+            int prev_l = -1;
+            long long prev_t = 0;
+            uint32_t prev_seq = 0;
+            unsigned long long prev_sync = 0, prev_read = 0;
+            auto publish = [&](int l, long long t, uint32_t sq, unsigned long long t_sync, unsigned long long t_read) {
+                if (p.only_layer < 0) {
+                    __threadfence();
+                    st_release(status_word(p, l, t), (int)((p.epoch << 2) | 2));
+                }
+                atomicAdd(&p.counters[0], 1ULL);
+                if (p.trace) {
+                    unsigned long long k = atomicAdd(&p.counters[5], 1ULL);
+                    if (k < (unsigned long long)p.trace_cap) {
+                        unsigned smid;
+                        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+                        unsigned long long *rec = p.trace + k * 12;
+                        rec[0] = ((unsigned long long)smid << 40) | ((unsigned long long)blockIdx.x << 8) | (unsigned)l;
+                        rec[1] = (unsigned long long)t;
+                        for (int f = 0; f < 7; f++) rec[2 + f] = sh.tr[sq % kRing][f];
+                        rec[9] = t_sync;
+                        rec[10] = t_read;
+                        rec[11] = gtime();
+                    }
+                }
+            };
             for (uint32_t seq = 0;; seq++) {
-                while (*reinterpret_cast<volatile int *>(&sh.desc_seq[seq % kRing]) != (int)seq + 1) __nanosleep(20);
+                if (lane == 0 && RL::TMA && prev_l >= 0) {
+                    ptx::bulk_wait_read0();              // previous task's staging read out
+                    prev_read = gtime();
+                    mbar_arrive(&sh.stg_free);
+                }
+                // wait for this task's descriptor; if it is not there yet, publish the previous task first
+                // (the loader may be waiting for exactly that publication: never hold it back)
+                while (*reinterpret_cast<volatile int *>(&sh.desc_seq[seq % kRing]) != (int)seq + 1) {
+                    if (lane == 0 && prev_l >= 0) {
+                        if constexpr (RL::TMA) {
+                            ptx::bulk_wait0();
+                            ptx::fence_proxy_async();
+                        }
+                        publish(prev_l, prev_t, prev_seq, prev_sync, prev_read);
+                        prev_l = -1;
+                    }
+                    __nanosleep(20);
+                }
+                prev_l = __shfl_sync(0xffffffff, prev_l, 0);
                 const int l = sh.desc_l[seq % kRing];
                 const long long t = sh.desc_t[seq % kRing];
+                if (lane == 0) {
+                    if (RL::TMA && l >= 0 && p.layer[l].res) {  // prefetch this task's residual rows
+                        const Layer &ly = p.layer[l];
+                        int n, ty, tx;
+                        decode(p, t, n, ty, tx);
+                        const int y0 = ty * p.Tb, x0 = tx * p.Tw;
+                        const int nrows = min(p.Tb, p.H - y0);
+                        for (int i = 0; i < nrows; i++) {
+                            const int y = y0 + i;
+                            for (int kb = 0; kb < C / 64; kb++) {
+                                ptx::mbar_expect_tx(&sh.res_full, (uint32_t)p.Tw * 128);
+                                ptx::tma_load_5d(stg + kb * stg_kb + (size_t)i * p.Wt * 128, &p.tm_res, kb * 64, 0,
+                                                 x0 >> p.lBw, y & ((1 << p.lBh) - 1), n * ly.out.nb[2] + (y >> p.lBh),
+                                                 &sh.res_full);
+                            }
+                        }
+                        mbar_arrive(&sh.res_full);
+                    }
+                    if (prev_l >= 0) {
+                        if constexpr (RL::TMA) {
+                            ptx::bulk_wait0();           // global writes performed
+                            ptx::fence_proxy_async();
+                        }
+                        publish(prev_l, prev_t, prev_seq, prev_sync, prev_read);
+                    }
+                }
+                __syncwarp();
+                prev_l = -1;
                 if (l < 0) break;
                 const Layer &ly = p.layer[l];
                 int n, ty, tx;
                 decode(p, t, n, ty, tx);
                 const int y0 = ty * p.Tb, x0 = tx * p.Tw;
-                const int nrows = min(p.Tb, p.H - y0);
-                if (RL::TMA && ly.res && lane == 0) {  // residual rows -> staging (staging is free here)
-                    for (int i = 0; i < nrows; i++) {
-                        const int y = y0 + i;
-                        for (int kb = 0; kb < C / 64; kb++) {
-                            ptx::mbar_expect_tx(&sh.res_full, (uint32_t)p.Tw * 128);
-                            ptx::tma_load_5d(stg + kb * stg_kb + (size_t)i * p.Wt * 128, &p.tm_res, kb * 64, 0, x0 >> p.lBw,
-                                             y & ((1 << p.lBh) - 1), n * ly.out.nb[2] + (y >> p.lBh), &sh.res_full);
-                        }
-                    }
-                    mbar_arrive(&sh.res_full);
-                }
                 // wait until the epilogue warps have written this task's results
                 asm volatile("bar.sync 2, %0;" ::"n"(32 * (kEpiWarps + 1)) : "memory");
-                if (lane == 0) {
-                    if constexpr (RL::TMA) {
-                        for (int i = 0; i < p.Tb && y0 + i < Hg; i++) {
-                            const int y = y0 + i;
-                            for (int kb = 0; kb < C / 64; kb++)
-                                ptx::tma_store_5d(&p.tm_out[l], stg + kb * stg_kb + (size_t)i * p.Wt * 128, kb * 64, 0,
-                                                  x0 >> p.lBw, y & ((1 << p.lBh) - 1), n * ly.out.nb[2] + (y >> p.lBh));
-                        }
-                        ptx::bulk_commit();
-                        ptx::bulk_wait_read0();          // staging read out
-                        mbar_arrive(&sh.stg_free);
-                        ptx::bulk_wait0();               // global writes performed
-                        ptx::fence_proxy_async();
+                prev_sync = gtime();
+                if (lane == 0 && RL::TMA) {
+                    for (int i = 0; i < p.Tb && y0 + i < Hg; i++) {
+                        const int y = y0 + i;
+                        for (int kb = 0; kb < C / 64; kb++)
+                            ptx::tma_store_5d(&p.tm_out[l], stg + kb * stg_kb + (size_t)i * p.Wt * 128, kb * 64, 0,
+                                              x0 >> p.lBw, y & ((1 << p.lBh) - 1), n * ly.out.nb[2] + (y >> p.lBh));
                     }
-                    if (p.only_layer < 0) {
-                        __threadfence();
-                        st_release(status_word(p, l, t), (int)((p.epoch << 2) | 2));
-                    }
-                    atomicAdd(&p.counters[0], 1ULL);
-                    if (p.trace) {
-                        unsigned long long k = atomicAdd(&p.counters[5], 1ULL);
-                        if (k < (unsigned long long)p.trace_cap) {
-                            unsigned smid;
-                            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-                            unsigned long long *rec = p.trace + k * 8;
-                            rec[0] = ((unsigned long long)smid << 40) | ((unsigned long long)blockIdx.x << 8) | (unsigned)l;
-                            rec[1] = (unsigned long long)t;
-                            rec[2] = sh.tr[seq % kRing][0];
-                            rec[3] = sh.tr[seq % kRing][1];
-                            rec[4] = sh.tr[seq % kRing][2];
-                            rec[5] = sh.tr[seq % kRing][3];
-                            rec[6] = sh.tr[seq % kRing][3];
-                            rec[7] = gtime();
-                        }
-                    }
+                    ptx::bulk_commit();
                 }
+                prev_l = l;
+                prev_t = t;
+                prev_seq = seq;
                 __syncwarp();
             }
         } else {
@@ -650,6 +698,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                 const int y0 = ty * p.Tb, x0 = tx * p.Tw;
                 if (RL::TMA && seq > 0) ptx::mbar_wait(&sh.stg_free, (seq - 1) & 1);  // last store read out
                 ptx::mbar_wait(&sh.acc_full[a], (seq / p.nacc) & 1);
+                if (ew == 0 && lane == 0) sh.tr[seq % kRing][5] = gtime();
                 ptx::tc_fence_after();
                 if (RL::TMA && ly.res) {
                     ptx::mbar_wait(&sh.res_full, res_phase);
@@ -729,6 +778,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                 }
                 ptx::tc_fence_before();
                 if (lane == 0) mbar_arrive(&sh.acc_empty[a]);
+                if (ew == 0 && lane == 0) sh.tr[seq % kRing][6] = gtime();
                 if constexpr (RL::TMA) ptx::fence_proxy_async_smem();
                 // hand the task to the store warp (memory ordering of the stores above: bar cumulativity)
                 asm volatile("bar.arrive 2, %0;" ::"n"(32 * (kEpiWarps + 1)) : "memory");
@@ -764,7 +814,7 @@ bool ws_geometry(const bdl_plan *p, const Subgraph &sg, WsGeom &g) {
     if (p->in_layout.nsp != 2 || ilog2(Bh) < 0 || ilog2(Bw) < 0) return false;
     const bool tma = C % 64 == 0;
     const int limit = 227 * 1024 - 4096;
-    const int wbytes = ws::kWS * C * C * 2;
+    const int wbytes = ws::kWS * ws::kTPS * C * C * 2;
     const int bias = (sg.last - sg.first + 1) * C * 4;
     const int Wfull = (W + Bw - 1) / Bw * Bw;
     double best = -1;
@@ -834,7 +884,7 @@ static bdl_status launch_ws_C(bdl_plan *p, Subgraph &sg, ws::Params &P, const Ws
         P.only_layer = -1;
         P.ticket_base = sg.ticket_base;
         sg.ticket_base += (unsigned long long)P.norder + grid;
-        k<<<grid, ws::Roles<C>::THREADS, g.smem, s>>>(P);
+        launch_pdl(k, dim3(grid), dim3(ws::Roles<C>::THREADS), g.smem, s, P);
         *launches += 1;
     } else {
         P.order = nullptr;
@@ -844,7 +894,7 @@ static bdl_status launch_ws_C(bdl_plan *p, Subgraph &sg, ws::Params &P, const Ws
             P.only_layer = l;
             P.ticket_base = sg.ticket_base;
             sg.ticket_base += (unsigned long long)P.norder + grid;
-            k<<<grid, ws::Roles<C>::THREADS, g.smem, s>>>(P);
+            launch_pdl(k, dim3(grid), dim3(ws::Roles<C>::THREADS), g.smem, s, P);
             *launches += 1;
         }
     }
@@ -971,10 +1021,10 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
         if (cap > 0) {
             if (!tbuf || cap > tcap) {
                 if (tbuf) cudaFree(tbuf);
-                cudaMalloc(&tbuf, (size_t)cap * 8 * 8);
+                cudaMalloc(&tbuf, (size_t)cap * 12 * 8);
                 tcap = cap;
             }
-            cudaMemsetAsync(tbuf, 0, (size_t)cap * 8 * 8, s);
+            cudaMemsetAsync(tbuf, 0, (size_t)cap * 12 * 8, s);
             cudaMemsetAsync(wsp + sg.counter_off + 5 * 8, 0, 8, s);
             P.trace = tbuf;
             P.trace_cap = cap;
@@ -997,7 +1047,15 @@ namespace bdl {
 std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg) {
     WsGeom g;
     if (!ws_geometry(p, sg, g)) return {};
-    int lag = 3;
+    // lag: how many band rows layer l trails layer l-1.  Larger = fewer dependency waits but a larger
+    // live intermediate; take the largest lag whose live intermediate (lag band rows of every image of
+    // the shard, per merged layer) fits in a quarter of L2, at least 3.
+    const Layer &f = p->layers[sg.first];
+    const int L = sg.last - sg.first + 1;
+    const int nty = (f.in_ext[2] + g.Tb - 1) / g.Tb;
+    const double band_bytes = (double)f.in_ext[0] * g.Tb * f.in_ext[3] * f.L.cin * 2.0;
+    int lag = (int)std::min<double>(nty, (double)p->l2_bytes / 4.0 / std::max(1, L - 1) / band_bytes);
+    lag = std::max(3, lag);
     if (const char *e = getenv("BDL_LAG")) lag = std::max(1, atoi(e));
     return ws_order(p, sg, g, lag);
 }
@@ -1008,7 +1066,7 @@ extern "C" int bdl_debug_ws_trace(unsigned long long *host, int max_records) {
     if (!bdl::ws_trace_buf) return 0;
     int n = max_records < bdl::ws_trace_cap ? max_records : bdl::ws_trace_cap;
     cudaDeviceSynchronize();
-    cudaMemcpy(host, bdl::ws_trace_buf, (size_t)n * 8 * 8, cudaMemcpyDeviceToHost);
+    cudaMemcpy(host, bdl::ws_trace_buf, (size_t)n * 12 * 8, cudaMemcpyDeviceToHost);
     return n;
 }
 
