@@ -103,6 +103,8 @@ typedef struct bdl_plan_opts {
     int32_t force_brick;         /* 0 = the rho/tau model; else this brick edge for every subgraph */
     int32_t max_subgraph_layers; /* 0 = unlimited */
     int32_t num_sms;             /* 0 = query the device */
+    int32_t schedule_seed;       /* 0 = locality-aware wavefront task order; else a seeded random
+                                    permutation of the memo tasks (schedule-invariance testing) */
 } bdl_plan_opts;
 
 typedef struct bdl_plan bdl_plan;  /* opaque, library-owned host object */

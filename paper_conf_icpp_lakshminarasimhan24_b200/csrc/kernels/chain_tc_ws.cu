@@ -16,6 +16,7 @@
 // Loads of task i+1, MMAs of task i and the epilogue of task i-1 overlap.
 #include <algorithm>
 #include <cstdlib>
+#include <random>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -104,7 +105,7 @@ struct Shared {
     long long q_t[kQ];
     int desc_l[kRing];
     long long desc_t[kRing];
-    int desc_seq[kRing];      // seq + 1 once desc_*[slot] holds task seq (polled by the epilogue)
+    uint64_t desc_full[kRing];   // completes (phase seq / kRing) once desc_*[slot] holds task seq
     unsigned long long tr[kRing][8];   // debug trace timestamps per task slot
     int stk_l[kStack];
     long long stk_t[kStack];
@@ -447,7 +448,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
         }
         ptx::mbar_init(&sh.res_full, 1);
         ptx::mbar_init(&sh.stg_free, 1);
-        for (int i = 0; i < kRing; i++) sh.desc_seq[i] = 0;
+        for (int i = 0; i < kRing; i++) ptx::mbar_init(&sh.desc_full[i], 1);
         ptx::fence_barrier_init();
     }
     if (warp == kMmaWarp) {
@@ -512,8 +513,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                 sh.tr[seq % kRing][0] = t_q;
                 sh.tr[seq % kRing][1] = t_dep;
                 sh.tr[seq % kRing][2] = gtime();
-                __threadfence_block();
-                *reinterpret_cast<volatile int *>(&sh.desc_seq[seq % kRing]) = (int)seq + 1;
+                mbar_arrive(&sh.desc_full[seq % kRing]);   // release: descriptor visible to its waiters
                 mbar_arrive(&sh.in_full[b]);
                 mbar_arrive(&sh.q_empty[slot]);
             }
@@ -616,7 +616,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                 }
                 // wait for this task's descriptor; if it is not there yet, publish the previous task first
                 // (the loader may be waiting for exactly that publication: never hold it back)
-                while (*reinterpret_cast<volatile int *>(&sh.desc_seq[seq % kRing]) != (int)seq + 1) {
+                while (!ptx::mbar_test(&sh.desc_full[seq % kRing], (seq / kRing) & 1)) {
                     if (lane == 0 && prev_l >= 0) {
                         if constexpr (RL::TMA) {
                             ptx::bulk_wait0();
@@ -688,7 +688,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
             uint32_t res_phase = 0;
             for (uint32_t seq = 0;; seq++) {
                 const int a = seq % p.nacc;
-                while (*reinterpret_cast<volatile int *>(&sh.desc_seq[seq % kRing]) != (int)seq + 1) __nanosleep(20);
+                ptx::mbar_wait(&sh.desc_full[seq % kRing], (seq / kRing) & 1);
                 const int l = sh.desc_l[seq % kRing];
                 const long long t = sh.desc_t[seq % kRing];
                 if (l < 0) break;
@@ -1057,7 +1057,12 @@ std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg) {
     int lag = (int)std::min<double>(nty, (double)p->l2_bytes / 4.0 / std::max(1, L - 1) / band_bytes);
     lag = std::max(3, lag);
     if (const char *e = getenv("BDL_LAG")) lag = std::max(1, atoi(e));
-    return ws_order(p, sg, g, lag);
+    std::vector<int> ord = ws_order(p, sg, g, lag);
+    if (p->opts.schedule_seed) {  // any order is valid: the scheduler claims missing dependencies first
+        std::mt19937 rng((unsigned)p->opts.schedule_seed);
+        std::shuffle(ord.begin(), ord.end(), rng);
+    }
+    return ord;
 }
 }  // namespace bdl
 

@@ -189,3 +189,52 @@ def test_cfg4_resnet50_small():
     plan = engine.plan_from_workload(wl)
     y = plan.forward(wl["x"]).float().cpu().numpy()
     assert rel_err(y, ref) <= TOL["bf16"]
+
+
+# ---------------------------------------------------------------- schedule invariance
+def test_memo_schedule_invariance():
+    """Any task order gives bit-identical results and exactly-once execution: the scheduler claims
+    not-started dependencies first (Fig 2d recursion) and waits for in-progress ones."""
+    wl = workloads.make_workload("cfg2", N=3, H=24, W=24)
+    ref = None
+    for seed in (0, 1, 7, 123):
+        plan = engine.plan_from_workload(wl, schedule_seed=seed)
+        plan.set_mode("memoized")
+        y = plan.forward(wl["x"]).float().cpu().numpy()
+        c = plan.counters(0)
+        tb = plan.subgraphs()[0]["tc_band"]
+        tasks = 2 * 3 * -(-24 // tb)
+        assert c["computed"] == tasks and c["cas_ok"] == tasks, (seed, c)
+        if ref is None:
+            ref = y
+            assert rel_err(y, oracle_out(wl)) <= TOL["bf16"]
+        else:
+            np.testing.assert_array_equal(y, ref)
+
+
+# ---------------------------------------------------------------- full-size configurations, sampled
+def test_cfg5_full_size_sampled_crops():
+    """cfg5 at full size (1 x 32 x 128^3, four 3x3x3 layers, 4^3 bricks); the oracle evaluates crops
+    whose interior (4 voxels from any crop face that is not a volume face) equals the full result."""
+    wl = workloads.make_workload("cfg5")
+    plan = engine.plan_from_workload(wl)
+    y = plan.forward(wl["x"]).float().cpu().numpy()
+    x = wl["x"].numpy()
+    for lo, hi in [((0, 0, 0), (20, 20, 20)), ((60, 100, 30), (84, 128, 54))]:
+        sl = tuple(slice(a, b) for a, b in zip(lo, hi))
+        crop = x[(slice(None), slice(None)) + sl]
+        ref = oracle.run_graph(wl["layers"], crop, wl["weights"], wl["biases"], dtype="bf16")
+        keep = tuple(slice(0 if a == 0 else 4, (b - a) if b == 128 else (b - a) - 4) for a, b in zip(lo, hi))
+        got = y[(slice(None), slice(None)) + sl][(slice(None), slice(None)) + keep]
+        assert rel_err(got, ref[(slice(None), slice(None)) + keep]) <= TOL["bf16"]
+
+
+@pytest.mark.parametrize("cfg", ["cfg3", "cfg4"])
+def test_full_resolution_single_image(cfg):
+    """VGG-16 / ResNet-50 backbone at the paper's 224x224 resolution (one image), whole graph
+    partitioned by the planner, against the oracle."""
+    wl = workloads.make_workload(cfg, N=1)
+    ref = oracle_out(wl)
+    plan = engine.plan_from_workload(wl)
+    y = plan.forward(wl["x"]).float().cpu().numpy()
+    assert rel_err(y, ref) <= TOL["bf16"]
