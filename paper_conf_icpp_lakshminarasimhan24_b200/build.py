@@ -21,6 +21,7 @@ SOURCES = [
     "plan.cpp",
     "run.cu",
     "kernels/brickify.cu",
+    "kernels/brickify_tma.cu",
     "kernels/chain_brick.cu",
     "kernels/chain_tc.cu",
     "kernels/chain_tc_ws.cu",

@@ -8,6 +8,7 @@
 // the channel group fastest, so a warp's brick-side accesses are whole 128-byte pixel rows (C = 64
 // bf16) and its dense-side accesses are 64-byte runs of each channel plane.
 #include <algorithm>
+#include <cstdlib>
 #include <string>
 
 #include "common.cuh"
@@ -124,8 +125,18 @@ __global__ void __launch_bounds__(256) unbrickify_kernel(TView v, T *__restrict_
     }
 }
 
+bool launch_convert_tma(const bdl_layout *l, const void *dense, void *bricked, cudaStream_t s, bool to_bricks,
+                        bdl_status *st);
+
 static bdl_status launch_convert(const bdl_layout *l, const void *src, void *dst, void *stream, bool to_bricks) {
     if (!layout_valid(l) || !src || !dst) return fail(BDL_EINVAL, "brickify/unbrickify: bad layout or NULL pointer");
+    {   // bf16, C % 64 == 0, identity BrickMap: TMA-staged transposes
+        static const bool off = getenv("BDL_NO_TMA_BRICKIFY") != nullptr;
+        bdl_status st;
+        if (!off && launch_convert_tma(l, to_bricks ? src : dst, to_bricks ? dst : const_cast<void *>(src),
+                                       (cudaStream_t)stream, to_bricks, &st))
+            return st;
+    }
     TView v = make_view(*l, to_bricks ? dst : const_cast<void *>(src));
     const int E = l->elem_bytes, V = 16 / E;
     ConvGeom cg;
