@@ -462,7 +462,10 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
     __syncthreads();
     ptx::tc_fence_after();
     pdl_launch_dependents();  // let the next kernel (unbrickify) get scheduled
-    pdl_wait();               // PDL: the previous kernel's outputs (our inputs) are complete from here on
+    // PDL: only the roles that touch the previous kernel's output (the subgraph input) wait for it; the
+    // scheduler (memo tags, tickets) and the weight producer (packed weights) start right away.
+    const bool reads_input = (warp >= kLoadWarp0 && warp < RL::WPROD) || warp == RL::STORE || (!RL::TMA && warp >= kEpiWarp0);
+    if (reads_input) pdl_wait();
 
     if (warp == kSchedWarp) {
         scheduler(p, sh);
