@@ -294,8 +294,6 @@ def main():
     peaks, peak_src = load_peaks()
     flops = useful_flops(wl)
     kernel_ms = statistics.mean(run_ms)
-    achieved = flops / (kernel_ms / 1e3) / 1e12
-    peak = float(peaks["bf16_tflops"])
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_summary_latest.json")
     if os.path.exists(tp):
@@ -304,13 +302,24 @@ def main():
                 traffic = json.load(f).get("dram_bytes_per_launch", {}).get(sg[0]["kernel"])
         except Exception:
             traffic = None
-    roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
-                "traffic": traffic, "peak_source": f"{peak_src} bf16_tflops (burst, cuBLAS 8192^3)",
-                "kernel": f"{sg[0]['kernel']} ({sg[0]['mode']})", "algorithmic_flops_per_launch": flops,
-                "kernel_ms_mean": kernel_ms, "hbm_frac_of_step_bytes": None}
-    # step bytes: brickify (read+write) + merged subgraph (in, out, weights) + unbrickify (read+write)
-    act = wl["N"] * wl["C"] * wl["H"] * wl["W"] * 2
-    step_bytes = 2 * act + 2 * act + 2 * act
+    kinds = {g["kernel"] for g in sg}
+    if kinds == {"cuda-core brick"}:
+        # plain FMA pipes: 148 SMs x 128 fp32 FMA/clk x 2 flop x max SM clock
+        bound, peak = "alu", 148 * 128 * 2 * 1.965e9 / 1e12
+        peak_src = "derived: 148 SM x 128 FFMA/clk x 2 x 1965 MHz"
+    else:
+        bound, peak = "tensor", float(peaks["bf16_tflops"])
+        peak_src = f"{peak_src} bf16_tflops (burst, cuBLAS 8192^3)"
+    achieved = flops / (kernel_ms / 1e3) / 1e12
+    kname = sg[0]["kernel"] if len(sg) == 1 else f"{len(sg)} subgraph launches ({', '.join(sorted(kinds))})"
+    roofline = {"bound": bound, "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                "traffic": traffic if len(sg) == 1 else None, "peak_source": peak_src,
+                "kernel": f"{kname} ({'/'.join(sorted({g['mode'] for g in sg}))})",
+                "algorithmic_flops_per_launch": flops, "kernel_ms_mean": kernel_ms, "hbm_frac_of_step_bytes": None}
+    # step bytes: brickify (read+write) + subgraphs (in, out) + unbrickify (read+write)
+    in_b = x_dense.numel() * x_dense.element_size()
+    out_b = y_dense.numel() * y_dense.element_size()
+    step_bytes = 3 * in_b + 3 * out_b
     roofline["hbm_frac_of_step_bytes"] = step_bytes / (statistics.mean(step_ms) / 1e3) / 1e9 / float(peaks["hbm_gbs"])
 
     # ---- layer-by-layer cuDNN reference (context): torch conv2d, channels_last bf16
@@ -327,11 +336,11 @@ def main():
         line = {
             "metric": "images/sec merged conv chain per B200", "value": value, "unit": "images/s",
             "n_gpus": world, "steps": K, "warmup": max(3, args.warmup), "ms_per_step": total_ms / K,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": wl["dtype"],
             "data": "synthetic (seeded N(0,1) inputs, He-normal weights; workloads.py)",
             "config": {"workload": workload_desc(wl), "images_per_gpu": wl["N"], "global_batch": wl["N"] * world,
                        "mode": sg[0]["mode"], "mode_model": sg[0]["mode_model"], "delta": round(sg[0]["delta"], 4),
-                       "kernel": sg[0]["kernel"], "step": "brickify + merged subgraph + unbrickify",
+                       "kernel": sg[0]["kernel"], "subgraphs": len(sg), "step": "brickify + merged subgraph + unbrickify",
                        "l2": "flushed between timed steps (256 MiB write + 256 MiB read, outside the events)",
                        "parallelism": f"batch-sharded x{world}, no data-path collective"},
             "clocks": clk.summary(),
@@ -356,16 +365,25 @@ def cudnn_lbl(wl, dev, K, flush):
     import torch
     import torch.nn.functional as F
     try:
-        x = wl["x"][:, :, 0].to(device=dev, dtype=torch.bfloat16).contiguous(memory_format=torch.channels_last)
-        ws = [w[:, :, 0].to(device=dev, dtype=torch.bfloat16).contiguous(memory_format=torch.channels_last)
-              for w in wl["weights"]]
-        bs = [b.to(device=dev, dtype=torch.bfloat16) for b in wl["biases"]]
+        nsp3 = wl["nsp"] == 3
+        fmt = torch.channels_last_3d if nsp3 else torch.channels_last
+        x = wl["x"] if nsp3 else wl["x"][:, :, 0]
+        x = x.to(device=dev, dtype=torch.bfloat16).contiguous(memory_format=fmt)
+        ws = [None if w is None else (w if nsp3 else w[:, :, 0]).to(device=dev, dtype=torch.bfloat16)
+              .contiguous(memory_format=fmt) for w in wl["weights"]]
+        bs = [None if b is None else b.to(device=dev, dtype=torch.bfloat16) for b in wl["biases"]]
+        sl = slice(None) if nsp3 else slice(1, None)
 
         def fwd():
             outs = []
             for l, w, b in zip(wl["layers"], ws, bs):
                 src = x if l["input"] == -1 else outs[l["input"]]
-                y = F.conv2d(src, w, b, stride=l["stride"][1:], padding=l["pad"][1:])
+                if l["kind"] == "maxpool":
+                    pool = F.max_pool3d if nsp3 else F.max_pool2d
+                    y = pool(src, l["k"][sl], l["stride"][sl], l["pad"][sl])
+                else:
+                    conv = F.conv3d if nsp3 else F.conv2d
+                    y = conv(src, w, b, stride=l["stride"][sl], padding=l["pad"][sl])
                 if l["residual"] is not None:
                     y = y + (x if l["residual"] == -1 else outs[l["residual"]])
                 if l["relu"]:
@@ -386,7 +404,7 @@ def cudnn_lbl(wl, dev, K, flush):
                 b.synchronize()
                 tot += a.elapsed_time(b)
         return {"ms_per_step": tot / K, "images_per_s": wl["N"] * K / (tot / 1e3),
-                "what": "torch conv2d (cuDNN) bf16 channels_last, separate add/ReLU, dense NHWC in/out"}
+                "what": "torch conv (cuDNN) bf16 channels_last, separate add/ReLU/pool, dense channels-last in/out"}
     except Exception as e:  # context measurement only
         return {"error": str(e)[:200]}
 

@@ -19,7 +19,7 @@ BDL_MODE_AUTO, BDL_MODE_PADDED, BDL_MODE_MEMOIZED, BDL_MODE_UNMERGED = range(4)
 BDL_OP_CONV, BDL_OP_MAXPOOL = 0, 1
 BDL_NO_RESIDUAL, BDL_GRAPH_INPUT = -2, -1
 MODE_NAMES = {1: "padded", 2: "memoized", 3: "unmerged"}
-KERNEL_NAMES = {0: "cuda-core brick", 1: "tcgen05 band"}
+KERNEL_NAMES = {0: "cuda-core brick", 1: "tcgen05 band", 2: "tcgen05 generic"}
 
 _i32, _i64, _f64, _vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_double, ctypes.c_void_p
 

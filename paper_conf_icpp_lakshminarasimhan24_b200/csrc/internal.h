@@ -36,13 +36,14 @@ struct GLayer {
     TView out;           // memo buffer / subgraph output (bricked) for this layer's output
 };
 
-enum KernelKind { KERNEL_BRICK = 0, KERNEL_TC_BAND = 1 };
+enum KernelKind { KERNEL_BRICK = 0, KERNEL_TC_BAND = 1, KERNEL_TC_GEN = 2 };
 
 struct Layer {
     bdl_layer L;               // as given
     int in_ext[4], out_ext[4]; // (n, d, h, w)
     int64_t w_off = -1, b_off = -1;  // workspace offsets of packed weights / bias
-    int64_t tc_w_off = -1;           // tcgen05 packed weights
+    int64_t tc_w_off = -1;           // tcgen05 packed weights (band kernels: [tap][cin/8][cout][8];
+                                     // generic kernel: [nc][kb][kstep][2][Nc][8])
 };
 
 struct Tensor {                 // materialized tensor between subgraphs
@@ -58,7 +59,8 @@ struct Subgraph {
     int model_brick;            // rho/tau choice (edge)
     int64_t rho;
     double delta, delta_first;
-    int kernel;                 // KernelKind
+    int kernel;                 // KernelKind the subgraph is able to run on
+    int gen_layers = 0;         // generic tcgen05 kernel: leading conv layers it runs (a pool tail follows)
     int in_tensor;              // index into Plan::tensors
     int out_tensor;
     std::vector<int> res_tensor;   // per layer in subgraph: tensor index of external residual, or -1
@@ -104,5 +106,8 @@ namespace bdl {
 void set_error(const std::string &msg);
 bdl_status fail(bdl_status s, const std::string &msg);
 bool layout_valid(const bdl_layout *l);
+// kernel that actually executes subgraph sg in its current mode (padded multi-layer subgraphs that the
+// generic tcgen05 kernel cannot run in padded form use the CUDA-core brick kernel)
+int effective_kernel(const Subgraph &sg);
 TView make_view(const bdl_layout &l, void *ptr);
 }  // namespace bdl

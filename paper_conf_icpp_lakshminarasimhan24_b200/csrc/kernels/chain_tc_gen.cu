@@ -1,0 +1,878 @@
+// Generic warp-specialized tcgen05 kernel for MEMOIZED and UNMERGED execution of conv chains of any
+// shape the paper's workloads use (§3.2.2 Fig 2d, §4.3-§4.5): 2-D and 3-D, kernel sizes up to
+// 7, stride 1 or 2, any channel counts (cin <= 8, multiples of 16, multiples of 64), cin != cout,
+// bias / residual / ReLU epilogues.  The C = 64/128 3x3 chain of the bench config has its own tuned
+// kernel (chain_tc_ws.cu); this one covers everything else on the tensor cores.
+//
+// Implicit GEMM over an output TILE (Tb rows x Tw columns of one output plane, one chunk of Nc output
+// channels): M = 128 flattened tile positions m = i*Wp + j, N = Nc, K = input channels x taps.  The input
+// tile is staged in shared memory as pixel rows such that every tap (a, r, s) is a constant row offset
+// ("shifted window"): for stride 2 the tile is stored as polyphase blocks (row parity x column parity),
+// so a tap's rows are again contiguous.  Channels stream through the K loop in K-blocks (64 channels =
+// one 128-B swizzled pixel row); taps x 16-channel k-steps of each K-block are MMAs with a per-layer
+// table of A-descriptor offsets.  cin <= 8 (the RGB stem layers) packs two taps into one K = 16 step
+// through the descriptor's leading-byte offset.
+//
+// Roles (one CTA per SM, persistent):
+//   warp 0       scheduler: ticket counter over a topological (image-group, layer) order, CAS claims
+//                (0 -> 1, L513-531), claims not-started dependencies first (Fig 2d recursion)
+//   warps 1-4    loaders: wait for the dependency tiles (state 2), cp.async the K-blocks of the input
+//                tile into an input-stage ring (zero-fill outside the image)
+//   warp 5       weight producer: bulk copies of packed weight stages into a ring
+//   warp 6       MMA issuer (warp-converged, elected lane issues)
+//   warps 7-22   epilogue: tcgen05.ld -> +bias (+residual) -> ReLU -> bf16 -> bricked global stores,
+//                then release-publish the tile (state 2)
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "common.cuh"
+#include "tc_ptx.cuh"
+
+namespace bdl {
+
+namespace gen {
+
+constexpr int kSched = 0, kLoad0 = 1, kLW = 4, kWProd = 5, kMma = 6, kEpi0 = 7, kEpiW = 16;
+constexpr int kThreads = 32 * (kEpi0 + kEpiW);
+constexpr int kLoadT = 32 * kLW;
+constexpr int kQ = 4, kRing = 16, kStack = 128;
+constexpr int kMaxIn = 4, kMaxW = 4, kMaxKs = 64;
+
+enum { AM_SW128 = 0, AM_PLANES = 1, AM_PAIR = 2 };
+
+struct LayerP {
+    TView src, out, res;
+    const __nv_bfloat16 *w;   // packed [nc][kb][ks][2][Nc][8]
+    const float *bias;        // [cout]
+    int relu, has_res;
+    int cin, cout;
+    int k[3], s[3], pd[3];    // (d, h, w)
+    int in_ext[3], out_ext[3];
+    int grid[3];              // output bricked-grid extents (D, H, W)
+    int Tb, Tw, Wp;
+    int ntd, nty, ntx, nnc, Nc;
+    int amode, nkb, kc, nks, kpw, nws;   // kc: 16-B chunks per pixel per K-block
+    int rb, nblk, blk_px, plane_px;
+    int in_rows, in_cols;
+    int rowsA, stage_bytes, row_u;       // row_u: 16-B units per A row (8 swizzled, 1 planes)
+    int ntl;
+    uint32_t idesc;
+    long long task_base, ntasks;
+};
+
+struct Params {
+    LayerP layer[kMaxLayers];
+    int L;
+    int nin, nw, in_stride, w_stride;    // ring depths and slot strides (bytes)
+    int nacc, acc_stride, tmem_cols;
+    int *status;
+    unsigned epoch;
+    unsigned long long *counters;        // [0] computed [1] cas_ok [2] cas_fail [3] spins [4] ticket
+    unsigned long long ticket_base;
+    const int *order;                    // (l << 26) | task, or null (unmerged)
+    long long norder;
+    int only_layer;
+};
+
+struct Shared {
+    uint64_t q_full[kQ], q_empty[kQ];
+    uint64_t in_full[kMaxIn], in_empty[kMaxIn], wfull[kMaxW], wempty[kMaxW];
+    uint64_t acc_full[2], acc_empty[2];
+    uint64_t desc_full[kRing];
+    uint32_t tmem_base;
+    int q_l[kQ];
+    long long q_t[kQ];
+    int desc_l[kRing];
+    long long desc_t[kRing];
+    int stk_l[kStack];
+    long long stk_t[kStack];
+    uint2 ks[kMaxLayers][kMaxKs];        // per k-step: A offset (16-B units), LBO (16-B units)
+};
+
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ptx::smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ int tag_state(int v, unsigned EP) { return ((v & ~3) == (int)EP) ? (v & 3) : 0; }
+__device__ __forceinline__ int *status_word(const Params &p, int l, long long t) {
+    return p.status + p.layer[l].task_base + t;
+}
+
+struct TaskC { int n, d, ty, tx, nc; };
+__device__ __forceinline__ TaskC decode(const LayerP &L, long long t) {
+    TaskC c;
+    c.nc = (int)(t % L.nnc); t /= L.nnc;
+    c.tx = (int)(t % L.ntx); t /= L.ntx;
+    c.ty = (int)(t % L.nty); t /= L.nty;
+    c.d = (int)(t % L.ntd);
+    c.n = (int)(t / L.ntd);
+    return c;
+}
+
+// Element offset of channel 0 of pixel (n, d, y, x) in a bricked view (Bn = 1).
+__device__ __forceinline__ long long pix(const TView &v, int n, int d, int y, int x) {
+    const int bd = d / v.B[1], by = y / v.B[2], bx = x / v.B[3];
+    const long long logical = (((long long)n * v.nb[1] + bd) * v.nb[2] + by) * v.nb[3] + bx;
+    const long long phys = v.bmap ? (long long)v.bmap[logical] : logical;
+    const int in = (((d - bd * v.B[1]) * v.B[2]) + (y - by * v.B[2])) * v.B[3] + (x - bx * v.B[3]);
+    return phys * v.brick_elems + (long long)in * v.Cp;
+}
+
+// Dependencies of task t of layer l (l >= 1): the layer l-1 tiles covering its input window.
+struct DepRange { int n, d0, nd, b0, nb, x0, nx, nnc; };
+__device__ __forceinline__ DepRange dep_range(const Params &p, int l, long long t) {
+    const LayerP &C = p.layer[l], &P = p.layer[l - 1];
+    const TaskC c = decode(C, t);
+    DepRange r;
+    r.n = c.n;
+    r.nnc = P.nnc;
+    int lo, hi;
+    lo = max(0, c.d * C.s[0] - C.pd[0]);
+    hi = min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.k[0] - 1);
+    r.d0 = lo;
+    r.nd = max(0, hi - lo + 1);
+    lo = max(0, c.ty * C.Tb * C.s[1] - C.pd[1]);
+    hi = min(C.in_ext[1] - 1, (c.ty * C.Tb + C.Tb - 1) * C.s[1] - C.pd[1] + C.k[1] - 1);
+    r.b0 = lo / P.Tb;
+    r.nb = hi >= lo ? hi / P.Tb - r.b0 + 1 : 0;
+    lo = max(0, c.tx * C.Tw * C.s[2] - C.pd[2]);
+    hi = min(C.in_ext[2] - 1, (c.tx * C.Tw + C.Tw - 1) * C.s[2] - C.pd[2] + C.k[2] - 1);
+    r.x0 = lo / P.Tw;
+    r.nx = hi >= lo ? hi / P.Tw - r.x0 + 1 : 0;
+    return r;
+}
+__device__ __forceinline__ int dep_count(const DepRange &r) { return r.nd * r.nb * r.nx * r.nnc; }
+__device__ __forceinline__ long long dep_task(const Params &p, int l, const DepRange &r, int i) {
+    const LayerP &P = p.layer[l - 1];
+    const int c = i % r.nnc; i /= r.nnc;
+    const int x = r.x0 + i % r.nx; i /= r.nx;
+    const int b = r.b0 + i % r.nb; i /= r.nb;
+    const int d = r.d0 + i;
+    return ((((long long)r.n * P.ntd + d) * P.nty + b) * P.ntx + x) * P.nnc + c;
+}
+
+// ---------------------------------------------------------------------------------------------- scheduler
+__device__ void scheduler(const Params &p, Shared &sh) {
+    const int lane = threadIdx.x % 32;
+    const unsigned EP = p.epoch << 2;
+    const bool unmerged = p.only_layer >= 0;
+    unsigned long long oks = 0, fails = 0;
+    int sp = 0;
+    uint32_t qseq = 0;
+    auto emit = [&](int l, long long t) {
+        const int slot = qseq % kQ;
+        if (qseq >= (uint32_t)kQ) ptx::mbar_wait(&sh.q_empty[slot], ((qseq / kQ) - 1) & 1);
+        if (lane == 0) {
+            sh.q_l[slot] = l;
+            sh.q_t[slot] = t;
+            mbar_arrive(&sh.q_full[slot]);
+        }
+        __syncwarp();
+        qseq++;
+    };
+    for (;;) {
+        unsigned long long tk = 0;
+        if (lane == 0) tk = atomicAdd(&p.counters[4], 1ULL) - p.ticket_base;
+        tk = __shfl_sync(0xffffffff, tk, 0);
+        if ((long long)tk >= p.norder) break;
+        int l;
+        long long t;
+        if (unmerged) {
+            l = p.only_layer;
+            t = (long long)tk;
+        } else {
+            const int e = p.order[tk];
+            l = e >> 26;
+            t = e & ((1 << 26) - 1);
+            int ok = 0;
+            if (lane == 0) {
+                int *sw = status_word(p, l, t);
+                const int cur = ld_acquire(sw);
+                ok = tag_state(cur, EP) == 0 && atomicCAS(sw, cur, (int)(EP | 1)) == cur;
+            }
+            ok = __shfl_sync(0xffffffff, ok, 0);
+            if (!ok) continue;   // already claimed (by a dependent's recursion)
+            oks++;
+        }
+        if (lane == 0) {
+            sh.stk_l[0] = l;
+            sh.stk_t[0] = t;
+        }
+        sp = 1;
+        if (!unmerged) {
+            // recursion (Fig 2d): claim not-started dependencies, deepest first in the emit order
+            for (int s = 0; s < sp; s++) {
+                __syncwarp();
+                const int sl = sh.stk_l[s];
+                const long long st = sh.stk_t[s];
+                if (sl == 0) continue;
+                const DepRange r = dep_range(p, sl, st);
+                const int nd = dep_count(r);
+                for (int i0 = 0; i0 < nd; i0 += 32) {
+                    const int i = i0 + lane;
+                    int claimed = 0, busy = 0;
+                    long long dt = 0;
+                    if (i < nd && sp < kStack - 32) {
+                        dt = dep_task(p, sl, r, i);
+                        int *dw = status_word(p, sl - 1, dt);
+                        const int cur = ld_acquire(dw);
+                        const int s2 = tag_state(cur, EP);
+                        if (s2 == 0 && atomicCAS(dw, cur, (int)(EP | 1)) == cur) claimed = 1;
+                        else if (s2 != 2) busy = 1;
+                    }
+                    const unsigned cm = __ballot_sync(0xffffffff, claimed);
+                    fails += __popc(__ballot_sync(0xffffffff, busy));
+                    oks += __popc(cm);
+                    if (claimed) {
+                        const int pos = sp + __popc(cm & ((1u << lane) - 1));
+                        sh.stk_l[pos] = sl - 1;
+                        sh.stk_t[pos] = dt;
+                    }
+                    sp += __popc(cm);
+                }
+            }
+            __syncwarp();
+        }
+        // emit dependencies before dependents (reverse stack order)
+        while (sp > 0) {
+            sp--;
+            __syncwarp();
+            emit(sh.stk_l[sp], sh.stk_t[sp]);
+        }
+    }
+    emit(-1, 0);
+    if (lane == 0) {
+        if (oks) atomicAdd(&p.counters[1], oks);
+        if (fails) atomicAdd(&p.counters[2], fails);
+    }
+}
+
+// ---------------------------------------------------------------------------------------------- loader
+// One K-block of the input tile of task (n, d, ty, tx) into stage `buf` (128 threads).
+__device__ __forceinline__ void load_stage(const LayerP &L, const TaskC &c, int kb, uint8_t *buf, int tid) {
+    const TView &v = L.src;
+    const __nv_bfloat16 *base = reinterpret_cast<const __nv_bfloat16 *>(v.ptr);
+    const int kc = L.kc;
+    const int npx = L.k[0] * L.in_rows * L.in_cols;
+    const int total = npx * kc;
+    const int z0 = c.d * L.s[0] - L.pd[0];
+    const int y0 = c.ty * L.Tb * L.s[1] - L.pd[1];
+    const int x0 = c.tx * L.Tw * L.s[2] - L.pd[2];
+    const uint32_t plane_bytes = (uint32_t)L.rowsA * 16;
+    for (int it = tid; it < total; it += kLoadT) {
+        const int P = it / kc, ch = it - P * kc;
+        const int xx = P % L.in_cols;
+        const int r2 = P / L.in_cols;
+        const int yy = r2 % L.in_rows, a = r2 / L.in_rows;
+        const int z = z0 + a, y = y0 + yy, x = x0 + xx;
+        const bool ok = z >= 0 && z < L.in_ext[0] && y >= 0 && y < L.in_ext[1] && x >= 0 && x < L.in_ext[2];
+        const int px = a * L.plane_px + ((yy % L.s[1]) * L.s[2] + (xx % L.s[2])) * L.blk_px + (yy / L.s[1]) * L.Wp +
+                       xx / L.s[2];
+        uint32_t off;
+        if (L.amode == AM_SW128) off = (uint32_t)px * 128 + ((ch ^ (px & 7)) << 4);
+        else off = (uint32_t)ch * plane_bytes + (uint32_t)px * 16;
+        const void *g = ok ? (const void *)(base + pix(v, c.n, z, y, x) + kb * 64 + ch * 8) : (const void *)base;
+        ptx::cp_async16(buf + off, g, ok ? 16u : 0u);
+    }
+}
+
+__device__ __forceinline__ uint32_t pack2(float a, float b) {
+    __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
+    return *reinterpret_cast<uint32_t *>(&v);
+}
+
+// ---------------------------------------------------------------------------------------------- kernel
+__global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant__ Params p) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    __shared__ Shared sh;
+    const int warp = __shfl_sync(0xffffffff, (int)threadIdx.x / 32, 0), lane = threadIdx.x % 32;
+    uint8_t *in_ring = smem;
+    uint8_t *w_ring = smem + (size_t)p.nin * p.in_stride;
+    if (ptx::smem_u32(smem) & 1023) __trap();   // 128-B swizzle atoms need 1024-B alignment
+
+    // k-step descriptor-offset tables
+    for (int i = threadIdx.x; i < p.L * kMaxKs; i += kThreads) {
+        const int l = i / kMaxKs, q = i % kMaxKs;
+        const LayerP &L = p.layer[l];
+        if (q >= L.nks) continue;
+        int tap, kk = 0, t1 = -1;
+        if (L.amode == AM_SW128) { tap = q / 4; kk = q % 4; }
+        else if (L.amode == AM_PLANES) { const int kpt = (L.cin + 15) / 16; tap = q / kpt; kk = q % kpt; }
+        else {   // pair taps (a, r, 2u) and (a, r, 2u+1)
+            const int np = (L.k[2] + 1) / 2;
+            const int u = q % np, ar = q / np;
+            tap = ar * L.k[2] + 2 * u;
+            t1 = 2 * u + 1 < L.k[2] ? tap + 1 : -1;
+        }
+        auto tap_px = [&](int tp) {
+            const int s = tp % L.k[2], r = (tp / L.k[2]) % L.k[1], a = tp / (L.k[2] * L.k[1]);
+            return a * L.plane_px + ((r % L.s[1]) * L.s[2] + (s % L.s[2])) * L.blk_px + (r / L.s[1]) * L.Wp + s / L.s[2];
+        };
+        uint32_t aoff, lbo;
+        if (L.amode == AM_SW128) { aoff = (uint32_t)tap_px(tap) * 8 + kk * 2; lbo = 1; }
+        else if (L.amode == AM_PLANES) { aoff = (uint32_t)tap_px(tap) + 2u * kk * L.rowsA; lbo = L.rowsA; }
+        else { aoff = tap_px(tap); lbo = t1 >= 0 ? (uint32_t)(tap_px(t1) - tap_px(tap)) : 0u; }
+        sh.ks[l][q] = make_uint2(aoff, lbo);
+    }
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < kQ; i++) {
+            ptx::mbar_init(&sh.q_full[i], 1);
+            ptx::mbar_init(&sh.q_empty[i], 2);          // loader + weight producer
+        }
+        for (int i = 0; i < kMaxIn; i++) {
+            ptx::mbar_init(&sh.in_full[i], kLoadT);      // every loader thread after its copies landed
+            ptx::mbar_init(&sh.in_empty[i], 1);
+        }
+        for (int i = 0; i < kMaxW; i++) {
+            ptx::mbar_init(&sh.wfull[i], 1);
+            ptx::mbar_init(&sh.wempty[i], 1);
+        }
+        for (int i = 0; i < 2; i++) {
+            ptx::mbar_init(&sh.acc_full[i], 1);
+            ptx::mbar_init(&sh.acc_empty[i], kEpiW);
+        }
+        for (int i = 0; i < kRing; i++) ptx::mbar_init(&sh.desc_full[i], 1);
+        ptx::fence_barrier_init();
+    }
+    if (warp == kMma) {
+        ptx::tmem_alloc(&sh.tmem_base, p.tmem_cols);
+        ptx::tmem_relinquish();
+    }
+    ptx::fence_proxy_async_smem();
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::tc_fence_after();
+    pdl_launch_dependents();
+    if ((warp >= kLoad0 && warp < kLoad0 + kLW) || warp >= kEpi0) pdl_wait();   // read the previous kernel's output
+
+    const unsigned EP = p.epoch << 2;
+    if (warp == kSched) {
+        scheduler(p, sh);
+    } else if (warp < kLoad0 + kLW) {
+        // ------------------------------------------------------------------ loaders
+        const int tid = threadIdx.x - 32 * kLoad0;
+        uint32_t gin = 0;
+        for (uint32_t seq = 0;; seq++) {
+            const int slot = seq % kQ;
+            ptx::mbar_wait(&sh.q_full[slot], (seq / kQ) & 1);
+            const int l = sh.q_l[slot];
+            const long long t = sh.q_t[slot];
+            if (l >= 0 && l > 0 && p.only_layer < 0 && warp == kLoad0) {
+                // wait for the dependency tiles (state 2 of this epoch)
+                const DepRange r = dep_range(p, l, t);
+                const int nd = dep_count(r);
+                unsigned long long spins = 0;
+                for (int i = lane; i < nd; i += 32) {
+                    const int *dw = status_word(p, l - 1, dep_task(p, l, r, i));
+                    while (ld_acquire(dw) != (int)(EP | 2)) {
+                        spins++;
+                        __nanosleep(32);
+                    }
+                }
+                __syncwarp();
+                for (int o = 16; o; o >>= 1) spins += __shfl_xor_sync(0xffffffff, spins, o);
+                if (lane == 0 && spins) atomicAdd(&p.counters[3], spins);
+            }
+            asm volatile("bar.sync 1, %0;" ::"n"(kLoadT) : "memory");
+            if (tid == 0) {
+                sh.desc_l[seq % kRing] = l;
+                sh.desc_t[seq % kRing] = t;
+                mbar_arrive(&sh.desc_full[seq % kRing]);
+                mbar_arrive(&sh.q_empty[slot]);
+            }
+            if (l < 0) break;
+            const LayerP &L = p.layer[l];
+            const TaskC c = decode(L, t);
+            for (int kb = 0; kb < L.nkb; kb++, gin++) {
+                const int s = gin % p.nin;
+                if (gin >= (uint32_t)p.nin) ptx::mbar_wait(&sh.in_empty[s], ((gin / p.nin) - 1) & 1);
+                load_stage(L, c, kb, in_ring + (size_t)s * p.in_stride, tid);
+                ptx::cp_async_wait_all();
+                ptx::fence_proxy_async_smem();
+                mbar_arrive(&sh.in_full[s]);
+            }
+        }
+    } else if (warp == kWProd) {
+        // ------------------------------------------------------------------ weight producer
+        uint32_t gw = 0;
+        for (uint32_t seq = 0;; seq++) {
+            const int slot = seq % kQ;
+            ptx::mbar_wait(&sh.q_full[slot], (seq / kQ) & 1);
+            const int l = sh.q_l[slot];
+            const long long t = sh.q_t[slot];
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&sh.q_empty[slot]);
+            if (l < 0) break;
+            const LayerP &L = p.layer[l];
+            const int nc = (int)(t % L.nnc);
+            const size_t ks_bytes = (size_t)2 * L.Nc * 16;
+            const uint8_t *wl = reinterpret_cast<const uint8_t *>(L.w) + (size_t)nc * L.nkb * L.nks * ks_bytes;
+            for (int kb = 0; kb < L.nkb; kb++) {
+                for (int j = 0; j < L.nws; j++, gw++) {
+                    const int st = gw % p.nw;
+                    const int q0 = j * L.kpw, nq = min(L.kpw, L.nks - q0);
+                    const uint32_t bytes = (uint32_t)(nq * ks_bytes);
+                    if (gw >= (uint32_t)p.nw) ptx::mbar_wait(&sh.wempty[st], ((gw / p.nw) - 1) & 1);
+                    if (ptx::elect_one()) {
+                        ptx::mbar_arrive_expect_tx(&sh.wfull[st], bytes);
+                        ptx::bulk_g2s(w_ring + (size_t)st * p.w_stride, wl + ((size_t)kb * L.nks + q0) * ks_bytes, bytes,
+                                      &sh.wfull[st]);
+                    }
+                    __syncwarp();
+                }
+            }
+        }
+    } else if (warp == kMma) {
+        // ------------------------------------------------------------------ MMA issuer
+        const uint32_t tmem_base = __shfl_sync(0xffffffff, sh.tmem_base, 0);
+        uint32_t gin = 0, gw = 0;
+        for (uint32_t seq = 0;; seq++) {
+            ptx::mbar_wait(&sh.desc_full[seq % kRing], (seq / kRing) & 1);
+            const int l = sh.desc_l[seq % kRing];
+            if (l < 0) break;
+            const LayerP &L = p.layer[l];
+            const int a = seq % p.nacc;
+            if (seq >= (uint32_t)p.nacc) ptx::mbar_wait(&sh.acc_empty[a], ((seq / p.nacc) - 1) & 1);
+            ptx::tc_fence_after();
+            const uint32_t d_base = tmem_base + a * p.acc_stride;
+            const uint32_t lbo_b = (uint32_t)L.Nc * 16;
+            const uint32_t ks_u = (uint32_t)L.Nc * 2;   // 16-B units per k-step of B
+            for (int kb = 0; kb < L.nkb; kb++, gin++) {
+                const int s = gin % p.nin;
+                ptx::mbar_wait(&sh.in_full[s], (gin / p.nin) & 1);
+                ptx::tc_fence_after();
+                const uint32_t a_base = ptx::smem_u32(in_ring + (size_t)s * p.in_stride) >> 4;
+                for (int j = 0; j < L.nws; j++, gw++) {
+                    const int st = gw % p.nw;
+                    ptx::mbar_wait(&sh.wfull[st], (gw / p.nw) & 1);
+                    ptx::tc_fence_after();
+                    const uint32_t b_base = ptx::smem_u32(w_ring + (size_t)st * p.w_stride) >> 4;
+                    const int q0 = j * L.kpw, q1 = min(L.nks, q0 + L.kpw);
+                    for (int q = q0; q < q1; q++) {
+                        const uint2 e = sh.ks[l][q];
+                        const uint64_t bd = ptx::umma_desc_noswz(0, lbo_b, 128) |
+                                            (uint64_t)((b_base + (q - q0) * ks_u) & 0x3FFF);
+                        uint64_t ad0;
+                        if (L.amode == AM_SW128) ad0 = ptx::umma_desc_sw128(0, 1024);
+                        else ad0 = ptx::umma_desc_noswz(0, e.y * 16, 128);
+                        for (int tl = 0; tl < L.ntl; tl++) {
+                            const uint64_t ad = ad0 | (uint64_t)((a_base + e.x + tl * 128 * L.row_u) & 0x3FFF);
+                            ptx::mma_bf16_elect(d_base + tl * L.Nc, ad, bd, L.idesc, (kb | q) != 0);
+                        }
+                    }
+                    ptx::mma_commit_elect(&sh.wempty[st]);
+                }
+                ptx::mma_commit_elect(&sh.in_empty[s]);
+            }
+            ptx::mma_commit_elect(&sh.acc_full[a]);
+            __syncwarp();
+        }
+    } else {
+        // ------------------------------------------------------------------ epilogue
+        const int ew = warp - kEpi0;
+        const int quad = warp % 4;        // TMEM lane quadrant this warp may access
+        const int rank = ew / 4;          // 4 warps per quadrant split the (tile, column batch) items
+        const uint32_t tmem_base = sh.tmem_base;
+        for (uint32_t seq = 0;; seq++) {
+            ptx::mbar_wait(&sh.desc_full[seq % kRing], (seq / kRing) & 1);
+            const int l = sh.desc_l[seq % kRing];
+            const long long t = sh.desc_t[seq % kRing];
+            if (l < 0) break;
+            const LayerP &L = p.layer[l];
+            const TaskC c = decode(L, t);
+            const int a = seq % p.nacc;
+            ptx::mbar_wait(&sh.acc_full[a], (seq / p.nacc) & 1);
+            ptx::tc_fence_after();
+            const int CB = L.Nc >= 32 ? 32 : 16;
+            const int ncb = L.Nc / CB;
+            const int items = L.ntl * ncb;
+            __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(L.out.ptr);
+            const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(L.res.ptr);
+            const int d = c.d;
+            for (int it = rank; it < items; it += 4) {
+                const int tl = it / ncb, cb = it - tl * ncb;
+                const int m = tl * 128 + quad * 32 + lane;
+                const int i = m / L.Wp, j = m - i * L.Wp;
+                const int y = c.ty * L.Tb + i, x = c.tx * L.Tw + j;
+                int kind = 0;   // 0 skip, 1 zero (masked), 2 value
+                if (i < L.Tb && j < L.Tw && d < L.grid[0] && y < L.grid[1] && x < L.grid[2])
+                    kind = (d < L.out_ext[0] && y < L.out_ext[1] && x < L.out_ext[2]) ? 2 : 1;
+                const int ch0 = c.nc * L.Nc + cb * CB;
+                uint32_t r[2][16];
+                const uint32_t taddr = tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) + tl * L.Nc + cb * CB;
+                ptx::tmem_ld16(taddr, r[0]);
+                if (CB == 32) ptx::tmem_ld16(taddr + 16, r[1]);
+                ptx::tmem_ld_wait();
+                ptx::reg_fence16(r[0]);
+                ptx::reg_fence16(r[1]);
+                if (!kind) continue;
+                uint4 *dst = reinterpret_cast<uint4 *>(outp + pix(L.out, c.n, d, y, x) + ch0);
+                if (kind == 1) {
+                    for (int k = 0; k < CB / 8; k++) dst[k] = make_uint4(0, 0, 0, 0);
+                    continue;
+                }
+                const uint4 *rs = L.has_res ? reinterpret_cast<const uint4 *>(resp + pix(L.res, c.n, d, y, x) + ch0) : nullptr;
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    if (k >= CB / 8) break;
+                    float v[8];
+                    const float4 b0 = __ldg(reinterpret_cast<const float4 *>(L.bias + ch0 + k * 8));
+                    const float4 b1 = __ldg(reinterpret_cast<const float4 *>(L.bias + ch0 + k * 8 + 4));
+                    const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+                    for (int e = 0; e < 8; e++) v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]) + bb[e];
+                    if (rs) {
+                        const uint4 rr = __ldcg(rs + k);
+                        const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr);
+#pragma unroll
+                        for (int e = 0; e < 4; e++) {
+                            const float2 f = __bfloat1622float2(h2[e]);
+                            v[2 * e] += f.x;
+                            v[2 * e + 1] += f.y;
+                        }
+                    }
+                    if (L.relu) {
+#pragma unroll
+                        for (int e = 0; e < 8; e++) v[e] = fmaxf(v[e], 0.f);
+                    }
+                    dst[k] = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
+                }
+            }
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&sh.acc_empty[a]);
+            // every epilogue warp's stores of this tile precede the publication
+            asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");
+            if (ew == 0 && lane == 0) {
+                __threadfence();
+                if (p.only_layer < 0) st_release(status_word(p, l, t), (int)(EP | 2));
+                atomicAdd(&p.counters[0], 1ULL);
+            }
+        }
+    }
+    ptx::tc_fence_before();
+    __syncthreads();
+    if (warp == kMma) ptx::tmem_dealloc(sh.tmem_base, p.tmem_cols);
+}
+
+// weights [cout][kd][kh][kw][cin] bf16 -> [nc][kb][ks][2][Nc][8] per the layer's A mode
+__global__ void pack_gen_kernel(const __nv_bfloat16 *__restrict__ w, __nv_bfloat16 *__restrict__ out, int cout, int cin,
+                                int kd, int kh, int kw, int amode, int Nc, int nkb, int nks) {
+    const long long total = (long long)(cout / Nc) * nkb * nks * 2 * Nc * 8;
+    const int taps = kd * kh * kw;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+        long long r = i;
+        const int e = (int)(r % 8); r /= 8;
+        const int col = (int)(r % Nc); r /= Nc;
+        const int j = (int)(r % 2); r /= 2;
+        const int q = (int)(r % nks); r /= nks;
+        const int kb = (int)(r % nkb);
+        const int nc = (int)(r / nkb);
+        int tap, ci;
+        if (amode == AM_SW128) { tap = q / 4; ci = kb * 64 + (q % 4) * 16 + j * 8 + e; }
+        else if (amode == AM_PLANES) { const int kpt = (cin + 15) / 16; tap = q / kpt; ci = (q % kpt) * 16 + j * 8 + e; }
+        else {
+            const int np = (kw + 1) / 2, u = q % np, ar = q / np;
+            const int s = 2 * u + j;
+            tap = s < kw ? ar * kw + s : -1;
+            ci = e;
+        }
+        const int co = nc * Nc + col;
+        float v = 0.f;
+        if (tap >= 0 && tap < taps && ci < cin) v = __bfloat162float(w[((long long)co * taps + tap) * cin + ci]);
+        out[i] = __float2bfloat16_rn(v);
+    }
+}
+
+}  // namespace gen
+
+// ------------------------------------------------------------------------------------------------ host
+static int gen_amode(int cin) {
+    if (cin <= 8) return gen::AM_PAIR;
+    if (cin % 64 == 0) return gen::AM_SW128;
+    if (cin % 16 == 0 && cin < 64) return gen::AM_PLANES;
+    return -1;
+}
+
+constexpr int kGenInBudget = 112 * 1024;   // input-stage ring
+constexpr int kGenWStage = 32 * 1024;      // one weight stage
+constexpr int kGenW = 3;                   // weight stages
+
+// Per-layer tile geometry of the generic kernel.  Returns false if the layer cannot run on it.
+static bool gen_layer_geom(const Layer &ly, int nsp, const bdl_layout &lo_out, gen::LayerP &G) {
+    const bdl_layer &l = ly.L;
+    if (l.kind != BDL_OP_CONV) return false;
+    G.amode = gen_amode(l.cin);
+    if (G.amode < 0 || l.cout % 16 != 0) return false;
+    for (int d = 0; d < 3; d++) {
+        G.k[d] = l.k[d];
+        G.s[d] = l.stride[d];
+        G.pd[d] = l.pad[d];
+        if (G.k[d] > 7 || (G.s[d] != 1 && G.s[d] != 2)) return false;
+        G.in_ext[d] = ly.in_ext[d + 1];
+        G.out_ext[d] = ly.out_ext[d + 1];
+    }
+    if (nsp == 2 && (G.k[0] != 1 || G.s[0] != 1 || G.pd[0] != 0)) return false;
+    if (G.s[0] != 1) return false;   // depth stride: not needed by the workloads
+    G.cin = l.cin;
+    G.cout = l.cout;
+    G.grid[0] = (int)(lo_out.nb[1] * lo_out.Bd);
+    G.grid[1] = (int)(lo_out.nb[2] * lo_out.Bh);
+    G.grid[2] = (int)(lo_out.nb[3] * lo_out.Bw);
+    G.Nc = l.cout <= 256 ? l.cout : 256;
+    if (l.cout % G.Nc) return false;
+    G.nnc = l.cout / G.Nc;
+    const int taps = G.k[0] * G.k[1] * G.k[2];
+    if (G.amode == gen::AM_SW128) { G.nkb = l.cin / 64; G.kc = 8; G.nks = taps * 4; G.row_u = 8; }
+    else if (G.amode == gen::AM_PLANES) { G.nkb = 1; G.kc = l.cin / 8; G.nks = taps * ((l.cin + 15) / 16); G.row_u = 1; }
+    else { G.nkb = 1; G.kc = 1; G.nks = G.k[0] * G.k[1] * ((G.k[2] + 1) / 2); G.row_u = 1; }
+    if (G.nks > gen::kMaxKs) return false;
+    const int ks_bytes = 2 * G.Nc * 16;
+    G.kpw = std::max(1, std::min(G.nks, kGenWStage / ks_bytes));
+    G.nws = (G.nks + G.kpw - 1) / G.kpw;
+    G.idesc = ptx::idesc_bf16_f32(128, G.Nc);
+    G.nblk = G.s[1] * G.s[2];
+    const int Bw = lo_out.Bw;
+    double best = -1e30;
+    bool found = false;
+    gen::LayerP cand = G;
+    const int Hg = G.grid[1], Wg = G.grid[2];
+    for (int Tb = std::min(Hg, 32); Tb >= 1; Tb--) {
+        for (int Tw = Wg; Tw >= std::min(Bw, Wg); Tw -= Bw) {
+            cand.Tb = Tb;
+            cand.Tw = Tw;
+            cand.in_rows = (Tb - 1) * G.s[1] + G.k[1];
+            cand.in_cols = (Tw - 1) * G.s[2] + G.k[2];
+            cand.Wp = (cand.in_cols + G.s[2] - 1) / G.s[2];
+            cand.rb = (cand.in_rows + G.s[1] - 1) / G.s[1];
+            cand.blk_px = cand.rb * cand.Wp;
+            cand.plane_px = cand.nblk * cand.blk_px;
+            const int M = Tb * cand.Wp;
+            cand.ntl = (M + 127) / 128;
+            if (cand.ntl * G.Nc > 256) continue;       // double-buffered accumulators
+            const int max_tap = (G.k[0] - 1) * cand.plane_px + (cand.nblk - 1) * cand.blk_px +
+                                ((G.k[1] - 1) / G.s[1]) * cand.Wp + (G.k[2] - 1) / G.s[2];
+            int rows = std::max(G.k[0] * cand.plane_px, max_tap + cand.ntl * 128);
+            rows = (rows + 7) / 8 * 8;
+            if (G.amode == gen::AM_PLANES) rows += 1;   // odd plane stride: conflict-free loader stores
+            cand.rowsA = rows;
+            cand.stage_bytes = G.amode == gen::AM_SW128 ? rows * 128 : (G.amode == gen::AM_PLANES ? G.kc * rows * 16 : rows * 16);
+            cand.stage_bytes = (cand.stage_bytes + 1023) / 1024 * 1024;
+            if (cand.stage_bytes * 2 > kGenInBudget) continue;
+            cand.ntd = G.grid[0];
+            cand.nty = (Hg + Tb - 1) / Tb;
+            cand.ntx = (Wg + Tw - 1) / Tw;
+            // useful fraction of the MMA rows, then fewer loaded halo pixels per output
+            const double useful = (double)G.out_ext[1] * G.out_ext[2] /
+                                  ((double)cand.nty * cand.ntx * cand.ntl * 128.0);
+            const double halo = (double)cand.in_rows * cand.in_cols / ((double)Tb * Tw * G.s[1] * G.s[2]);
+            const double score = useful - 0.1 * (halo - 1.0) + 1e-4 * Tb * Tw;
+            if (score > best) {
+                best = score;
+                G = cand;
+                found = true;
+            }
+        }
+    }
+    return found;
+}
+
+struct GenGeom {
+    gen::LayerP layer[kMaxLayers];
+    int L;
+    int nin, in_stride, nw, w_stride, acc_stride, nacc, tmem_cols, smem;
+};
+
+static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, GenGeom &g) {
+    g.L = nconv;
+    int in_stride = 0, w_stride = 0, acc = 0;
+    for (int j = 0; j < nconv; j++) {
+        const Layer &ly = p->layers[sg.first + j];
+        bdl_layout lo;
+        bdl_layout_init(&lo, p->in_layout.nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
+                        p->in_layout.Bn, p->in_layout.Bd, p->in_layout.Bh, p->in_layout.Bw, BDL_BF16);
+        gen::LayerP &G = g.layer[j];
+        memset(&G, 0, sizeof(G));
+        if (!gen_layer_geom(ly, p->in_layout.nsp, lo, G)) return false;
+        in_stride = std::max(in_stride, G.stage_bytes);
+        w_stride = std::max(w_stride, G.kpw * 2 * G.Nc * 16);
+        acc = std::max(acc, G.ntl * G.Nc);
+        G.ntasks = (long long)ly.out_ext[0] * G.ntd * G.nty * G.ntx * G.nnc;
+    }
+    g.in_stride = in_stride;
+    g.w_stride = (w_stride + 1023) / 1024 * 1024;
+    g.nin = std::min(gen::kMaxIn, kGenInBudget / in_stride);
+    g.nw = kGenW;
+    g.acc_stride = acc;
+    g.nacc = 2 * acc <= 512 ? 2 : 1;
+    g.tmem_cols = 32;
+    while (g.tmem_cols < g.nacc * acc) g.tmem_cols *= 2;
+    g.smem = g.nin * in_stride + g.nw * g.w_stride + 1024;
+    return g.nin >= 2 && g.smem <= 227 * 1024 - (int)sizeof(gen::Shared) - 1024;
+}
+
+// Number of leading conv layers of subgraph sg the generic kernel runs (a trailing pool runs after it
+// on the CUDA-core layer kernel), or 0 if it cannot run the subgraph.
+int gen_conv_layers(const bdl_plan *p, const Subgraph &sg) {
+    if (p->in_layout.dtype != BDL_BF16 || p->in_layout.Bn != 1) return 0;
+    int L = sg.last - sg.first + 1;
+    if (p->layers[sg.last].L.kind == BDL_OP_MAXPOOL) L--;
+    if (L < 1 || L > kMaxLayers) return 0;
+    for (int j = 0; j < L; j++) {
+        if (p->layers[sg.first + j].L.kind != BDL_OP_CONV) return 0;
+        int rt = sg.res_tensor[j];
+        if (p->layers[sg.first + j].L.residual != BDL_NO_RESIDUAL && rt < 0) return 0;
+    }
+    GenGeom g;
+    return gen_geometry(p, sg, L, g) ? L : 0;
+}
+
+// Tasks (memo status words) of conv layer j of the generic kernel's subgraph.
+int64_t gen_layer_tasks(const bdl_plan *p, const Subgraph &sg, int j) {
+    const int L = gen_conv_layers(p, sg);
+    if (j >= L) return 0;
+    GenGeom g;
+    gen_geometry(p, sg, L, g);
+    return g.layer[j].ntasks;
+}
+
+size_t gen_packed_bytes(const bdl_plan *p, const Subgraph &sg, int j) {
+    const int L = gen_conv_layers(p, sg);
+    if (j >= L) return 0;
+    GenGeom g;
+    gen_geometry(p, sg, L, g);
+    const gen::LayerP &G = g.layer[j];
+    return (size_t)G.nnc * G.nkb * G.nks * 2 * G.Nc * 8 * 2;
+}
+
+// Topological task order: images in groups (enough tiles in flight to fill the GPU, intermediates of a
+// group L2-resident), layer by layer within a group.
+std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
+    const int L = gen_conv_layers(p, sg);
+    std::vector<int> ord;
+    if (L <= 0) return ord;
+    GenGeom g;
+    gen_geometry(p, sg, L, g);
+    const int N = p->layers[sg.first].in_ext[0];
+    long long per_img0 = g.layer[0].ntasks / N;
+    int G = (int)std::max<long long>(1, (2LL * p->num_sms + per_img0 - 1) / std::max<long long>(1, per_img0));
+    G = std::min(G, N);
+    for (int n0 = 0; n0 < N; n0 += G)
+        for (int j = 0; j < L; j++) {
+            const long long per = g.layer[j].ntasks / N;
+            for (int n = n0; n < std::min(N, n0 + G); n++)
+                for (long long t = 0; t < per; t++) ord.push_back((j << 26) | (int)(n * per + t));
+        }
+    return ord;
+}
+
+bdl_status launch_pack_gen(const bdl_plan *p, const Subgraph &sg, int j, void *w_out, cudaStream_t s) {
+    const int L = gen_conv_layers(p, sg);
+    GenGeom g;
+    gen_geometry(p, sg, L, g);
+    const gen::LayerP &G = g.layer[j];
+    const bdl_layer &l = p->layers[sg.first + j].L;
+    const long long total = (long long)G.nnc * G.nkb * G.nks * 2 * G.Nc * 8;
+    const int grid = (int)std::min<long long>((total + 255) / 256, 4096);
+    gen::pack_gen_kernel<<<grid, 256, 0, s>>>((const __nv_bfloat16 *)l.w, (__nv_bfloat16 *)w_out, l.cout, l.cin, l.k[0],
+                                              l.k[1], l.k[2], G.amode, G.Nc, G.nkb, G.nks);
+    BDL_CUDA_CHECK_LAUNCH("pack_gen");
+    return BDL_OK;
+}
+
+bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &in, const TView &out,
+                                 const std::vector<TView> &res_views, unsigned char *ws, cudaStream_t s, int *launches);
+
+bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out,
+                               const std::vector<TView> &res, unsigned char *wsp, cudaStream_t s, int *launches) {
+    const int L = gen_conv_layers(p, sg);
+    if (L <= 0) return fail(BDL_EUNSUPPORTED, "generic tcgen05 kernel: subgraph not supported");
+    const bool pool_tail = L < sg.last - sg.first + 1;
+    GenGeom g;
+    gen_geometry(p, sg, L, g);
+    gen::Params P;
+    memset(&P, 0, sizeof(P));
+    P.L = L;
+    const int nsp = p->in_layout.nsp;
+    std::vector<TView> outs(L);
+    for (int j = 0; j < L; j++) {
+        const Layer &ly = p->layers[sg.first + j];
+        gen::LayerP &G = P.layer[j];
+        G = g.layer[j];
+        if (j == L - 1 && !pool_tail) {
+            outs[j] = out;
+        } else {
+            bdl_layout lo;
+            bdl_layout_init(&lo, nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
+                            p->in_layout.Bn, p->in_layout.Bd, p->in_layout.Bh, p->in_layout.Bw, BDL_BF16);
+            outs[j] = make_view(lo, wsp + sg.memo_off[j]);
+        }
+        G.src = j == 0 ? in : outs[j - 1];
+        G.out = outs[j];
+        G.has_res = sg.res_tensor[j] >= 0;
+        if (G.has_res) G.res = res[j];
+        G.relu = ly.L.relu;
+        G.w = (const __nv_bfloat16 *)(wsp + ly.tc_w_off);
+        G.bias = (const float *)(wsp + ly.b_off);
+        G.task_base = sg.task_base[j];
+    }
+    P.nin = g.nin;
+    P.in_stride = g.in_stride;
+    P.nw = g.nw;
+    P.w_stride = g.w_stride;
+    P.nacc = g.nacc;
+    P.acc_stride = g.acc_stride;
+    P.tmem_cols = g.tmem_cols;
+    P.status = (int *)(wsp + sg.status_off);
+    P.epoch = sg.epoch;
+    P.counters = (unsigned long long *)(wsp + sg.counter_off);
+    cudaFuncSetAttribute(gen::gen_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
+    const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;
+    if (!unmerged) {
+        P.only_layer = -1;
+        P.order = (const int *)(wsp + sg.order_off);
+        P.norder = sg.norder;
+        const int grid = (int)std::min<long long>(P.norder, p->num_sms);
+        P.ticket_base = sg.ticket_base;
+        sg.ticket_base += (unsigned long long)P.norder + grid;
+        launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+        *launches += 1;
+    } else {
+        P.order = nullptr;
+        for (int j = 0; j < L; j++) {
+            P.only_layer = j;
+            P.norder = P.layer[j].ntasks;
+            const int grid = (int)std::min<long long>(P.norder, p->num_sms);
+            P.ticket_base = sg.ticket_base;
+            sg.ticket_base += (unsigned long long)P.norder + grid;
+            launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+            *launches += 1;
+        }
+    }
+    BDL_CUDA_CHECK_LAUNCH("generic tcgen05 kernel");
+    if (pool_tail) {   // trailing pool: CUDA-core layer kernel on the materialized conv output
+        Subgraph ps;
+        ps.first = ps.last = sg.last;
+        ps.mode = BDL_MODE_UNMERGED;
+        ps.res_tensor = {-1};
+        ps.status_off = sg.status_off;
+        ps.counter_off = sg.counter_off + 64;   // the pool's own counters
+        ps.task_base = {0};
+        ps.scratch_off = -1;
+        ps.grid = 4 * p->num_sms;
+        std::vector<TView> nores(1);
+        return launch_brick_subgraph(p, ps, outs[L - 1], out, nores, wsp, s, launches);
+    }
+    return BDL_OK;
+}
+
+int gen_launches(const bdl_plan *p, const Subgraph &sg) {
+    const int L = gen_conv_layers(p, sg);
+    const bool pool_tail = L < sg.last - sg.first + 1;
+    const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;
+    return (unmerged ? L : 1) + (pool_tail ? 1 : 0);
+}
+
+}  // namespace bdl

@@ -118,6 +118,15 @@ namespace bdl {
 int tc_band_rows(const bdl_plan *p, const Subgraph &sg, int *smem_out);
 int ws_band_rows(const bdl_plan *p, const Subgraph &sg);
 std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg);
+int gen_conv_layers(const bdl_plan *p, const Subgraph &sg);
+int64_t gen_layer_tasks(const bdl_plan *p, const Subgraph &sg, int j);
+size_t gen_packed_bytes(const bdl_plan *p, const Subgraph &sg, int j);
+std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg);
+
+int effective_kernel(const Subgraph &sg) {
+    if (sg.kernel == KERNEL_TC_GEN && sg.mode == BDL_MODE_PADDED && sg.gen_layers > 1) return KERNEL_BRICK;
+    return sg.kernel;
+}
 }
 using namespace bdl;
 
@@ -352,7 +361,10 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
     }
     p->tensors.back().ws_off = -1;  // graph output is the user's buffer
     p->out_layout = p->tensors.back().layout;
-    for (auto &sg : p->sgs) sg.kernel = tc_eligible(p, sg) ? KERNEL_TC_BAND : KERNEL_BRICK;
+    for (auto &sg : p->sgs) {
+        sg.kernel = tc_eligible(p, sg) ? KERNEL_TC_BAND : KERNEL_BRICK;
+        if (sg.kernel == KERNEL_BRICK && (sg.gen_layers = gen_conv_layers(p, sg)) > 0) sg.kernel = KERNEL_TC_GEN;
+    }
 
     // ---- workspace layout
     int64_t off = 0;
@@ -374,6 +386,8 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
                 int64_t taps = (int64_t)L.L.k[0] * L.L.k[1] * L.L.k[2];
                 L.tc_w_off = take(taps * L.L.cin * L.L.cout * 2);
             }
+        else if (sg.kernel == KERNEL_TC_GEN)
+            for (int j = 0; j < sg.gen_layers; j++) p->layers[sg.first + j].tc_w_off = take(gen_packed_bytes(p, sg, j));
     for (size_t t = 1; t + 1 < p->tensors.size(); t++) p->tensors[t].ws_off = take(p->tensors[t].layout.total_bytes);
     for (auto &sg : p->sgs) {
         int L = sg.last - sg.first + 1;
@@ -388,11 +402,13 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             if (j < L - 1) sg.memo_off[j] = take(lo.total_bytes);
             sg.task_base[j] = words;
             // memo tags: one per brick, or per band task of the tcgen05 kernels (bands of >= 1 row)
-            words += std::max<int64_t>(lo.nbricks, lo.N * lo.D * lo.H * lo.nb[3]);
+            int64_t w = std::max<int64_t>(lo.nbricks, lo.N * lo.D * lo.H * lo.nb[3]);
+            if (sg.kernel == KERNEL_TC_GEN) w = std::max<int64_t>(w, gen_layer_tasks(p, sg, j));
+            words += w;
         }
         sg.ntasks_total = words;
         sg.status_off = take(words * 4);
-        sg.counter_off = take(8 * 8);
+        sg.counter_off = take(16 * 8);   // [0..7] subgraph kernel, [8..15] trailing-pool kernel
         // padded-mode scratch for the CUDA-core kernel: two ping-pong region buffers per CTA
         int64_t maxvol = 1;
         {
@@ -414,6 +430,10 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             sg.order_host = ws_task_order(p, sg);
             sg.norder = (int64_t)sg.order_host.size();
             sg.order_off = sg.norder ? take(sg.norder * 4) : -1;
+        } else if (sg.kernel == KERNEL_TC_GEN) {
+            sg.order_host = gen_task_order(p, sg);
+            sg.norder = (int64_t)sg.order_host.size();
+            sg.order_off = sg.norder ? take(sg.norder * 4) : -1;
         }
     }
     p->ws_bytes = align_up(off, 256);
@@ -432,7 +452,7 @@ bdl_status bdl_plan_subgraph(const bdl_plan *p, int32_t i, int32_t *first, int32
     if (mode) *mode = s.mode;
     if (mbrick) *mbrick = s.model_brick;
     if (delta) *delta = s.delta;
-    if (kernel) *kernel = s.kernel;
+    if (kernel) *kernel = effective_kernel(s);
     return BDL_OK;
 }
 

@@ -20,6 +20,10 @@ bdl_status launch_tc_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
 bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out, const TView *res,
                               unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged);
 int tc_launches(const bdl_plan *p, const Subgraph &sg);
+bdl_status launch_pack_gen(const bdl_plan *p, const Subgraph &sg, int j, void *w_out, cudaStream_t s);
+bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out,
+                               const std::vector<TView> &res, unsigned char *wsp, cudaStream_t s, int *launches);
+int gen_launches(const bdl_plan *p, const Subgraph &sg);
 
 static void *tensor_ptr(const bdl_plan *p, int t, const void *in_b, void *out_b, unsigned char *ws) {
     const Tensor &T = p->tensors[t];
@@ -43,8 +47,13 @@ bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream) {
         if (L.L.kind != BDL_OP_CONV) continue;
         bdl_status st = launch_pack_f32(L.L, p->in_layout.dtype, (float *)(ws + L.w_off), (float *)(ws + L.b_off), s);
         if (st != BDL_OK) return st;
-        if (L.tc_w_off >= 0) {
-            st = launch_pack_tc(L.L, ws + L.tc_w_off, s);
+    }
+    for (auto &sg : p->sgs) {
+        for (int j = sg.first; j <= sg.last; j++) {
+            const Layer &L = p->layers[j];
+            if (L.tc_w_off < 0) continue;
+            bdl_status st = sg.kernel == KERNEL_TC_GEN ? launch_pack_gen(p, sg, j - sg.first, ws + L.tc_w_off, s)
+                                                       : launch_pack_tc(L.L, ws + L.tc_w_off, s);
             if (st != BDL_OK) return st;
         }
     }
@@ -52,7 +61,7 @@ bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream) {
         if (sg.order_off >= 0)
             cudaMemcpyAsync(ws + sg.order_off, sg.order_host.data(), sg.norder * 4, cudaMemcpyHostToDevice, s);
         cudaMemsetAsync(ws + sg.status_off, 0, sg.ntasks_total * 4, s);
-        cudaMemsetAsync(ws + sg.counter_off, 0, 64, s);
+        cudaMemsetAsync(ws + sg.counter_off, 0, 128, s);
         sg.ticket_base = 0;
         sg.epoch = 0;
     }
@@ -86,7 +95,9 @@ bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void
         tc_res = &res[j];
     }
     int launches = 0;
-    if (sg.kernel == KERNEL_TC_BAND) {
+    const int kern = effective_kernel(sg);
+    if (kern == KERNEL_TC_GEN) return launch_gen_subgraph(p, sg, vin, vout, res, ws, s, &launches);
+    if (kern == KERNEL_TC_BAND) {
         const bool single = sg.first == sg.last;
         if (sg.mode == BDL_MODE_PADDED && !single) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
         static const bool legacy = getenv("BDL_TC_LEGACY") != nullptr;  // A/B against the synchronous kernel
@@ -111,7 +122,9 @@ int32_t bdl_plan_launches_per_run(const bdl_plan *p) {
     int n = 0;
     for (auto &sg : p->sgs) {
         int L = sg.last - sg.first + 1;
-        if (sg.kernel == KERNEL_TC_BAND) n += tc_launches(p, sg);
+        const int k = effective_kernel(sg);
+        if (k == KERNEL_TC_BAND) n += tc_launches(p, sg);
+        else if (k == KERNEL_TC_GEN) n += gen_launches(p, sg);
         else n += (sg.mode == BDL_MODE_UNMERGED || L == 1) ? L : 1;
     }
     return n;

@@ -31,7 +31,7 @@ import math
 
 import torch
 
-__all__ = ["CONFIGS", "make_layers", "make_workload", "layer_out_shape"]
+__all__ = ["CONFIGS", "make_layers", "make_workload", "make_graph_workload", "conv", "pool", "layer_out_shape"]
 
 CONFIGS = {
     "cfg1": dict(nsp=2, N=1, C=8, D=1, H=32, W=32, dtype="f32", brick=(1, 1, 8, 8)),
@@ -128,15 +128,35 @@ def make_workload(cfg: str, N=None, C=None, D=None, H=None, W=None, nlayers=None
             c[k] = v
     num = _CFG_NUM[cfg] + seed_offset
     layers = make_layers(cfg, C=c["C"], nlayers=nlayers)
-    bf16 = c["dtype"] == "bf16"
+    wl = make_graph_workload(layers, c["N"], c["C"], c["D"], c["H"], c["W"], c["nsp"], c["brick"], c["dtype"],
+                             seed=num, input_seed_offset=input_seed_offset)
+    wl["cfg"] = cfg
+    return wl
 
-    g = torch.Generator().manual_seed(1000 + num + 100 * input_seed_offset)  # per-shard inputs (ranks)
-    x = torch.randn(c["N"], c["C"], c["D"], c["H"], c["W"], generator=g, dtype=torch.float32)
+
+def conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2):
+    """Layer dict of a conv (public form of the graph builder used by the configurations)."""
+    return _conv(cin, cout, k, s, p, relu, inp, res, wscale, nsp)
+
+
+def pool(c, k, s, p):
+    return _pool(c, k, s, p)
+
+
+def make_graph_workload(layers, N, C, D, H, W, nsp, brick, dtype, seed=0, input_seed_offset=0):
+    """Seeded synthetic input, weights and biases for an arbitrary layer graph (same recipe as the
+    configurations: seeds 1000/2000/3000 + seed)."""
+    layers = [dict(l) for l in layers]
+    for i, l in enumerate(layers):
+        if l["input"] is None:
+            l["input"] = i - 1
+    bf16 = dtype == "bf16"
+    g = torch.Generator().manual_seed(1000 + seed + 100 * input_seed_offset)  # per-shard inputs (ranks)
+    x = torch.randn(N, C, D, H, W, generator=g, dtype=torch.float32)
     if bf16:
         x = x.to(torch.bfloat16).to(torch.float32)
-
-    gw = torch.Generator().manual_seed(2000 + num)
-    gb = torch.Generator().manual_seed(3000 + num)
+    gw = torch.Generator().manual_seed(2000 + seed)
+    gb = torch.Generator().manual_seed(3000 + seed)
     weights, biases = [], []
     for l in layers:
         if l["kind"] != "conv":
@@ -152,6 +172,5 @@ def make_workload(cfg: str, N=None, C=None, D=None, H=None, W=None, nlayers=None
         b = (torch.rand(l["cout"], generator=gb, dtype=torch.float32) * 0.2 - 0.1)
         weights.append(w)
         biases.append(b)
-    return dict(cfg=cfg, nsp=c["nsp"], dtype=c["dtype"], N=c["N"], C=c["C"], D=c["D"],
-                H=c["H"], W=c["W"], brick=c["brick"], layers=layers, x=x,
-                weights=weights, biases=biases)
+    return dict(cfg="custom", nsp=nsp, dtype=dtype, N=N, C=C, D=D, H=H, W=W, brick=tuple(brick), layers=layers,
+                x=x, weights=weights, biases=biases)
