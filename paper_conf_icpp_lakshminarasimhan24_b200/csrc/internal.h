@@ -61,6 +61,7 @@ struct Subgraph {
     double delta, delta_first;
     int kernel;                 // KernelKind the subgraph is able to run on
     int gen_layers = 0;         // generic tcgen05 kernel: leading conv layers it runs (a pool tail follows)
+    int64_t gen_scr_off = -1;   // generic tcgen05 kernel, padded mode: per-CTA region scratch
     int in_tensor;              // index into Plan::tensors
     int out_tensor;
     std::vector<int> res_tensor;   // per layer in subgraph: tensor index of external residual, or -1
@@ -106,8 +107,7 @@ namespace bdl {
 void set_error(const std::string &msg);
 bdl_status fail(bdl_status s, const std::string &msg);
 bool layout_valid(const bdl_layout *l);
-// kernel that actually executes subgraph sg in its current mode (padded multi-layer subgraphs that the
-// generic tcgen05 kernel cannot run in padded form use the CUDA-core brick kernel)
+// kernel that actually executes subgraph sg in its current mode
 int effective_kernel(const Subgraph &sg);
 TView make_view(const bdl_layout &l, void *ptr);
 }  // namespace bdl

@@ -61,6 +61,8 @@ struct LayerP {
     int ntl;
     uint32_t idesc;
     long long task_base, ntasks;
+    int pR[3];                // padded: largest region of this layer's output (scratch pitches)
+    long long scr_off;        // padded: byte offset of the layer's region buffer in a scratch slot
 };
 
 struct Params {
@@ -75,6 +77,13 @@ struct Params {
     const int *order;                    // (l << 26) | task, or null (unmerged)
     long long norder;
     int only_layer;
+    // padded mode (§3.2.1): a task is a PB block of the last layer's output; every layer's
+    // halo-extended region is recomputed by the CTA into its private scratch (two slots, so two blocks
+    // interleave and one block's loads overlap the other's MMAs)
+    int padded;
+    int PB[3], npb[3];
+    unsigned char *scratch;
+    long long scr_slot;
 };
 
 struct Shared {
@@ -83,8 +92,9 @@ struct Shared {
     uint64_t acc_full[2], acc_empty[2];
     uint64_t desc_full[kRing];
     uint32_t tmem_base;
-    int q_l[kQ];
+    int q_l[kQ], q_w[kQ];                // q_w: padded: sub-task seq whose epilogue must be done first
     long long q_t[kQ];
+    int done_seq;                        // padded: sub-tasks whose epilogue stores are complete
     int desc_l[kRing];
     long long desc_t[kRing];
     int stk_l[kStack];
@@ -153,7 +163,140 @@ __device__ __forceinline__ long long dep_task(const Params &p, int l, const DepR
     return ((((long long)r.n * P.ntd + d) * P.nty + b) * P.ntx + x) * P.nnc + c;
 }
 
+// Padded mode: region of layer l's output needed for block (bd, by, bx) of the last layer (Fig 4:
+// reverse traversal, input extent s*(O-1) + k, clipped to the feature map).  lo/hi: [lo, hi) per dim.
+__host__ __device__ inline void region_of(const LayerP *ly, int L, const int PB[3], const int blk[3], int l, int lo[3],
+                                          int hi[3]) {
+    for (int d = 0; d < 3; d++) {
+        lo[d] = blk[d] * PB[d];
+        hi[d] = lo[d] + PB[d] < ly[L - 1].grid[d] ? lo[d] + PB[d] : ly[L - 1].grid[d];
+    }
+    for (int j = L - 1; j > l; j--) {
+        const LayerP &J = ly[j];
+        for (int d = 0; d < 3; d++) {
+            const int h = hi[d] < J.out_ext[d] ? hi[d] : J.out_ext[d];
+            if (h <= lo[d]) {
+                lo[d] = hi[d] = 0;
+                continue;
+            }
+            const int nlo = lo[d] * J.s[d] - J.pd[d], nhi = (h - 1) * J.s[d] - J.pd[d] + J.k[d];
+            lo[d] = nlo > 0 ? nlo : 0;
+            hi[d] = nhi < J.in_ext[d] ? nhi : J.in_ext[d];
+            if (hi[d] < lo[d]) hi[d] = lo[d];
+        }
+    }
+}
+__host__ __device__ inline int region_subtiles(const LayerP &L, const int lo[3], const int hi[3]) {
+    const int a = hi[0] - lo[0], b = hi[1] - lo[1], c = hi[2] - lo[2];
+    if (a <= 0 || b <= 0 || c <= 0) return 0;
+    return a * ((b + L.Tb - 1) / L.Tb) * ((c + L.Tw - 1) / L.Tw) * L.nnc;
+}
+
+// One unit of work of the pipeline: an output tile of layer l (memoized/unmerged: a tile of the bricked
+// grid; padded: a tile of a block's region), with where its input comes from and its output goes.
+struct Tile {
+    int n, d, y0, x0, nc;
+    int hi[3];                 // exclusive bounds of the positions this tile writes
+    int src_scr, dst_scr;      // padded: input / output in the CTA's scratch
+    int slo[3], shi[3];        // source region (scratch) bounds
+    int dlo[3];                // destination region origin (scratch)
+    int slot;
+};
+__device__ __forceinline__ Tile make_tile(const Params &p, int l, long long t) {
+    const LayerP &L = p.layer[l];
+    Tile T;
+    if (!p.padded) {
+        const TaskC c = decode(L, t);
+        T.n = c.n; T.d = c.d; T.y0 = c.ty * L.Tb; T.x0 = c.tx * L.Tw; T.nc = c.nc;
+        T.hi[0] = L.grid[0]; T.hi[1] = L.grid[1]; T.hi[2] = L.grid[2];
+        T.src_scr = T.dst_scr = 0;
+        T.slot = 0;
+        return T;
+    }
+    // t = ((P << 16 | k) << 8 | nc) << 1 | slot
+    T.slot = (int)(t & 1);
+    T.nc = (int)((t >> 1) & 0xFF);
+    int k = (int)((t >> 9) & 0xFFFF);
+    long long P = t >> 25;
+    int blk[3];
+    blk[2] = (int)(P % p.npb[2]); P /= p.npb[2];
+    blk[1] = (int)(P % p.npb[1]); P /= p.npb[1];
+    blk[0] = (int)(P % p.npb[0]);
+    T.n = (int)(P / p.npb[0]);
+    int lo[3], hi[3];
+    region_of(p.layer, p.L, p.PB, blk, l, lo, hi);
+    const int nty = (hi[1] - lo[1] + L.Tb - 1) / L.Tb, ntx = (hi[2] - lo[2] + L.Tw - 1) / L.Tw;
+    const int kx = k % ntx; k /= ntx;
+    const int ky = k % nty;
+    const int kd = k / nty;
+    T.d = lo[0] + kd; T.y0 = lo[1] + ky * L.Tb; T.x0 = lo[2] + kx * L.Tw;
+    for (int d = 0; d < 3; d++) { T.hi[d] = hi[d]; T.dlo[d] = lo[d]; }
+    T.dst_scr = l < p.L - 1;
+    T.src_scr = l > 0;
+    if (T.src_scr) region_of(p.layer, p.L, p.PB, blk, l - 1, T.slo, T.shi);
+    return T;
+}
+__device__ __forceinline__ unsigned char *scr_slot(const Params &p, int slot) {
+    return p.scratch + ((long long)blockIdx.x * 2 + slot) * p.scr_slot;
+}
+
 // ---------------------------------------------------------------------------------------------- scheduler
+__device__ void scheduler_padded(const Params &p, Shared &sh) {
+    const int lane = threadIdx.x % 32;
+    uint32_t qseq = 0;
+    auto emit = [&](int l, long long t, int wait) {
+        const int slot = qseq % kQ;
+        if (qseq >= (uint32_t)kQ) ptx::mbar_wait(&sh.q_empty[slot], ((qseq / kQ) - 1) & 1);
+        if (lane == 0) {
+            sh.q_l[slot] = l;
+            sh.q_t[slot] = t;
+            sh.q_w[slot] = wait;
+            mbar_arrive(&sh.q_full[slot]);
+        }
+        __syncwarp();
+        qseq++;
+    };
+    unsigned long long computed = 0;
+    for (;;) {
+        // two blocks at a time: their layers interleave (A.l0, B.l0, A.l1, B.l1, ...) so that a layer's
+        // loads wait for the previous layer of the same block while the other block's MMAs run
+        // one ticket draw per pair, so every CTA overshoots by exactly one draw and the counter
+        // advance per run is deterministic (2*ceil(norder/2) + 2*grid; the host offsets ticket_base)
+        long long P[2];
+        int np = 0;
+        unsigned long long tk = 0;
+        if (lane == 0) tk = atomicAdd(&p.counters[4], 2ULL) - p.ticket_base;
+        tk = __shfl_sync(0xffffffff, tk, 0);
+        if ((long long)tk < 0) __trap();   // ticket accounting broken: fail loudly
+        for (int i = 0; i < 2; i++)
+            if ((long long)(tk + i) < p.norder) P[np++] = (long long)(tk + i);
+        if (np == 0) break;
+        int last[2] = {-1, -1};
+        for (int l = 0; l < p.L; l++) {
+            const LayerP &L = p.layer[l];
+            for (int i = 0; i < np; i++) {
+                long long q = P[i];
+                int blk[3];
+                blk[2] = (int)(q % p.npb[2]); q /= p.npb[2];
+                blk[1] = (int)(q % p.npb[1]); q /= p.npb[1];
+                blk[0] = (int)(q % p.npb[0]);
+                int lo[3], hi[3];
+                region_of(p.layer, p.L, p.PB, blk, l, lo, hi);
+                const int nsub = region_subtiles(L, lo, hi);
+                const int wait = last[i];
+                for (int k = 0; k < nsub; k++) {
+                    const int kk = k / L.nnc, nc = k % L.nnc;
+                    emit(l, ((((P[i] << 16) | kk) << 8 | nc) << 1) | i, wait);
+                    last[i] = (int)qseq - 1;
+                }
+                computed += nsub;
+            }
+        }
+    }
+    emit(-1, 0, -1);
+    (void)computed;
+}
+
 __device__ void scheduler(const Params &p, Shared &sh) {
     const int lane = threadIdx.x % 32;
     const unsigned EP = p.epoch << 2;
@@ -167,6 +310,7 @@ __device__ void scheduler(const Params &p, Shared &sh) {
         if (lane == 0) {
             sh.q_l[slot] = l;
             sh.q_t[slot] = t;
+            sh.q_w[slot] = -1;
             mbar_arrive(&sh.q_full[slot]);
         }
         __syncwarp();
@@ -177,6 +321,7 @@ __device__ void scheduler(const Params &p, Shared &sh) {
         if (lane == 0) tk = atomicAdd(&p.counters[4], 1ULL) - p.ticket_base;
         tk = __shfl_sync(0xffffffff, tk, 0);
         if ((long long)tk >= p.norder) break;
+        if ((long long)tk < 0) __trap();   // ticket accounting broken: fail loudly
         int l;
         long long t;
         if (unmerged) {
@@ -250,16 +395,26 @@ __device__ void scheduler(const Params &p, Shared &sh) {
 }
 
 // ---------------------------------------------------------------------------------------------- loader
-// One K-block of the input tile of task (n, d, ty, tx) into stage `buf` (128 threads).
-__device__ __forceinline__ void load_stage(const LayerP &L, const TaskC &c, int kb, uint8_t *buf, int tid) {
+// One K-block of the input tile of a tile into stage `buf` (128 threads).  Positions outside the feature
+// map (and, in padded mode, outside the source region) are zero-filled.
+__device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, const Tile &T, int kb, uint8_t *buf,
+                                           int tid) {
     const TView &v = L.src;
     const __nv_bfloat16 *base = reinterpret_cast<const __nv_bfloat16 *>(v.ptr);
+    const __nv_bfloat16 *sbase = nullptr;
+    int sp1 = 0, sp2 = 0;
+    if (T.src_scr) {
+        const LayerP &S = p.layer[&L - p.layer - 1];
+        sbase = reinterpret_cast<const __nv_bfloat16 *>(scr_slot(p, T.slot) + S.scr_off);
+        sp1 = S.pR[1];
+        sp2 = S.pR[2];
+    }
     const int kc = L.kc;
     const int npx = L.k[0] * L.in_rows * L.in_cols;
     const int total = npx * kc;
-    const int z0 = c.d * L.s[0] - L.pd[0];
-    const int y0 = c.ty * L.Tb * L.s[1] - L.pd[1];
-    const int x0 = c.tx * L.Tw * L.s[2] - L.pd[2];
+    const int z0 = T.d * L.s[0] - L.pd[0];
+    const int y0 = T.y0 * L.s[1] - L.pd[1];
+    const int x0 = T.x0 * L.s[2] - L.pd[2];
     const uint32_t plane_bytes = (uint32_t)L.rowsA * 16;
     for (int it = tid; it < total; it += kLoadT) {
         const int P = it / kc, ch = it - P * kc;
@@ -267,13 +422,21 @@ __device__ __forceinline__ void load_stage(const LayerP &L, const TaskC &c, int 
         const int r2 = P / L.in_cols;
         const int yy = r2 % L.in_rows, a = r2 / L.in_rows;
         const int z = z0 + a, y = y0 + yy, x = x0 + xx;
-        const bool ok = z >= 0 && z < L.in_ext[0] && y >= 0 && y < L.in_ext[1] && x >= 0 && x < L.in_ext[2];
+        bool ok = z >= 0 && z < L.in_ext[0] && y >= 0 && y < L.in_ext[1] && x >= 0 && x < L.in_ext[2];
         const int px = a * L.plane_px + ((yy % L.s[1]) * L.s[2] + (xx % L.s[2])) * L.blk_px + (yy / L.s[1]) * L.Wp +
                        xx / L.s[2];
         uint32_t off;
         if (L.amode == AM_SW128) off = (uint32_t)px * 128 + ((ch ^ (px & 7)) << 4);
         else off = (uint32_t)ch * plane_bytes + (uint32_t)px * 16;
-        const void *g = ok ? (const void *)(base + pix(v, c.n, z, y, x) + kb * 64 + ch * 8) : (const void *)base;
+        const void *g = base;
+        if (T.src_scr) {
+            ok = ok && z >= T.slo[0] && z < T.shi[0] && y >= T.slo[1] && y < T.shi[1] && x >= T.slo[2] && x < T.shi[2];
+            if (ok)
+                g = sbase + ((((long long)(z - T.slo[0]) * sp1 + (y - T.slo[1])) * sp2 + (x - T.slo[2])) * L.cin +
+                             kb * 64 + ch * 8);
+        } else if (ok) {
+            g = base + pix(v, T.n, z, y, x) + kb * 64 + ch * 8;
+        }
         ptx::cp_async16(buf + off, g, ok ? 16u : 0u);
     }
 }
@@ -334,6 +497,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             ptx::mbar_init(&sh.acc_empty[i], kEpiW);
         }
         for (int i = 0; i < kRing; i++) ptx::mbar_init(&sh.desc_full[i], 1);
+        sh.done_seq = 0;
         ptx::fence_barrier_init();
     }
     if (warp == kMma) {
@@ -349,7 +513,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
 
     const unsigned EP = p.epoch << 2;
     if (warp == kSched) {
-        scheduler(p, sh);
+        if (p.padded) scheduler_padded(p, sh);
+        else scheduler(p, sh);
     } else if (warp < kLoad0 + kLW) {
         // ------------------------------------------------------------------ loaders
         const int tid = threadIdx.x - 32 * kLoad0;
@@ -359,7 +524,15 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             ptx::mbar_wait(&sh.q_full[slot], (seq / kQ) & 1);
             const int l = sh.q_l[slot];
             const long long t = sh.q_t[slot];
-            if (l >= 0 && l > 0 && p.only_layer < 0 && warp == kLoad0) {
+            const int wait = sh.q_w[slot];
+            if (l > 0 && p.padded && wait >= 0 && warp == kLoad0) {
+                // padded: the source region is written by this CTA's epilogue of sub-task `wait`
+                if (lane == 0) {
+                    while (*reinterpret_cast<volatile int *>(&sh.done_seq) <= wait) __nanosleep(64);
+                    __threadfence();
+                }
+                __syncwarp();
+            } else if (l > 0 && !p.padded && p.only_layer < 0 && warp == kLoad0) {
                 // wait for the dependency tiles (state 2 of this epoch)
                 const DepRange r = dep_range(p, l, t);
                 const int nd = dep_count(r);
@@ -384,11 +557,11 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             }
             if (l < 0) break;
             const LayerP &L = p.layer[l];
-            const TaskC c = decode(L, t);
+            const Tile T = make_tile(p, l, t);
             for (int kb = 0; kb < L.nkb; kb++, gin++) {
                 const int s = gin % p.nin;
                 if (gin >= (uint32_t)p.nin) ptx::mbar_wait(&sh.in_empty[s], ((gin / p.nin) - 1) & 1);
-                load_stage(L, c, kb, in_ring + (size_t)s * p.in_stride, tid);
+                load_stage(p, L, T, kb, in_ring + (size_t)s * p.in_stride, tid);
                 ptx::cp_async_wait_all();
                 ptx::fence_proxy_async_smem();
                 mbar_arrive(&sh.in_full[s]);
@@ -406,7 +579,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             if (lane == 0) mbar_arrive(&sh.q_empty[slot]);
             if (l < 0) break;
             const LayerP &L = p.layer[l];
-            const int nc = (int)(t % L.nnc);
+            const int nc = p.padded ? (int)((t >> 1) & 0xFF) : (int)(t % L.nnc);
             const size_t ks_bytes = (size_t)2 * L.Nc * 16;
             const uint8_t *wl = reinterpret_cast<const uint8_t *>(L.w) + (size_t)nc * L.nkb * L.nks * ks_bytes;
             for (int kb = 0; kb < L.nkb; kb++) {
@@ -481,7 +654,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             const long long t = sh.desc_t[seq % kRing];
             if (l < 0) break;
             const LayerP &L = p.layer[l];
-            const TaskC c = decode(L, t);
+            const Tile T = make_tile(p, l, t);
             const int a = seq % p.nacc;
             ptx::mbar_wait(&sh.acc_full[a], (seq / p.nacc) & 1);
             ptx::tc_fence_after();
@@ -490,16 +663,17 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             const int items = L.ntl * ncb;
             __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(L.out.ptr);
             const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(L.res.ptr);
-            const int d = c.d;
+            const int d = T.d;
+            __nv_bfloat16 *scr = T.dst_scr ? reinterpret_cast<__nv_bfloat16 *>(scr_slot(p, T.slot) + L.scr_off) : nullptr;
             for (int it = rank; it < items; it += 4) {
                 const int tl = it / ncb, cb = it - tl * ncb;
                 const int m = tl * 128 + quad * 32 + lane;
                 const int i = m / L.Wp, j = m - i * L.Wp;
-                const int y = c.ty * L.Tb + i, x = c.tx * L.Tw + j;
+                const int y = T.y0 + i, x = T.x0 + j;
                 int kind = 0;   // 0 skip, 1 zero (masked), 2 value
-                if (i < L.Tb && j < L.Tw && d < L.grid[0] && y < L.grid[1] && x < L.grid[2])
+                if (i < L.Tb && j < L.Tw && d < T.hi[0] && y < T.hi[1] && x < T.hi[2])
                     kind = (d < L.out_ext[0] && y < L.out_ext[1] && x < L.out_ext[2]) ? 2 : 1;
-                const int ch0 = c.nc * L.Nc + cb * CB;
+                const int ch0 = T.nc * L.Nc + cb * CB;
                 uint32_t r[2][16];
                 const uint32_t taddr = tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) + tl * L.Nc + cb * CB;
                 ptx::tmem_ld16(taddr, r[0]);
@@ -508,12 +682,15 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 ptx::reg_fence16(r[0]);
                 ptx::reg_fence16(r[1]);
                 if (!kind) continue;
-                uint4 *dst = reinterpret_cast<uint4 *>(outp + pix(L.out, c.n, d, y, x) + ch0);
+                uint4 *dst = reinterpret_cast<uint4 *>(
+                    T.dst_scr ? scr + ((((long long)(d - T.dlo[0]) * L.pR[1] + (y - T.dlo[1])) * L.pR[2] + (x - T.dlo[2])) *
+                                           L.cout + ch0)
+                              : outp + pix(L.out, T.n, d, y, x) + ch0);
                 if (kind == 1) {
                     for (int k = 0; k < CB / 8; k++) dst[k] = make_uint4(0, 0, 0, 0);
                     continue;
                 }
-                const uint4 *rs = L.has_res ? reinterpret_cast<const uint4 *>(resp + pix(L.res, c.n, d, y, x) + ch0) : nullptr;
+                const uint4 *rs = L.has_res ? reinterpret_cast<const uint4 *>(resp + pix(L.res, T.n, d, y, x) + ch0) : nullptr;
 #pragma unroll
                 for (int k = 0; k < 4; k++) {
                     if (k >= CB / 8) break;
@@ -547,7 +724,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");
             if (ew == 0 && lane == 0) {
                 __threadfence();
-                if (p.only_layer < 0) st_release(status_word(p, l, t), (int)(EP | 2));
+                if (p.padded) *reinterpret_cast<volatile int *>(&sh.done_seq) = (int)seq + 1;
+                else if (p.only_layer < 0) st_release(status_word(p, l, t), (int)(EP | 2));
                 atomicAdd(&p.counters[0], 1ULL);
             }
         }
@@ -600,8 +778,8 @@ constexpr int kGenInBudget = 112 * 1024;   // input-stage ring
 constexpr int kGenWStage = 32 * 1024;      // one weight stage
 constexpr int kGenW = 3;                   // weight stages
 
-// Per-layer tile geometry of the generic kernel.  Returns false if the layer cannot run on it.
-static bool gen_layer_geom(const Layer &ly, int nsp, const bdl_layout &lo_out, gen::LayerP &G) {
+// Static (tile-independent) fields of a layer.  Returns false if the layer cannot run on the kernel.
+static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out, gen::LayerP &G) {
     const bdl_layer &l = ly.L;
     if (l.kind != BDL_OP_CONV) return false;
     G.amode = gen_amode(l.cin);
@@ -634,13 +812,17 @@ static bool gen_layer_geom(const Layer &ly, int nsp, const bdl_layout &lo_out, g
     G.nws = (G.nks + G.kpw - 1) / G.kpw;
     G.idesc = ptx::idesc_bf16_f32(128, G.Nc);
     G.nblk = G.s[1] * G.s[2];
-    const int Bw = lo_out.Bw;
+    return true;
+}
+
+// Tile geometry: output tiles of Tb rows x Tw columns (Tw a multiple of walign) covering cover_h x
+// cover_w positions of one plane; the best useful fraction of MMA rows that fits the shared memory.
+static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign) {
     double best = -1e30;
     bool found = false;
     gen::LayerP cand = G;
-    const int Hg = G.grid[1], Wg = G.grid[2];
-    for (int Tb = std::min(Hg, 32); Tb >= 1; Tb--) {
-        for (int Tw = Wg; Tw >= std::min(Bw, Wg); Tw -= Bw) {
+    for (int Tb = std::min(cover_h, 32); Tb >= 1; Tb--) {
+        for (int Tw = (cover_w + walign - 1) / walign * walign; Tw >= walign; Tw -= walign) {
             cand.Tb = Tb;
             cand.Tw = Tw;
             cand.in_rows = (Tb - 1) * G.s[1] + G.k[1];
@@ -661,12 +843,9 @@ static bool gen_layer_geom(const Layer &ly, int nsp, const bdl_layout &lo_out, g
             cand.stage_bytes = G.amode == gen::AM_SW128 ? rows * 128 : (G.amode == gen::AM_PLANES ? G.kc * rows * 16 : rows * 16);
             cand.stage_bytes = (cand.stage_bytes + 1023) / 1024 * 1024;
             if (cand.stage_bytes * 2 > kGenInBudget) continue;
-            cand.ntd = G.grid[0];
-            cand.nty = (Hg + Tb - 1) / Tb;
-            cand.ntx = (Wg + Tw - 1) / Tw;
+            const int nty = (cover_h + Tb - 1) / Tb, ntx = (cover_w + Tw - 1) / Tw;
             // useful fraction of the MMA rows, then fewer loaded halo pixels per output
-            const double useful = (double)G.out_ext[1] * G.out_ext[2] /
-                                  ((double)cand.nty * cand.ntx * cand.ntl * 128.0);
+            const double useful = (double)cover_h * cover_w / ((double)nty * ntx * cand.ntl * 128.0);
             const double halo = (double)cand.in_rows * cand.in_cols / ((double)Tb * Tw * G.s[1] * G.s[2]);
             const double score = useful - 0.1 * (halo - 1.0) + 1e-4 * Tb * Tw;
             if (score > best) {
@@ -683,23 +862,66 @@ struct GenGeom {
     gen::LayerP layer[kMaxLayers];
     int L;
     int nin, in_stride, nw, w_stride, acc_stride, nacc, tmem_cols, smem;
+    int PB[3], npb[3];
+    long long scr_slot;
 };
 
-static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, GenGeom &g) {
+static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool padded, GenGeom &g) {
+    memset(&g, 0, sizeof(g));
     g.L = nconv;
-    int in_stride = 0, w_stride = 0, acc = 0;
+    const int nsp = p->in_layout.nsp;
     for (int j = 0; j < nconv; j++) {
         const Layer &ly = p->layers[sg.first + j];
         bdl_layout lo;
-        bdl_layout_init(&lo, p->in_layout.nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
+        bdl_layout_init(&lo, nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
                         p->in_layout.Bn, p->in_layout.Bd, p->in_layout.Bh, p->in_layout.Bw, BDL_BF16);
-        gen::LayerP &G = g.layer[j];
-        memset(&G, 0, sizeof(G));
-        if (!gen_layer_geom(ly, p->in_layout.nsp, lo, G)) return false;
+        if (!gen_layer_static(ly, nsp, lo, g.layer[j])) return false;
+    }
+    if (padded && nconv > 1) {
+        // blocks of the planner's brick edge (rho/tau model, L649-658) over the last layer's grid
+        const gen::LayerP &last = g.layer[nconv - 1];
+        const int B = std::max(1, sg.model_brick);
+        for (int d = 0; d < 3; d++) {
+            const bool spatial = d > 0 || nsp == 3;
+            g.PB[d] = spatial ? std::min(B, last.grid[d]) : 1;
+            g.npb[d] = (last.grid[d] + g.PB[d] - 1) / g.PB[d];
+        }
+        g.scr_slot = 0;
+        for (int j = 0; j < nconv; j++) {
+            gen::LayerP &G = g.layer[j];
+            // largest region of this layer over the blocks (the region is separable per dimension)
+            for (int d = 0; d < 3; d++) {
+                int mx = 0;
+                for (int b = 0; b < g.npb[d]; b++) {
+                    int blk[3] = {0, 0, 0}, lo[3], hi[3];
+                    blk[d] = b;
+                    gen::region_of(g.layer, nconv, g.PB, blk, j, lo, hi);
+                    mx = std::max(mx, hi[d] - lo[d]);
+                }
+                G.pR[d] = std::max(1, mx);
+            }
+            if (!gen_layer_tiles(G, G.pR[1], G.pR[2], 1)) return false;
+            if (j < nconv - 1) {
+                G.scr_off = g.scr_slot;
+                g.scr_slot += ((long long)G.pR[0] * G.pR[1] * G.pR[2] * G.cout * 2 + 255) / 256 * 256;
+            }
+        }
+    } else {
+        for (int j = 0; j < nconv; j++) {
+            gen::LayerP &G = g.layer[j];
+            if (!gen_layer_tiles(G, G.grid[1], G.grid[2], p->in_layout.Bw)) return false;
+            G.ntd = G.grid[0];
+            G.nty = (G.grid[1] + G.Tb - 1) / G.Tb;
+            G.ntx = (G.grid[2] + G.Tw - 1) / G.Tw;
+            G.ntasks = (long long)p->layers[sg.first + j].out_ext[0] * G.ntd * G.nty * G.ntx * G.nnc;
+        }
+    }
+    int in_stride = 0, w_stride = 0, acc = 0;
+    for (int j = 0; j < nconv; j++) {
+        const gen::LayerP &G = g.layer[j];
         in_stride = std::max(in_stride, G.stage_bytes);
         w_stride = std::max(w_stride, G.kpw * 2 * G.Nc * 16);
         acc = std::max(acc, G.ntl * G.Nc);
-        G.ntasks = (long long)ly.out_ext[0] * G.ntd * G.nty * G.ntx * G.nnc;
     }
     g.in_stride = in_stride;
     g.w_stride = (w_stride + 1023) / 1024 * 1024;
@@ -714,7 +936,7 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, GenGe
 }
 
 // Number of leading conv layers of subgraph sg the generic kernel runs (a trailing pool runs after it
-// on the CUDA-core layer kernel), or 0 if it cannot run the subgraph.
+// on the CUDA-core layer kernel), or 0 if it cannot run the subgraph (in every mode).
 int gen_conv_layers(const bdl_plan *p, const Subgraph &sg) {
     if (p->in_layout.dtype != BDL_BF16 || p->in_layout.Bn != 1) return 0;
     int L = sg.last - sg.first + 1;
@@ -726,7 +948,9 @@ int gen_conv_layers(const bdl_plan *p, const Subgraph &sg) {
         if (p->layers[sg.first + j].L.residual != BDL_NO_RESIDUAL && rt < 0) return 0;
     }
     GenGeom g;
-    return gen_geometry(p, sg, L, g) ? L : 0;
+    if (!gen_geometry(p, sg, L, false, g)) return 0;
+    if (L > 1 && !gen_geometry(p, sg, L, true, g)) return 0;
+    return L;
 }
 
 // Tasks (memo status words) of conv layer j of the generic kernel's subgraph.
@@ -734,15 +958,24 @@ int64_t gen_layer_tasks(const bdl_plan *p, const Subgraph &sg, int j) {
     const int L = gen_conv_layers(p, sg);
     if (j >= L) return 0;
     GenGeom g;
-    gen_geometry(p, sg, L, g);
+    gen_geometry(p, sg, L, false, g);
     return g.layer[j].ntasks;
+}
+
+// Padded-mode scratch: two region slots per CTA.
+int64_t gen_scratch_bytes(const bdl_plan *p, const Subgraph &sg) {
+    const int L = gen_conv_layers(p, sg);
+    if (L <= 1) return 0;
+    GenGeom g;
+    gen_geometry(p, sg, L, true, g);
+    return (int64_t)p->num_sms * 2 * g.scr_slot;
 }
 
 size_t gen_packed_bytes(const bdl_plan *p, const Subgraph &sg, int j) {
     const int L = gen_conv_layers(p, sg);
     if (j >= L) return 0;
     GenGeom g;
-    gen_geometry(p, sg, L, g);
+    gen_geometry(p, sg, L, false, g);
     const gen::LayerP &G = g.layer[j];
     return (size_t)G.nnc * G.nkb * G.nks * 2 * G.Nc * 8 * 2;
 }
@@ -754,7 +987,7 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
     std::vector<int> ord;
     if (L <= 0) return ord;
     GenGeom g;
-    gen_geometry(p, sg, L, g);
+    gen_geometry(p, sg, L, false, g);
     const int N = p->layers[sg.first].in_ext[0];
     long long per_img0 = g.layer[0].ntasks / N;
     int G = (int)std::max<long long>(1, (2LL * p->num_sms + per_img0 - 1) / std::max<long long>(1, per_img0));
@@ -771,7 +1004,7 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
 bdl_status launch_pack_gen(const bdl_plan *p, const Subgraph &sg, int j, void *w_out, cudaStream_t s) {
     const int L = gen_conv_layers(p, sg);
     GenGeom g;
-    gen_geometry(p, sg, L, g);
+    gen_geometry(p, sg, L, false, g);   // packing depends only on the static fields
     const gen::LayerP &G = g.layer[j];
     const bdl_layer &l = p->layers[sg.first + j].L;
     const long long total = (long long)G.nnc * G.nkb * G.nks * 2 * G.Nc * 8;
@@ -790,8 +1023,9 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
     const int L = gen_conv_layers(p, sg);
     if (L <= 0) return fail(BDL_EUNSUPPORTED, "generic tcgen05 kernel: subgraph not supported");
     const bool pool_tail = L < sg.last - sg.first + 1;
+    const bool padded = sg.mode == BDL_MODE_PADDED && L > 1;
     GenGeom g;
-    gen_geometry(p, sg, L, g);
+    gen_geometry(p, sg, L, padded, g);
     gen::Params P;
     memset(&P, 0, sizeof(P));
     P.L = L;
@@ -830,7 +1064,22 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
     P.counters = (unsigned long long *)(wsp + sg.counter_off);
     cudaFuncSetAttribute(gen::gen_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
     const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;
-    if (!unmerged) {
+    if (padded) {
+        P.padded = 1;
+        P.only_layer = -1;
+        for (int d = 0; d < 3; d++) {
+            P.PB[d] = g.PB[d];
+            P.npb[d] = g.npb[d];
+        }
+        P.scratch = wsp + sg.gen_scr_off;
+        P.scr_slot = g.scr_slot;
+        P.norder = (long long)p->layers[sg.first].in_ext[0] * g.npb[0] * g.npb[1] * g.npb[2];
+        const int grid = (int)std::min<long long>(P.norder, p->num_sms);
+        P.ticket_base = sg.ticket_base;
+        sg.ticket_base += 2 * (((unsigned long long)P.norder + 1) / 2) + 2 * grid;
+        launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+        *launches += 1;
+    } else if (!unmerged) {
         P.only_layer = -1;
         P.order = (const int *)(wsp + sg.order_off);
         P.norder = sg.norder;

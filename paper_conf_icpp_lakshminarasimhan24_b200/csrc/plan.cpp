@@ -123,10 +123,9 @@ int64_t gen_layer_tasks(const bdl_plan *p, const Subgraph &sg, int j);
 size_t gen_packed_bytes(const bdl_plan *p, const Subgraph &sg, int j);
 std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg);
 
-int effective_kernel(const Subgraph &sg) {
-    if (sg.kernel == KERNEL_TC_GEN && sg.mode == BDL_MODE_PADDED && sg.gen_layers > 1) return KERNEL_BRICK;
-    return sg.kernel;
-}
+int64_t gen_scratch_bytes(const bdl_plan *p, const Subgraph &sg);
+
+int effective_kernel(const Subgraph &sg) { return sg.kernel; }
 }
 using namespace bdl;
 
@@ -344,6 +343,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
         int ext_in[4];
         for (int d = 0; d < 4; d++) ext_in[d] = fl.in_ext[d];
         sg.model_brick = model_brick(p->opts, nsp, ext_in, &sg.rho);
+        if (p->opts.force_brick > 0) sg.model_brick = p->opts.force_brick;   // padded block edge override
         sg.delta = compute_delta(p->layers, sg.first, sg.last, Bx, false);
         sg.delta_first = compute_delta(p->layers, sg.first, sg.last, Bx, true);
         // executed brick = the layout's; the tiny-layer rule (L659-662) uses it
@@ -431,6 +431,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             sg.norder = (int64_t)sg.order_host.size();
             sg.order_off = sg.norder ? take(sg.norder * 4) : -1;
         } else if (sg.kernel == KERNEL_TC_GEN) {
+            if (int64_t sb = gen_scratch_bytes(p, sg)) sg.gen_scr_off = take(sb);
             sg.order_host = gen_task_order(p, sg);
             sg.norder = (int64_t)sg.order_host.size();
             sg.order_off = sg.norder ? take(sg.norder * 4) : -1;

@@ -161,6 +161,12 @@ class Plan:
                             ctypes.c_void_p(self.ws_ptr), _stream_handle(stream)))
         return bricked_out
 
+    def run_subgraph(self, i, bricked_in, bricked_out, stream=None):
+        """Run subgraph i alone (its input/output tensors: graph input/output buffers or workspace)."""
+        check(lib().bdl_run_subgraph(self.h, i, ctypes.c_void_p(bricked_in.data_ptr()),
+                                     ctypes.c_void_p(bricked_out.data_ptr()), ctypes.c_void_p(self.ws_ptr),
+                                     _stream_handle(stream)))
+
     def forward(self, x, stream=None):
         """Dense NC(D)HW -> dense output: brickify, every merged subgraph, unbrickify."""
         return self.unbrickify(self.run(self.brickify(x, stream=stream), stream=stream), stream=stream)

@@ -50,17 +50,36 @@ def test_gen_vs_oracle(name):
     sgs = plan.subgraphs()
     assert any(s["kernel"] == "tcgen05 generic" for s in sgs), sgs
     outs = {}
-    for mode in ("memoized", "unmerged"):
+    for mode in ("memoized", "unmerged", "padded"):
         plan.set_mode(mode)
         outs[mode] = plan.forward(wl["x"]).float().cpu().numpy()
         assert rel_err(outs[mode], ref) <= TOL, (mode, rel_err(outs[mode], ref))
     np.testing.assert_array_equal(outs["memoized"], outs["unmerged"])
+    np.testing.assert_array_equal(outs["memoized"], outs["padded"])
     plan.set_mode("memoized")
     plan.forward(wl["x"])
     for i, s in enumerate(sgs):
         if s["kernel"] == "tcgen05 generic" and s["last"] > s["first"]:
             c = plan.counters(i)
             assert c["computed"] == c["cas_ok"] and c["computed"] > 0, c
+
+
+@pytest.mark.parametrize("brick", [4, 8, 16, 64])
+def test_gen_padded_block_sizes(brick):
+    """Padded mode with blocks of several edges (regions of edge, interior and single-block images):
+    every block recomputes its halo (§3.2.1, Fig 4) and matches memoized execution exactly."""
+    layers = [W.conv(64, 64, 3), W.conv(64, 128, 1), W.conv(128, 64, 3, res=-1, wscale=0.5)]
+    wl = W.make_graph_workload(layers, 2, 64, 1, 30, 27, 2, (1, 1, 8, 8), "bf16", seed=3)
+    ref = oracle.run_graph(wl["layers"], wl["x"].numpy(), wl["weights"], wl["biases"], dtype="bf16")
+    plan = engine.plan_from_workload(wl, force_mode=1, force_brick=brick)
+    assert plan.subgraphs()[0]["kernel"] == "tcgen05 generic" and plan.subgraphs()[0]["last"] == 2
+    yp = plan.forward(wl["x"]).float().cpu().numpy()
+    assert rel_err(yp, ref) <= TOL
+    for _ in range(3):   # repeated runs: ticket accounting across launches
+        np.testing.assert_array_equal(plan.forward(wl["x"]).float().cpu().numpy(), yp)
+    plan.set_mode("memoized")
+    ym = plan.forward(wl["x"]).float().cpu().numpy()
+    np.testing.assert_array_equal(yp, ym)
 
 
 def test_gen_repeat_and_masking():
