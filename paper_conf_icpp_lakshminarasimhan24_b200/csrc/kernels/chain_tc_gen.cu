@@ -509,7 +509,9 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
     __syncthreads();
     ptx::tc_fence_after();
     pdl_launch_dependents();
-    if ((warp >= kLoad0 && warp < kLoad0 + kLW) || warp >= kEpi0) pdl_wait();   // read the previous kernel's output
+    // loaders / epilogue read the previous kernel's output; the scheduler rewrites memo tags that a previous
+    // run of this subgraph may still be waiting on
+    if ((warp >= kLoad0 && warp < kLoad0 + kLW) || warp >= kEpi0 || warp == kSched) pdl_wait();
 
     const unsigned EP = p.epoch << 2;
     if (warp == kSched) {

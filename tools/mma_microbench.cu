@@ -69,14 +69,16 @@ __global__ void __launch_bounds__(128, 1) mma_loop(int iters, unsigned long long
                     tc_fence_after();
                     bb = (smem_u32(B) + (g % 4) * WB) >> 4;
                 }
-                const uint32_t shift = (it % 9) / 3 * 58 + (it % 3);
+                uint32_t shift = (it % 9) / 3 * 58 + (it % 3);
+                if (MODE == 5) shift = shift / 8 * 8;        // 1024-B aligned A starts
+                if (MODE == 6) shift = 0;                    // same A every tap
 #pragma unroll
-                for (int t = 0; t < 4; t++)
+                for (int t = 0; t < (MODE >= 4 ? 3 : 4); t++)
 #pragma unroll
                     for (int kk = 0; kk < 4; kk++) {
                         uint64_t ad = a0 | ((abase + (shift + t * 128) * 8 + kk * 2) & 0x3FFF);
                         uint64_t bd = b0 | ((bb + kk * 2 * (LBO_B >> 4)) & 0x3FFF);
-                        mma_bf16_elect(tb + t * N, ad, bd, ID, 1);
+                        mma_bf16_elect(tb + (N > 128 ? 0 : t * N), ad, bd, ID, 1);
                     }
                 if (MODE == 3) mma_commit_elect(&wempty[g % 4]);
                 if (MODE == 2) {
@@ -125,10 +127,11 @@ template <int N, int MODE> void run(int sms, const uint8_t *gw) {
     cudaEventRecord(b); cudaEventSynchronize(b);
     float ms; cudaEventElapsedTime(&ms, a, b);
     unsigned long long h[256]; cudaMemcpy(h, d, sms * 8, cudaMemcpyDeviceToHost);
-    double n_mma = (double)iters * 16;
+    double n_mma = (double)iters * (MODE >= 4 ? 12 : 16);
     double flops = n_mma * 2.0 * 128 * N * 16 * sms;
     printf("mode=%d N=%3d  cycles/MMA=%.1f (ideal %d)  chip %.1f TFLOP/s  (%s)\n", MODE, N, h[0] / n_mma, 128 * N / 256,
            flops / (ms * 1e-3) / 1e12, cudaGetErrorString(cudaGetLastError()));
+    fflush(stdout);
     cudaFree(d);
 }
 int main() {
@@ -136,5 +139,8 @@ int main() {
     uint8_t *gw; cudaMalloc(&gw, 9 * 64 * 64 * 2 * 4); cudaMemset(gw, 0, 9 * 64 * 64 * 2 * 4);
     run<32, 0>(sms, gw); run<64, 0>(sms, gw); run<128, 0>(sms, gw); run<256, 0>(sms, gw);
     run<64, 1>(sms, gw); run<64, 2>(sms, gw); run<64, 3>(sms, gw);
+    run<64, 4>(sms, gw); run<64, 5>(sms, gw); run<64, 6>(sms, gw);
+    run<64, 4>(1, gw); run<64, 5>(1, gw); run<64, 6>(1, gw);
+    run<192, 0>(sms, gw); run<192, 4>(sms, gw); run<128, 4>(sms, gw); run<256, 4>(sms, gw);
     return 0;
 }

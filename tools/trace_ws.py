@@ -38,6 +38,14 @@ def st(name, v):
     v = np.array([x for x in v if x is not None]) / 1e3
     if len(v): print(f"{name:14s} mean {v.mean():7.2f} p50 {np.median(v):7.2f} p90 {np.percentile(v, 90):7.2f} max {v.max():7.2f} us")
 def dif(a_, b_): return [r[b_] - r[a_] for r in rec if r[a_] is not None and r[b_] is not None]
+if os.environ.get("BY_LAYER"):
+    allrec = rec
+    for L_ in sorted({r["l"] for r in allrec}):
+        rec = [r for r in allrec if r["l"] == L_]
+        print("-- layer", L_)
+        for a_, b_ in [("mma1", "epi0"), ("epi0", "epi1"), ("epi1", "sync"), ("sync", "read")]:
+            st(f"{a_}->{b_}", dif(a_, b_))
+    rec = allrec
 for a_, b_ in [("q", "dep"), ("dep", "loaded"), ("loaded", "mma0"), ("mma0", "mma1"), ("mma1", "epi0"),
                ("epi0", "epi1"), ("epi1", "sync"), ("sync", "read"), ("read", "end"), ("q", "end")]:
     st(f"{a_}->{b_}", dif(a_, b_))
