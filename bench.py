@@ -38,6 +38,9 @@ def parse():
     ap.add_argument("--mode", default="auto")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cudnn", action="store_true")
+    ap.add_argument("--spatial", action="store_true",
+                    help="3-D configs: shard ONE volume into depth slabs with a brick-plane halo exchange "
+                         "(default for 3-D configs when WORLD_SIZE > 1)")
     return ap.parse_args()
 
 
@@ -197,6 +200,8 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
 
+    if workloads.CONFIGS[args.config]["nsp"] == 3 and (world > 1 or args.spatial):
+        return bench_spatial(args, world, rank, local, dev)
     wl = workloads.make_workload(args.config, input_seed_offset=rank)
     plan = engine.plan_from_workload(wl, device=dev)
     if args.mode != "auto":
@@ -353,6 +358,97 @@ def main():
                              "merged_subgraph": kernel_ms,
                              "unbrickify": statistics.mean(e[2].elapsed_time(e[3]) for e in ev)},
             "cudnn_layer_by_layer": cudnn,
+        }
+        print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def bench_spatial(args, world, rank, local, dev):
+    """One 3-D volume split into `world` depth slabs (strong scaling): per step each rank brickifies its slab
+    into an extended buffer, exchanges one brick plane of halo per face with its neighbours (NCCL
+    point-to-point over NVLink), runs the merged plan on the extended slab and unbrickifies its own planes."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_lakshminarasimhan24_b200 import parallel, workloads
+    wl = workloads.make_workload(args.config)
+    run = parallel.SpatialRunner(wl["layers"], wl["weights"], wl["biases"], wl["C"], wl["D"], wl["H"], wl["W"],
+                                 wl["brick"], wl["dtype"], rank, world, device=dev,
+                                 mode=None if args.mode == "auto" else args.mode)
+    g = run.geo
+    x_own = wl["x"][:, :, g.lo:g.hi].to(device=dev, dtype=run.plan.tdtype).contiguous()
+    y_own = torch.empty((1, run.own_out.C, g.own, wl["H"], wl["W"]), dtype=run.plan.tdtype, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    flush_rd = torch.ones(64 << 20, dtype=torch.float32, device=dev)
+    exch = run.exchange if world > 1 else (lambda: None)
+
+    def step():
+        run.load(x_own)
+        exch()
+        run.compute(out=y_own)
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    K = args.steps
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(K)]
+    with ClockSampler(local) as clk:
+        t_end = time.time() + 0.5
+        while time.time() < t_end:
+            for _ in range(5):
+                step()
+            torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        for k in range(K):
+            flush.zero_()
+            flush_rd.sum()
+            if world > 1:
+                dist.barrier()
+            e = ev[k]
+            e[0].record(stream)
+            run.load(x_own)
+            exch()
+            e[1].record(stream)
+            run.plan.run(run.xb, run.yb)
+            e[2].record(stream)
+            run.plan.unbrickify(run.yb[g.own_slice(run.out_plane)], layout=run.own_out, out=y_own)
+            e[3].record(stream)
+        torch.cuda.synchronize()
+    step_ms = [e[0].elapsed_time(e[3]) for e in ev]
+    t = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_ms = float(t.item())
+    kernel_ms = statistics.mean(e[1].elapsed_time(e[2]) for e in ev)
+    flops = useful_flops(wl)
+    peaks, peak_src = load_peaks()
+    achieved = flops / world / (kernel_ms / 1e3) / 1e12
+    if rank == 0:
+        line = {
+            "metric": "images/sec merged conv chain per B200", "value": K / (total_ms / 1e3), "unit": "volumes/s",
+            "n_gpus": world, "steps": K, "warmup": max(3, args.warmup), "ms_per_step": total_ms / K,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": wl["dtype"],
+            "data": "synthetic (seeded N(0,1) inputs, He-normal weights; workloads.py)",
+            "config": {"workload": workload_desc(wl), "global_batch": 1,
+                       "parallelism": f"spatial depth slabs x{world}, {g.halo_planes}-brick-plane halo exchange "
+                                      f"(NCCL point-to-point)",
+                       "slab_planes": g.own, "halo_planes_per_face": g.halo_planes * wl["brick"][1],
+                       "mode": run.plan.subgraphs()[0]["mode"],
+                       "l2": "flushed between timed steps (256 MiB write + 256 MiB read, outside the events)"},
+            "clocks": clk.summary(),
+            "gpu_launches": K * (2 + run.plan.launches_per_run),
+            "roofline": {"bound": "tensor", "achieved": achieved, "peak": float(peaks["bf16_tflops"]),
+                         "unit": "TFLOP/s", "frac": achieved / float(peaks["bf16_tflops"]), "traffic": None,
+                         "peak_source": f"{peak_src} bf16_tflops",
+                         "kernel": "merged subgraph on the extended slab (useful FLOPs of the own slab)"},
+            "breakdown_ms": {"brickify+halo_exchange": statistics.mean(e[0].elapsed_time(e[1]) for e in ev),
+                             "merged_subgraph": kernel_ms,
+                             "unbrickify": statistics.mean(e[2].elapsed_time(e[3]) for e in ev)},
         }
         print(json.dumps(line))
     if world > 1:

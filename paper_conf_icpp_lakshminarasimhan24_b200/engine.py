@@ -140,10 +140,11 @@ class Plan:
     def alloc_bricked(self, layout):
         return torch.empty(int(layout.total_bytes), dtype=torch.uint8, device=self.device)
 
-    def brickify(self, x, out=None, stream=None):
+    def brickify(self, x, out=None, layout=None, stream=None):
+        layout = layout if layout is not None else self.in_layout
         x = x.to(device=self.device, dtype=self.tdtype).contiguous()
-        out = out if out is not None else self.alloc_bricked(self.in_layout)
-        check(lib().bdl_brickify(ctypes.byref(self.in_layout), ctypes.c_void_p(x.data_ptr()),
+        out = out if out is not None else self.alloc_bricked(layout)
+        check(lib().bdl_brickify(ctypes.byref(layout), ctypes.c_void_p(x.data_ptr()),
                                  ctypes.c_void_p(out.data_ptr()), _stream_handle(stream)))
         return out
 

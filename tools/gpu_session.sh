@@ -1,3 +1,3 @@
 cd $GRAFT_REPO_ROOT
-timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
-timeout 300 python bench.py --no-cpu-baseline 2>/dev/null | python -c "import json,sys;d=json.loads(sys.stdin.read());print(d['value'],d['ms_per_step'],d['roofline']['frac'],d['breakdown_ms'])"
+timeout 600 python -m pytest tests/test_gpu_sharding.py -x -q 2>&1 | tail -5
+timeout 300 python bench.py --config cfg5 --spatial --steps 5 --warmup 3 2>&1 | tail -2
