@@ -60,16 +60,18 @@ def workload_desc(wl):
 
 
 def useful_flops(wl):
-    """2*MACs of plain layer-by-layer execution (padded-mode recompute not credited)."""
+    """2*MACs of plain layer-by-layer execution (padded-mode recompute not credited).  Each layer's
+    input extent is that of the layer it reads (`input`), so branches (projections) are sized right."""
     from paper_conf_icpp_lakshminarasimhan24_b200 import workloads
     f = 0
-    D, H, W = wl["D"], wl["H"], wl["W"]
-    for l in wl["layers"]:
+    shapes = {-1: (wl["D"], wl["H"], wl["W"])}
+    for i, l in enumerate(wl["layers"]):
+        D, H, W = shapes[l["input"]]
         Do, Ho, Wo = workloads.layer_out_shape(l, D, H, W)
         if l["kind"] == "conv":
             kd, kh, kw = l["k"]
             f += 2 * wl["N"] * Do * Ho * Wo * l["cout"] * l["cin"] * kd * kh * kw
-        D, H, W = Do, Ho, Wo
+        shapes[i] = (Do, Ho, Wo)
     return f
 
 

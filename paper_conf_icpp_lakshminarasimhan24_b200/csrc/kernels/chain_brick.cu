@@ -330,6 +330,66 @@ __global__ void __launch_bounds__(256) layer_kernel(GChain g, int l) {
     if (threadIdx.x == 0 && blockIdx.x == 0) atomicAdd(&g.counters[0], (unsigned long long)nb);
 }
 
+// Max-pool (L456-458; out-of-range taps ignored) as its own HBM-bound layer kernel: one
+// thread per (output pixel, 16-byte channel vector), 16-B loads of each in-range window tap and one
+// 16-B store into the bricked output (consecutive threads -> consecutive 16-B chunks of a brick, so
+// loads and stores are coalesced along the channels-innermost brick rows).  Masked positions of
+// partial bricks and padded channels are written as 0 (Q11).
+template <typename T>
+__global__ void __launch_bounds__(256) pool_vec_kernel(GLayer ly, TView in, unsigned long long *counter) {
+    constexpr int V = 16 / sizeof(T);
+    const TView &o = ly.out;
+    const int nvec = o.Cp / V;
+    const int bpx = o.B[0] * o.B[1] * o.B[2] * o.B[3];
+    const long long nbr = (long long)o.nb[0] * o.nb[1] * o.nb[2] * o.nb[3];
+    const long long total = nbr * bpx * nvec;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+        const int cv = (int)(i % nvec);
+        long long r = i / nvec;
+        int inner = (int)(r % bpx);
+        long long b = r / bpx;   // logical brick
+        int lo[4], ext[4];
+        brick_region(o, b, lo, ext);
+        const int w = lo[3] + inner % o.B[3]; inner /= o.B[3];
+        const int h = lo[2] + inner % o.B[2]; inner /= o.B[2];
+        const int d = lo[1] + inner % o.B[1];
+        const int n = lo[0] + inner / o.B[1];
+        float m[V];
+#pragma unroll
+        for (int j = 0; j < V; j++) m[j] = -INFINITY;
+        bool any = false;
+        if (inside4(ly.out_ext, n, d, h, w)) {
+            for (int td = 0; td < ly.k[1]; td++) {
+                const int id = d * ly.s[1] - ly.p[1] + td;
+                for (int th = 0; th < ly.k[2]; th++) {
+                    const int ih = h * ly.s[2] - ly.p[2] + th;
+                    for (int tw = 0; tw < ly.k[3]; tw++) {
+                        const int iw = w * ly.s[3] - ly.p[3] + tw;
+                        if (!inside4(ly.in_ext, n, id, ih, iw)) continue;
+                        const uint4 q = __ldg(reinterpret_cast<const uint4 *>(
+                            reinterpret_cast<const T *>(in.ptr) + tv_off(in, n, id, ih, iw) + cv * V));
+                        const T *e = reinterpret_cast<const T *>(&q);
+#pragma unroll
+                        for (int j = 0; j < V; j++) m[j] = fmaxf(m[j], to_f(e[j]));
+                        any = true;
+                    }
+                }
+            }
+        }
+        uint4 outv;
+        T *oe = reinterpret_cast<T *>(&outv);
+#pragma unroll
+        for (int j = 0; j < V; j++) {
+            float v = (any && cv * V + j < ly.cout) ? m[j] : 0.f;
+            if (ly.relu) v = fmaxf(v, 0.f);
+            oe[j] = from_f<T>(v);
+        }
+        *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(o.ptr) + tv_phys(o, b) * o.brick_elems +
+                                   (long long)(r % bpx) * o.Cp + cv * V) = outv;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(counter, (unsigned long long)nbr);
+}
+
 // weights [cout][kd][kh][kw][cin] (dtype) -> [taps][cin][cout] fp32
 template <typename T>
 __global__ void pack_weights_f32_kernel(const T *__restrict__ w, float *__restrict__ out, int cout, int taps, int cin,
@@ -416,6 +476,17 @@ bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &i
         for (int l = 0; l < g.L; l++) {
             const TView &ov = g.layer[l].out;
             long long nb = (long long)ov.nb[0] * ov.nb[1] * ov.nb[2] * ov.nb[3];
+            const GLayer &G = g.layer[l];
+            const int esz = g.bf16 ? 2 : 4;
+            const TView &src = l == 0 ? g.in : g.layer[l - 1].out;
+            if (G.kind == BDL_OP_MAXPOOL && !G.res_ext && (G.out.Cp * esz) % 16 == 0 && (src.Cp * esz) % 16 == 0) {
+                const long long threads = nb * G.out.B[0] * G.out.B[1] * G.out.B[2] * G.out.B[3] * (G.out.Cp * esz / 16);
+                const int gp = (int)std::min<long long>((threads + 255) / 256, 148LL * 64);
+                if (g.bf16) pool_vec_kernel<__nv_bfloat16><<<gp, 256, 0, s>>>(G, src, g.counters);
+                else pool_vec_kernel<float><<<gp, 256, 0, s>>>(G, src, g.counters);
+                *launches += 1;
+                continue;
+            }
             int gl = (int)std::min<long long>(nb, 65535LL * 16);
             if (g.bf16) layer_kernel<__nv_bfloat16><<<gl, 256, 0, s>>>(g, l);
             else layer_kernel<float><<<gl, 256, 0, s>>>(g, l);
