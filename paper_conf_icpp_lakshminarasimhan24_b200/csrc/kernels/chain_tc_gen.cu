@@ -55,6 +55,8 @@ struct LayerP {
     int Tb, Tw, Wp;
     int ntd, nty, ntx, nnc, Nc;
     int amode, nkb, kc, nks, kpw, nws;   // kc: 16-B chunks per pixel per K-block
+    int lkc;                  // log2(kc)
+    int lB[3];                // log2 of the source view's brick extents (d, h, w)
     int rb, nblk, blk_px, plane_px;
     int in_rows, in_cols;
     int rowsA, stage_bytes, row_u;       // row_u: 16-B units per A row (8 swizzled, 1 planes)
@@ -399,6 +401,9 @@ __device__ void scheduler(const Params &p, Shared &sh) {
 // map (and, in padded mode, outside the source region) are zero-filled.
 __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, const Tile &T, int kb, uint8_t *buf,
                                            int tid) {
+    // Row-by-row: loader warp w takes input rows (plane a, row yy) w, w + 4, ...; per row the brick-row
+    // and scratch-row address arithmetic is done once, and the lanes walk (column, 16-B chunk) pairs with
+    // shifts only (power-of-two brick extents, stride 1 or 2, chunk counts a power of two).
     const TView &v = L.src;
     const __nv_bfloat16 *base = reinterpret_cast<const __nv_bfloat16 *>(v.ptr);
     const __nv_bfloat16 *sbase = nullptr;
@@ -409,35 +414,56 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
         sp1 = S.pR[1];
         sp2 = S.pR[2];
     }
-    const int kc = L.kc;
-    const int npx = L.k[0] * L.in_rows * L.in_cols;
-    const int total = npx * kc;
+    const int lane = tid & 31, w = tid >> 5;
+    const int lkc = L.lkc, kc = 1 << lkc;
+    const int nrow = L.k[0] * L.in_rows;
     const int z0 = T.d * L.s[0] - L.pd[0];
     const int y0 = T.y0 * L.s[1] - L.pd[1];
     const int x0 = T.x0 * L.s[2] - L.pd[2];
     const uint32_t plane_bytes = (uint32_t)L.rowsA * 16;
-    for (int it = tid; it < total; it += kLoadT) {
-        const int P = it / kc, ch = it - P * kc;
-        const int xx = P % L.in_cols;
-        const int r2 = P / L.in_cols;
-        const int yy = r2 % L.in_rows, a = r2 / L.in_rows;
-        const int z = z0 + a, y = y0 + yy, x = x0 + xx;
-        bool ok = z >= 0 && z < L.in_ext[0] && y >= 0 && y < L.in_ext[1] && x >= 0 && x < L.in_ext[2];
-        const int px = a * L.plane_px + ((yy % L.s[1]) * L.s[2] + (xx % L.s[2])) * L.blk_px + (yy / L.s[1]) * L.Wp +
-                       xx / L.s[2];
-        uint32_t off;
-        if (L.amode == AM_SW128) off = (uint32_t)px * 128 + ((ch ^ (px & 7)) << 4);
-        else off = (uint32_t)ch * plane_bytes + (uint32_t)px * 16;
-        const void *g = base;
-        if (T.src_scr) {
-            ok = ok && z >= T.slo[0] && z < T.shi[0] && y >= T.slo[1] && y < T.shi[1] && x >= T.slo[2] && x < T.shi[2];
-            if (ok)
-                g = sbase + ((((long long)(z - T.slo[0]) * sp1 + (y - T.slo[1])) * sp2 + (x - T.slo[2])) * L.cin +
-                             kb * 64 + ch * 8);
-        } else if (ok) {
-            g = base + pix(v, T.n, z, y, x) + kb * 64 + ch * 8;
+    const int ls2 = L.s[2] - 1;                   // log2 of the column stride (1 or 2)
+    const int lBd = L.lB[0], lBh = L.lB[1], lBw = L.lB[2];
+    const int nchunk = L.in_cols << lkc;
+    for (int r2 = w; r2 < nrow; r2 += kLW) {
+        const int a = r2 / L.in_rows, yy = r2 - a * L.in_rows;
+        const int z = z0 + a, y = y0 + yy;
+        bool rok = z >= 0 && z < L.in_ext[0] && y >= 0 && y < L.in_ext[1];
+        if (T.src_scr) rok = rok && z >= T.slo[0] && z < T.shi[0] && y >= T.slo[1] && y < T.shi[1];
+        const int yq = L.s[1] == 2 ? (yy >> 1) : yy, yr = L.s[1] == 2 ? (yy & 1) : 0;
+        const int rowpx = a * L.plane_px + yr * L.s[2] * L.blk_px + yq * L.Wp;
+        long long rowlog = 0, srow = 0;
+        int rowin = 0;
+        if (rok) {
+            if (T.src_scr) {
+                srow = ((long long)(z - T.slo[0]) * sp1 + (y - T.slo[1])) * sp2;
+            } else {
+                const int bd = z >> lBd, by = y >> lBh;
+                rowlog = (((long long)T.n * v.nb[1] + bd) * v.nb[2] + by) * v.nb[3];
+                rowin = (((z - (bd << lBd)) << lBh) + (y - (by << lBh))) << lBw;
+            }
         }
-        ptx::cp_async16(buf + off, g, ok ? 16u : 0u);
+        for (int q = lane; q < nchunk; q += 32) {
+            const int xx = q >> lkc, ch = q & (kc - 1);
+            const int x = x0 + xx;
+            bool ok = rok && x >= 0 && x < L.in_ext[2];
+            if (T.src_scr) ok = ok && x >= T.slo[2] && x < T.shi[2];
+            const int px = rowpx + (xx & ls2) * L.blk_px + (xx >> ls2);
+            uint32_t off;
+            if (L.amode == AM_SW128) off = (uint32_t)px * 128 + ((ch ^ (px & 7)) << 4);
+            else off = (uint32_t)ch * plane_bytes + (uint32_t)px * 16;
+            const void *g = base;
+            if (ok) {
+                if (T.src_scr) {
+                    g = sbase + ((srow + (x - T.slo[2])) * L.cin + kb * 64 + ch * 8);
+                } else {
+                    const int bx = x >> lBw;
+                    const long long logical = rowlog + bx;
+                    const long long phys = v.bmap ? (long long)v.bmap[logical] : logical;
+                    g = base + phys * v.brick_elems + (long long)(rowin + x - (bx << lBw)) * v.Cp + kb * 64 + ch * 8;
+                }
+            }
+            ptx::cp_async16(buf + off, g, ok ? 16u : 0u);
+        }
     }
 }
 
@@ -564,9 +590,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 const int s = gin % p.nin;
                 if (gin >= (uint32_t)p.nin) ptx::mbar_wait(&sh.in_empty[s], ((gin / p.nin) - 1) & 1);
                 load_stage(p, L, T, kb, in_ring + (size_t)s * p.in_stride, tid);
-                ptx::cp_async_wait_all();
-                ptx::fence_proxy_async_smem();
-                mbar_arrive(&sh.in_full[s]);
+                // completion tracked by the barrier (the loader moves on to the next stage / task at once)
+                ptx::cp_async_arrive_noinc(&sh.in_full[s]);
             }
         }
     } else if (warp == kWProd) {
@@ -617,6 +642,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             for (int kb = 0; kb < L.nkb; kb++, gin++) {
                 const int s = gin % p.nin;
                 ptx::mbar_wait(&sh.in_full[s], (gin / p.nin) & 1);
+                ptx::fence_proxy_async_smem();   // cp.async (generic proxy) data -> tcgen05 operand reads
                 ptx::tc_fence_after();
                 const uint32_t a_base = ptx::smem_u32(in_ring + (size_t)s * p.in_stride) >> 4;
                 for (int j = 0; j < L.nws; j++, gw++) {
@@ -808,6 +834,13 @@ static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out,
     if (G.amode == gen::AM_SW128) { G.nkb = l.cin / 64; G.kc = 8; G.nks = taps * 4; G.row_u = 8; }
     else if (G.amode == gen::AM_PLANES) { G.nkb = 1; G.kc = l.cin / 8; G.nks = taps * ((l.cin + 15) / 16); G.row_u = 1; }
     else { G.nkb = 1; G.kc = 1; G.nks = G.k[0] * G.k[1] * ((G.k[2] + 1) / 2); G.row_u = 1; }
+    // the loader's address arithmetic uses shifts: power-of-two chunk counts and brick extents
+    auto lg = [](int v) { int r = 0; while ((1 << r) < v) r++; return (1 << r) == v ? r : -1; };
+    G.lkc = lg(G.kc);
+    G.lB[0] = lg(lo_out.Bd);
+    G.lB[1] = lg(lo_out.Bh);
+    G.lB[2] = lg(lo_out.Bw);
+    if (G.lkc < 0 || G.lB[0] < 0 || G.lB[1] < 0 || G.lB[2] < 0) return false;
     if (G.nks > gen::kMaxKs) return false;
     const int ks_bytes = 2 * G.Nc * 16;
     G.kpw = std::max(1, std::min(G.nks, kGenWStage / ks_bytes));

@@ -36,13 +36,22 @@ def main():
             plan.run_subgraph(i, xb, yb)
             ev[r][i + 1].record()
     torch.cuda.synchronize()
+    shapes = {-1: (wl["D"], wl["H"], wl["W"])}
+    fl = []
+    for j, l in enumerate(wl["layers"]):
+        o = workloads.layer_out_shape(l, *shapes[l["input"]])
+        shapes[j] = o
+        fl.append(2 * wl["N"] * o[0] * o[1] * o[2] * l["cout"] * l["cin"] * l["k"][0] * l["k"][1] * l["k"][2]
+                  if l["kind"] == "conv" else 0)
     tot = 0.0
     for i, s in enumerate(sgs):
         ms = sorted(ev[r][i].elapsed_time(ev[r][i + 1]) for r in range(a.reps))[a.reps // 2]
         tot += ms
         ls = wl["layers"][s["first"]:s["last"] + 1]
         desc = " ".join(f"{l['kind'][0]}{l['cin']}>{l['cout']}k{l['k'][-1]}s{l['stride'][-1]}" for l in ls)
-        print(f"{i:3d} [{s['first']:2d},{s['last']:2d}] {s['mode']:9s} {s['kernel']:16s} {ms:9.3f} ms  {desc}")
+        f = sum(fl[s["first"]:s["last"] + 1])
+        print(f"{i:3d} [{s['first']:2d},{s['last']:2d}] {s['mode']:9s} {s['kernel']:16s} {ms:9.3f} ms "
+              f"{f / ms / 1e9:7.1f} TF/s  {desc}")
     print(f"total {tot:.3f} ms")
 
 
