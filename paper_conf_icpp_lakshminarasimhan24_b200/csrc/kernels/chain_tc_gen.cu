@@ -28,6 +28,9 @@
 #include <string>
 #include <vector>
 
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include "common.cuh"
 #include "tc_ptx.cuh"
 
@@ -56,6 +59,7 @@ struct LayerP {
     int ntd, nty, ntx, nnc, Nc;
     int amode, nkb, kc, nks, kpw, nws;   // kc: 16-B chunks per pixel per K-block
     int lkc;                  // log2(kc)
+    int tma;                  // 1: the in-image columns of each input row arrive by one TMA box (tm_row)
     int lB[3];                // log2 of the source view's brick extents (d, h, w)
     int rb, nblk, blk_px, plane_px;
     int in_rows, in_cols;
@@ -68,6 +72,7 @@ struct LayerP {
 };
 
 struct Params {
+    CUtensorMap tm_row[kMaxLayers];      // 5-D row map of each layer's source (LayerP::tma): box = Tw pixels x 64 ch
     LayerP layer[kMaxLayers];
     int L;
     int nin, nw, in_stride, w_stride;    // ring depths and slot strides (bytes)
@@ -82,6 +87,7 @@ struct Params {
     // padded mode (§3.2.1): a task is a PB block of the last layer's output; every layer's
     // halo-extended region is recomputed by the CTA into its private scratch (two slots, so two blocks
     // interleave and one block's loads overlap the other's MMAs)
+    unsigned long long *prof;            // debug (BDL_GEN_PROF): per CTA 16 x u64 of role wait / busy cycles, or null
     int padded;
     int PB[3], npb[3];
     unsigned char *scratch;
@@ -107,6 +113,16 @@ struct Shared {
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ptx::smem_u32(bar)) : "memory");
 }
+// debug profiler: time spent blocked in an mbarrier wait (only when p.prof is set)
+__device__ __forceinline__ void pwait(const Params &p, uint64_t *bar, uint32_t parity, unsigned long long &acc) {
+    if (p.prof) {
+        const unsigned long long t0 = clock64();
+        ptx::mbar_wait(bar, parity);
+        acc += clock64() - t0;
+    } else {
+        ptx::mbar_wait(bar, parity);
+    }
+}
 __device__ __forceinline__ int tag_state(int v, unsigned EP) { return ((v & ~3) == (int)EP) ? (v & 3) : 0; }
 __device__ __forceinline__ int *status_word(const Params &p, int l, long long t) {
     return p.status + p.layer[l].task_base + t;
@@ -121,6 +137,16 @@ __device__ __forceinline__ TaskC decode(const LayerP &L, long long t) {
     c.d = (int)(t % L.ntd);
     c.n = (int)(t / L.ntd);
     return c;
+}
+
+// Element offset of channel 0 of pixel (n, d, y, x) in a bricked view (Bn = 1), power-of-two bricks
+// with log2 extents lB (d, h, w).
+__device__ __forceinline__ long long pix_pow2(const TView &v, const int *lB, int n, int d, int y, int x) {
+    const int bd = d >> lB[0], by = y >> lB[1], bx = x >> lB[2];
+    const long long logical = (((long long)n * v.nb[1] + bd) * v.nb[2] + by) * v.nb[3] + bx;
+    const long long phys = v.bmap ? (long long)v.bmap[logical] : logical;
+    const int in = ((((d - (bd << lB[0])) << lB[1]) + (y - (by << lB[1]))) << lB[2]) + (x - (bx << lB[2]));
+    return phys * v.brick_elems + (long long)in * v.Cp;
 }
 
 // Element offset of channel 0 of pixel (n, d, y, x) in a bricked view (Bn = 1).
@@ -400,7 +426,7 @@ __device__ void scheduler(const Params &p, Shared &sh) {
 // One K-block of the input tile of a tile into stage `buf` (128 threads).  Positions outside the feature
 // map (and, in padded mode, outside the source region) are zero-filled.
 __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, const Tile &T, int kb, uint8_t *buf,
-                                           int tid) {
+                                           int tid, uint64_t *bar) {
     // Row-by-row: loader warp w takes input rows (plane a, row yy) w, w + 4, ...; per row the brick-row
     // and scratch-row address arithmetic is done once, and the lanes walk (column, 16-B chunk) pairs with
     // shifts only (power-of-two brick extents, stride 1 or 2, chunk counts a power of two).
@@ -424,6 +450,48 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
     const int ls2 = L.s[2] - 1;                   // log2 of the column stride (1 or 2)
     const int lBd = L.lB[0], lBh = L.lB[1], lBw = L.lB[2];
     const int nchunk = L.in_cols << lkc;
+    if (L.tma && !T.src_scr) {
+        // stride-1 SW128 rows: the Tw in-tile columns of an in-image row by one TMA box (completion on `bar` by
+        // transaction count), halo columns by cp.async, rows outside the image zero-filled
+        const int l = (int)(&L - p.layer);
+        const int pdw = L.pd[2];
+        const int nh = L.in_cols - L.Tw;          // halo columns (k - 1)
+        for (int r2 = w; r2 < nrow; r2 += kLW) {
+            const int a = r2 / L.in_rows, yy = r2 - a * L.in_rows;
+            const int z = z0 + a, y = y0 + yy;
+            const bool rok = z >= 0 && z < L.in_ext[0] && y >= 0 && y < L.in_ext[1];
+            const int rowpx = a * L.plane_px + yy * L.Wp;
+            if (rok) {
+                if (lane == 0) {
+                    ptx::mbar_expect_tx(bar, (uint32_t)L.Tw * 128);
+                    const int by = y >> lBh;
+                    ptx::tma_load_5d(buf + (size_t)(rowpx + pdw) * 128, &p.tm_row[l], kb * 64, 0, T.x0 >> lBw,
+                                     y - (by << lBh), (T.n * v.nb[1] + z) * v.nb[2] + by, bar);
+                }
+            } else {
+                for (int q = lane; q < L.Tw * 8; q += 32)
+                    *reinterpret_cast<uint4 *>(buf + (size_t)(rowpx + pdw + (q >> 3)) * 128 + ((q & 7) << 4)) =
+                        make_uint4(0, 0, 0, 0);
+            }
+            for (int q = lane; q < nh * 8; q += 32) {
+                const int hc = q >> 3, ch = q & 7;
+                const int xx = hc < pdw ? hc : L.Tw + hc;
+                const int x = x0 + xx;
+                const bool ok = rok && x >= 0 && x < L.in_ext[2];
+                const int px = rowpx + xx;
+                const void *g = base;
+                if (ok) {
+                    const int bd = z >> lBd, by = y >> lBh, bx = x >> lBw;
+                    const long long logical = (((long long)T.n * v.nb[1] + bd) * v.nb[2] + by) * v.nb[3] + bx;
+                    const int in = ((((z - (bd << lBd)) << lBh) + (y - (by << lBh))) << lBw) + (x - (bx << lBw));
+                    g = base + logical * v.brick_elems + (long long)in * v.Cp + kb * 64 + ch * 8;
+                }
+                ptx::cp_async16(buf + (uint32_t)px * 128 + ((ch ^ (px & 7)) << 4), g, ok ? 16u : 0u);
+            }
+        }
+        ptx::fence_proxy_async_smem();   // zero-filled rows (generic stores) -> tcgen05 operand reads
+        return;
+    }
     for (int r2 = w; r2 < nrow; r2 += kLW) {
         const int a = r2 / L.in_rows, yy = r2 - a * L.in_rows;
         const int z = z0 + a, y = y0 + yy;
@@ -547,9 +615,11 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         // ------------------------------------------------------------------ loaders
         const int tid = threadIdx.x - 32 * kLoad0;
         uint32_t gin = 0;
+        unsigned long long wq = 0, wdep = 0, wbuf = 0;
+        const unsigned long long t_start = clock64();
         for (uint32_t seq = 0;; seq++) {
             const int slot = seq % kQ;
-            ptx::mbar_wait(&sh.q_full[slot], (seq / kQ) & 1);
+            pwait(p, &sh.q_full[slot], (seq / kQ) & 1, wq);
             const int l = sh.q_l[slot];
             const long long t = sh.q_t[slot];
             const int wait = sh.q_w[slot];
@@ -565,6 +635,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 const DepRange r = dep_range(p, l, t);
                 const int nd = dep_count(r);
                 unsigned long long spins = 0;
+                const unsigned long long td0 = clock64();
                 for (int i = lane; i < nd; i += 32) {
                     const int *dw = status_word(p, l - 1, dep_task(p, l, r, i));
                     while (ld_acquire(dw) != (int)(EP | 2)) {
@@ -573,10 +644,12 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     }
                 }
                 __syncwarp();
+                wdep += clock64() - td0;
                 for (int o = 16; o; o >>= 1) spins += __shfl_xor_sync(0xffffffff, spins, o);
                 if (lane == 0 && spins) atomicAdd(&p.counters[3], spins);
             }
             asm volatile("bar.sync 1, %0;" ::"n"(kLoadT) : "memory");
+            if (l >= 0 && p.layer[l].tma) ptx::fence_proxy_async();   // acquired data is read by TMA (async proxy)
             if (tid == 0) {
                 sh.desc_l[seq % kRing] = l;
                 sh.desc_t[seq % kRing] = t;
@@ -588,15 +661,21 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             const Tile T = make_tile(p, l, t);
             for (int kb = 0; kb < L.nkb; kb++, gin++) {
                 const int s = gin % p.nin;
-                if (gin >= (uint32_t)p.nin) ptx::mbar_wait(&sh.in_empty[s], ((gin / p.nin) - 1) & 1);
-                load_stage(p, L, T, kb, in_ring + (size_t)s * p.in_stride, tid);
+                if (gin >= (uint32_t)p.nin) pwait(p, &sh.in_empty[s], ((gin / p.nin) - 1) & 1, wbuf);
+                load_stage(p, L, T, kb, in_ring + (size_t)s * p.in_stride, tid, &sh.in_full[s]);
                 // completion tracked by the barrier (the loader moves on to the next stage / task at once)
                 ptx::cp_async_arrive_noinc(&sh.in_full[s]);
             }
         }
+        if (p.prof && tid == 0) {
+            unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
+            r[0] = wq; r[1] = wdep; r[2] = wbuf; r[3] = clock64() - t_start;
+        }
     } else if (warp == kWProd) {
         // ------------------------------------------------------------------ weight producer
         uint32_t gw = 0;
+        unsigned long long ww = 0;
+        const unsigned long long t_start = clock64();
         for (uint32_t seq = 0;; seq++) {
             const int slot = seq % kQ;
             ptx::mbar_wait(&sh.q_full[slot], (seq / kQ) & 1);
@@ -614,7 +693,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     const int st = gw % p.nw;
                     const int q0 = j * L.kpw, nq = min(L.kpw, L.nks - q0);
                     const uint32_t bytes = (uint32_t)(nq * ks_bytes);
-                    if (gw >= (uint32_t)p.nw) ptx::mbar_wait(&sh.wempty[st], ((gw / p.nw) - 1) & 1);
+                    if (gw >= (uint32_t)p.nw) pwait(p, &sh.wempty[st], ((gw / p.nw) - 1) & 1, ww);
                     if (ptx::elect_one()) {
                         ptx::mbar_arrive_expect_tx(&sh.wfull[st], bytes);
                         ptx::bulk_g2s(w_ring + (size_t)st * p.w_stride, wl + ((size_t)kb * L.nks + q0) * ks_bytes, bytes,
@@ -624,30 +703,36 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 }
             }
         }
+        if (p.prof && lane == 0) {
+            unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
+            r[4] = ww; r[5] = clock64() - t_start;
+        }
     } else if (warp == kMma) {
         // ------------------------------------------------------------------ MMA issuer
         const uint32_t tmem_base = __shfl_sync(0xffffffff, sh.tmem_base, 0);
         uint32_t gin = 0, gw = 0;
+        unsigned long long wdesc = 0, wacc = 0, win = 0, wwt = 0;
+        const unsigned long long t_start = clock64();
         for (uint32_t seq = 0;; seq++) {
-            ptx::mbar_wait(&sh.desc_full[seq % kRing], (seq / kRing) & 1);
+            pwait(p, &sh.desc_full[seq % kRing], (seq / kRing) & 1, wdesc);
             const int l = sh.desc_l[seq % kRing];
             if (l < 0) break;
             const LayerP &L = p.layer[l];
             const int a = seq % p.nacc;
-            if (seq >= (uint32_t)p.nacc) ptx::mbar_wait(&sh.acc_empty[a], ((seq / p.nacc) - 1) & 1);
+            if (seq >= (uint32_t)p.nacc) pwait(p, &sh.acc_empty[a], ((seq / p.nacc) - 1) & 1, wacc);
             ptx::tc_fence_after();
             const uint32_t d_base = tmem_base + a * p.acc_stride;
             const uint32_t lbo_b = (uint32_t)L.Nc * 16;
             const uint32_t ks_u = (uint32_t)L.Nc * 2;   // 16-B units per k-step of B
             for (int kb = 0; kb < L.nkb; kb++, gin++) {
                 const int s = gin % p.nin;
-                ptx::mbar_wait(&sh.in_full[s], (gin / p.nin) & 1);
+                pwait(p, &sh.in_full[s], (gin / p.nin) & 1, win);
                 ptx::fence_proxy_async_smem();   // cp.async (generic proxy) data -> tcgen05 operand reads
                 ptx::tc_fence_after();
                 const uint32_t a_base = ptx::smem_u32(in_ring + (size_t)s * p.in_stride) >> 4;
                 for (int j = 0; j < L.nws; j++, gw++) {
                     const int st = gw % p.nw;
-                    ptx::mbar_wait(&sh.wfull[st], (gw / p.nw) & 1);
+                    pwait(p, &sh.wfull[st], (gw / p.nw) & 1, wwt);
                     ptx::tc_fence_after();
                     const uint32_t b_base = ptx::smem_u32(w_ring + (size_t)st * p.w_stride) >> 4;
                     const int q0 = j * L.kpw, q1 = min(L.nks, q0 + L.kpw);
@@ -670,21 +755,27 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             ptx::mma_commit_elect(&sh.acc_full[a]);
             __syncwarp();
         }
+        if (p.prof && lane == 0) {
+            unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
+            r[6] = wdesc; r[7] = wacc; r[8] = win; r[9] = wwt; r[10] = clock64() - t_start;
+        }
     } else {
         // ------------------------------------------------------------------ epilogue
         const int ew = warp - kEpi0;
+        unsigned long long wed = 0, wea = 0, web = 0;
+        const unsigned long long t_start = clock64();
         const int quad = warp % 4;        // TMEM lane quadrant this warp may access
         const int rank = ew / 4;          // 4 warps per quadrant split the (tile, column batch) items
         const uint32_t tmem_base = sh.tmem_base;
         for (uint32_t seq = 0;; seq++) {
-            ptx::mbar_wait(&sh.desc_full[seq % kRing], (seq / kRing) & 1);
+            pwait(p, &sh.desc_full[seq % kRing], (seq / kRing) & 1, wed);
             const int l = sh.desc_l[seq % kRing];
             const long long t = sh.desc_t[seq % kRing];
             if (l < 0) break;
             const LayerP &L = p.layer[l];
             const Tile T = make_tile(p, l, t);
             const int a = seq % p.nacc;
-            ptx::mbar_wait(&sh.acc_full[a], (seq / p.nacc) & 1);
+            pwait(p, &sh.acc_full[a], (seq / p.nacc) & 1, wea);
             ptx::tc_fence_after();
             const int CB = L.Nc >= 32 ? 32 : 16;
             const int ncb = L.Nc / CB;
@@ -713,12 +804,12 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 uint4 *dst = reinterpret_cast<uint4 *>(
                     T.dst_scr ? scr + ((((long long)(d - T.dlo[0]) * L.pR[1] + (y - T.dlo[1])) * L.pR[2] + (x - T.dlo[2])) *
                                            L.cout + ch0)
-                              : outp + pix(L.out, T.n, d, y, x) + ch0);
+                              : outp + pix_pow2(L.out, L.lB, T.n, d, y, x) + ch0);
                 if (kind == 1) {
                     for (int k = 0; k < CB / 8; k++) dst[k] = make_uint4(0, 0, 0, 0);
                     continue;
                 }
-                const uint4 *rs = L.has_res ? reinterpret_cast<const uint4 *>(resp + pix(L.res, T.n, d, y, x) + ch0) : nullptr;
+                const uint4 *rs = L.has_res ? reinterpret_cast<const uint4 *>(resp + pix_pow2(L.res, L.lB, T.n, d, y, x) + ch0) : nullptr;
 #pragma unroll
                 for (int k = 0; k < 4; k++) {
                     if (k >= CB / 8) break;
@@ -749,13 +840,19 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             __syncwarp();
             if (lane == 0) mbar_arrive(&sh.acc_empty[a]);
             // every epilogue warp's stores of this tile precede the publication
+            const unsigned long long tb0 = p.prof ? clock64() : 0;
             asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");
+            if (p.prof) web += clock64() - tb0;
             if (ew == 0 && lane == 0) {
                 __threadfence();
                 if (p.padded) *reinterpret_cast<volatile int *>(&sh.done_seq) = (int)seq + 1;
                 else if (p.only_layer < 0) st_release(status_word(p, l, t), (int)(EP | 2));
                 atomicAdd(&p.counters[0], 1ULL);
             }
+        }
+        if (p.prof && ew == 0 && lane == 0) {
+            unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
+            r[11] = wed; r[12] = wea; r[13] = web; r[14] = clock64() - t_start;
         }
     }
     ptx::tc_fence_before();
@@ -891,6 +988,42 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
         }
     }
     return found;
+}
+
+// TMA rows for the generic kernel's stride-1 SW128 layers (BDL_GEN_TMA=0 disables, for A/B runs).
+static bool gen_tma_ok() {
+    static const int v = [] { const char *e = getenv("BDL_GEN_TMA"); return e ? atoi(e) : 1; }();
+    return v != 0;
+}
+// 5-D view of a 2-D bricked bf16 tensor (identity BrickMap): (channel, x in brick, brick column, y in brick,
+// brick row over (n, by)); box = 64 channels x Bw x nseg bricks x 1 x 1, 128-B swizzled (the SW128 A layout).
+static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg) {
+    static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+    if (!enc) {
+        cudaDriverEntryPointQueryResult qr;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void **)&enc, cudaEnableDefault, &qr) != cudaSuccess ||
+            !enc)
+            return false;
+    }
+    const cuuint64_t px = (cuuint64_t)v.Cp * 2, brick = (cuuint64_t)v.brick_elems * 2;
+    cuuint64_t dims[5] = {(cuuint64_t)v.Cp, (cuuint64_t)v.B[3], (cuuint64_t)v.nb[3], (cuuint64_t)v.B[2],
+                          (cuuint64_t)v.nb[0] * v.nb[1] * v.nb[2]};
+    cuuint64_t strides[4] = {px, brick, px * v.B[3], brick * v.nb[3]};
+    cuuint32_t box[5] = {64, (cuuint32_t)v.B[3], (cuuint32_t)nseg, 1, 1};
+    cuuint32_t es[5] = {1, 1, 1, 1, 1};
+    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, v.ptr, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) ==
+           CUDA_SUCCESS;
+}
+
+// Debug profiler buffer (BDL_GEN_PROF=1): 16 x u64 per CTA, zeroed before each launch.
+static unsigned long long *gen_prof_buf = nullptr;
+static unsigned long long *gen_prof_buffer(cudaStream_t s) {
+    static const bool on = getenv("BDL_GEN_PROF") != nullptr;
+    if (!on) return nullptr;
+    if (!gen_prof_buf) cudaMalloc(&gen_prof_buf, 1024 * 16 * 8);
+    cudaMemsetAsync(gen_prof_buf, 0, 1024 * 16 * 8, s);
+    return gen_prof_buf;
 }
 
 struct GenGeom {
@@ -1064,6 +1197,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
     gen::Params P;
     memset(&P, 0, sizeof(P));
     P.L = L;
+    P.prof = gen_prof_buffer(s);
     const int nsp = p->in_layout.nsp;
     std::vector<TView> outs(L);
     for (int j = 0; j < L; j++) {
@@ -1080,6 +1214,11 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
         }
         G.src = j == 0 ? in : outs[j - 1];
         G.out = outs[j];
+        G.tma = 0;
+        if (!padded && G.amode == gen::AM_SW128 && G.s[1] == 1 && G.s[2] == 1 && G.k[0] == 1 && nsp == 2 &&
+            !G.src.bmap && G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
+            gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw))
+            G.tma = 1;
         G.has_res = sg.res_tensor[j] >= 0;
         if (G.has_res) G.res = res[j];
         G.relu = ly.L.relu;
@@ -1160,3 +1299,12 @@ int gen_launches(const bdl_plan *p, const Subgraph &sg) {
 }
 
 }  // namespace bdl
+
+// Debug: copy the generic kernel's per-CTA role profile (16 x u64 per CTA) of the last launch to host.
+extern "C" int bdl_debug_gen_prof(unsigned long long *host, int max_ctas) {
+    if (!bdl::gen_prof_buf) return 0;
+    const int n = max_ctas < 1024 ? max_ctas : 1024;
+    cudaDeviceSynchronize();
+    cudaMemcpy(host, bdl::gen_prof_buf, (size_t)n * 16 * 8, cudaMemcpyDeviceToHost);
+    return n;
+}

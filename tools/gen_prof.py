@@ -1,0 +1,30 @@
+"""Per-role wait/busy split of the generic tcgen05 kernel, per subgraph (debug, BDL_GEN_PROF).
+    python tools/gen_prof.py cfg4 [subgraph ...]"""
+import ctypes, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+os.environ["BDL_GEN_PROF"] = "1"
+import numpy as np, torch
+from paper_conf_icpp_lakshminarasimhan24_b200 import engine, workloads, lib
+cfg = sys.argv[1]
+wl = workloads.make_workload(cfg)
+plan = engine.plan_from_workload(wl)
+xb = plan.brickify(wl["x"]); yb = plan.alloc_bricked(plan.out_layout)
+plan.run(xb, yb); torch.cuda.synchronize()
+sgs = plan.subgraphs()
+ids = [int(a) for a in sys.argv[2:]] or range(len(sgs))
+f = lib().bdl_debug_gen_prof; f.restype = ctypes.c_int
+names = ["ld q_full", "ld deps", "ld in_empty", "ld total", "wp wempty", "wp total", "mma desc", "mma acc_empty",
+         "mma in_full", "mma wfull", "mma total", "epi desc", "epi acc_full", "epi bar", "epi total"]
+for i in ids:
+    if sgs[i]["kernel"] != "tcgen05 generic":
+        continue
+    plan.run_subgraph(i, xb, yb); torch.cuda.synchronize()
+    buf = (ctypes.c_ulonglong * (1024 * 16))()
+    f(buf, 1024)
+    a = np.frombuffer(buf, dtype=np.uint64).reshape(1024, 16).astype(np.float64)
+    a = a[a[:, 3] > 0]
+    m = a.mean(axis=0)
+    ls = wl["layers"][sgs[i]["first"]:sgs[i]["last"] + 1]
+    desc = " ".join(f"{l['kind'][0]}{l['cin']}>{l['cout']}k{l['k'][-1]}s{l['stride'][-1]}" for l in ls)
+    print(f"sg {i} {sgs[i]['mode']} {desc}: ctas {len(a)}  total {m[14]/1.9e3:.0f} us")
+    print("   " + "  ".join(f"{n} {100*m[k]/max(m[14],1):.0f}%" for k, n in enumerate(names) if k not in (3, 5, 10, 14)))
