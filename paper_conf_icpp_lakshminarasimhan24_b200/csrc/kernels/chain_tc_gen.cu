@@ -450,6 +450,29 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
     const int ls2 = L.s[2] - 1;                   // log2 of the column stride (1 or 2)
     const int lBd = L.lB[0], lBh = L.lB[1], lBw = L.lB[2];
     const int nchunk = L.in_cols << lkc;
+    if (L.tma == 2 && !T.src_scr) {
+        // 1x1 stride-2 SW128 layer: only polyphase block (0, 0) is read by the MMAs.  Output row i reads input
+        // row 2 * (y0 + i); one TMA box per row picks every other pixel (element stride 2 along x in brick)
+        // and lands the Tw pixels contiguously at block row i.
+        const int l = (int)(&L - p.layer);
+        for (int i = w; i < L.Tb; i += kLW) {
+            const int y = y0 + 2 * i;
+            uint8_t *dst = buf + (size_t)(i * L.Wp) * 128;
+            if (y >= 0 && y < L.in_ext[1]) {
+                if (lane == 0) {
+                    ptx::mbar_expect_tx(bar, (uint32_t)L.Tw * 128);
+                    const int by = y >> lBh;
+                    ptx::tma_load_5d(dst, &p.tm_row[l], kb * 64, 0, x0 >> lBw, y - (by << lBh),
+                                     T.n * v.nb[2] + by, bar);
+                }
+            } else {
+                for (int q = lane; q < L.Tw * 8; q += 32)
+                    *reinterpret_cast<uint4 *>(dst + (size_t)(q >> 3) * 128 + ((q & 7) << 4)) = make_uint4(0, 0, 0, 0);
+            }
+        }
+        ptx::fence_proxy_async_smem();
+        return;
+    }
     if (L.tma && !T.src_scr) {
         // stride-1 SW128 rows: the Tw in-tile columns of an in-image row by one TMA box (completion on `bar` by
         // transaction count), halo columns by cp.async, rows outside the image zero-filled
@@ -997,7 +1020,7 @@ static bool gen_tma_ok() {
 }
 // 5-D view of a 2-D bricked bf16 tensor (identity BrickMap): (channel, x in brick, brick column, y in brick,
 // brick row over (n, by)); box = 64 channels x Bw x nseg bricks x 1 x 1, 128-B swizzled (the SW128 A layout).
-static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg) {
+static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int xstride = 1) {
     static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
     if (!enc) {
         cudaDriverEntryPointQueryResult qr;
@@ -1010,7 +1033,7 @@ static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg) {
                           (cuuint64_t)v.nb[0] * v.nb[1] * v.nb[2]};
     cuuint64_t strides[4] = {px, brick, px * v.B[3], brick * v.nb[3]};
     cuuint32_t box[5] = {64, (cuuint32_t)v.B[3], (cuuint32_t)nseg, 1, 1};
-    cuuint32_t es[5] = {1, 1, 1, 1, 1};
+    cuuint32_t es[5] = {1, (cuuint32_t)xstride, 1, 1, 1};   // xstride 2: every other pixel of a brick row
     return enc(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, v.ptr, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) ==
            CUDA_SUCCESS;
@@ -1219,6 +1242,11 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
             !G.src.bmap && G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
             gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw))
             G.tma = 1;
+        else if (!padded && G.amode == gen::AM_SW128 && G.k[0] == 1 && G.k[1] == 1 && G.k[2] == 1 && G.s[1] == 2 &&
+                 G.s[2] == 2 && G.pd[1] == 0 && G.pd[2] == 0 && nsp == 2 && !G.src.bmap && p->in_layout.Bw % 2 == 0 &&
+                 G.Tw % p->in_layout.Bw == 0 && 2 * G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
+                 gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, 2 * G.Tw / p->in_layout.Bw, 2))
+            G.tma = 2;
         G.has_res = sg.res_tensor[j] >= 0;
         if (G.has_res) G.res = res[j];
         G.relu = ly.L.relu;
