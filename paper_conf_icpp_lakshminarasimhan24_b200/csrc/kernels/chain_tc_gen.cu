@@ -23,6 +23,7 @@
 //   warps 7-22   epilogue: tcgen05.ld -> +bias (+residual) -> ReLU -> bf16 -> bricked global stores,
 //                then release-publish the tile (state 2)
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <string>
@@ -87,6 +88,8 @@ struct Params {
     // padded mode (§3.2.1): a task is a PB block of the last layer's output; every layer's
     // halo-extended region is recomputed by the CTA into its private scratch (two slots, so two blocks
     // interleave and one block's loads overlap the other's MMAs)
+    int dbg;                             // debug timing knobs (BDL_GEN_DBG): 1 = one k-step per task, 2 = no input loads,
+                                         // 4 = no epilogue stores (all give wrong results)
     unsigned long long *prof;            // debug (BDL_GEN_PROF): per CTA 16 x u64 of role wait / busy cycles, or null
     int padded;
     int PB[3], npb[3];
@@ -685,7 +688,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             for (int kb = 0; kb < L.nkb; kb++, gin++) {
                 const int s = gin % p.nin;
                 if (gin >= (uint32_t)p.nin) pwait(p, &sh.in_empty[s], ((gin / p.nin) - 1) & 1, wbuf);
-                load_stage(p, L, T, kb, in_ring + (size_t)s * p.in_stride, tid, &sh.in_full[s]);
+                if (!(p.dbg & 2)) load_stage(p, L, T, kb, in_ring + (size_t)s * p.in_stride, tid, &sh.in_full[s]);
                 // completion tracked by the barrier (the loader moves on to the next stage / task at once)
                 ptx::cp_async_arrive_noinc(&sh.in_full[s]);
             }
@@ -734,7 +737,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         // ------------------------------------------------------------------ MMA issuer
         const uint32_t tmem_base = __shfl_sync(0xffffffff, sh.tmem_base, 0);
         uint32_t gin = 0, gw = 0;
-        unsigned long long wdesc = 0, wacc = 0, win = 0, wwt = 0;
+        unsigned long long wdesc = 0, wacc = 0, win = 0, wwt = 0, wfence = 0;
         const unsigned long long t_start = clock64();
         for (uint32_t seq = 0;; seq++) {
             pwait(p, &sh.desc_full[seq % kRing], (seq / kRing) & 1, wdesc);
@@ -750,15 +753,17 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             for (int kb = 0; kb < L.nkb; kb++, gin++) {
                 const int s = gin % p.nin;
                 pwait(p, &sh.in_full[s], (gin / p.nin) & 1, win);
+                const unsigned long long tf0 = p.prof ? clock64() : 0;
                 ptx::fence_proxy_async_smem();   // cp.async (generic proxy) data -> tcgen05 operand reads
                 ptx::tc_fence_after();
+                if (p.prof) wfence += clock64() - tf0;
                 const uint32_t a_base = ptx::smem_u32(in_ring + (size_t)s * p.in_stride) >> 4;
                 for (int j = 0; j < L.nws; j++, gw++) {
                     const int st = gw % p.nw;
                     pwait(p, &sh.wfull[st], (gw / p.nw) & 1, wwt);
                     ptx::tc_fence_after();
                     const uint32_t b_base = ptx::smem_u32(w_ring + (size_t)st * p.w_stride) >> 4;
-                    const int q0 = j * L.kpw, q1 = min(L.nks, q0 + L.kpw);
+                    const int q0 = j * L.kpw, q1 = (p.dbg & 1) ? q0 + 1 : min(L.nks, q0 + L.kpw);
                     for (int q = q0; q < q1; q++) {
                         const uint2 e = sh.ks[l][q];
                         const uint64_t bd = ptx::umma_desc_noswz(0, lbo_b, 128) |
@@ -780,7 +785,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         }
         if (p.prof && lane == 0) {
             unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
-            r[6] = wdesc; r[7] = wacc; r[8] = win; r[9] = wwt; r[10] = clock64() - t_start;
+            r[6] = wdesc; r[7] = wacc; r[8] = win; r[9] = wwt; r[10] = clock64() - t_start; r[15] = wfence;
         }
     } else {
         // ------------------------------------------------------------------ epilogue
@@ -856,7 +861,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
 #pragma unroll
                         for (int e = 0; e < 8; e++) v[e] = fmaxf(v[e], 0.f);
                     }
-                    dst[k] = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
+                    if (!(p.dbg & 4))
+                        dst[k] = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
                 }
             }
             ptx::tc_fence_before();
@@ -925,6 +931,7 @@ static int gen_amode(int cin) {
 constexpr int kGenInBudget = 112 * 1024;   // input-stage ring
 constexpr int kGenWStage = 32 * 1024;      // one weight stage
 constexpr int kGenW = 3;                   // weight stages
+constexpr double kGenTaskOverheadMmas = 96.0;   // fixed per-task cost in units of one 128-row MMA (tile model)
 
 // Static (tile-independent) fields of a layer.  Returns false if the layer cannot run on the kernel.
 static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out, gen::LayerP &G) {
@@ -999,10 +1006,15 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
             cand.stage_bytes = (cand.stage_bytes + 1023) / 1024 * 1024;
             if (cand.stage_bytes * 2 > kGenInBudget) continue;
             const int nty = (cover_h + Tb - 1) / Tb, ntx = (cover_w + Tw - 1) / Tw;
-            // useful fraction of the MMA rows, then fewer loaded halo pixels per output
-            const double useful = (double)cover_h * cover_w / ((double)nty * ntx * cand.ntl * 128.0);
+            // time model per plane: tasks x (MMAs per task + a fixed per-task cost), times a penalty for loaded
+            // halo pixels.  The fixed cost (claim, dependency acquire, barriers, epilogue hand-off, publication)
+            // was measured on B200 at ~3.7 us per task with the MMAs, loads and stores disabled (cfg5,
+            // BDL_GEN_DBG=7), i.e. on the order of a hundred 128-row MMAs, so small tiles lose even when their
+            // MMA rows are better used.
             const double halo = (double)cand.in_rows * cand.in_cols / ((double)Tb * Tw * G.s[1] * G.s[2]);
-            const double score = useful - 0.1 * (halo - 1.0) + 1e-4 * Tb * Tw;
+            const double mmas = (double)cand.ntl * G.nks * G.nkb;
+            const double cost = (double)nty * ntx * (mmas + kGenTaskOverheadMmas) * (1.0 + 0.1 * (halo - 1.0));
+            const double score = -cost + 1e-6 * Tb * Tw;
             if (score > best) {
                 best = score;
                 G = cand;
@@ -1221,6 +1233,16 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
     memset(&P, 0, sizeof(P));
     P.L = L;
     P.prof = gen_prof_buffer(s);
+    if (const char *e = getenv("BDL_GEN_DBG")) P.dbg = atoi(e);
+    if (getenv("BDL_GEN_GEOM")) {
+        for (int j = 0; j < L; j++) {
+            const gen::LayerP &G = g.layer[j];
+            fprintf(stderr, "gen sg[%d..%d] layer %d: cin %d cout %d amode %d Tb %d Tw %d Wp %d ntl %d Nc %d nnc %d nkb %d nks %d kpw %d nws %d "
+                    "in_rows %d in_cols %d rowsA %d stage %d ntasks %lld | nin %d nw %d w_stride %d smem %d padded %d\n",
+                    sg.first, sg.last, j, G.cin, G.cout, G.amode, G.Tb, G.Tw, G.Wp, G.ntl, G.Nc, G.nnc, G.nkb, G.nks, G.kpw,
+                    G.nws, G.in_rows, G.in_cols, G.rowsA, G.stage_bytes, G.ntasks, g.nin, g.nw, g.w_stride, g.smem, (int)padded);
+        }
+    }
     const int nsp = p->in_layout.nsp;
     std::vector<TView> outs(L);
     for (int j = 0; j < L; j++) {

@@ -14,7 +14,7 @@ sgs = plan.subgraphs()
 ids = [int(a) for a in sys.argv[2:]] or range(len(sgs))
 f = lib().bdl_debug_gen_prof; f.restype = ctypes.c_int
 names = ["ld q_full", "ld deps", "ld in_empty", "ld total", "wp wempty", "wp total", "mma desc", "mma acc_empty",
-         "mma in_full", "mma wfull", "mma total", "epi desc", "epi acc_full", "epi bar", "epi total"]
+         "mma in_full", "mma wfull", "mma total", "epi desc", "epi acc_full", "epi bar", "epi total", "mma fence"]
 for i in ids:
     if sgs[i]["kernel"] != "tcgen05 generic":
         continue
@@ -28,3 +28,4 @@ for i in ids:
     desc = " ".join(f"{l['kind'][0]}{l['cin']}>{l['cout']}k{l['k'][-1]}s{l['stride'][-1]}" for l in ls)
     print(f"sg {i} {sgs[i]['mode']} {desc}: ctas {len(a)}  total {m[14]/1.9e3:.0f} us")
     print("   " + "  ".join(f"{n} {100*m[k]/max(m[14],1):.0f}%" for k, n in enumerate(names) if k not in (3, 5, 10, 14)))
+    print(f"   per-role totals (us): loader {m[3]/1.9e3:.0f} wprod {m[5]/1.9e3:.0f} mma {m[10]/1.9e3:.0f} epi {m[14]/1.9e3:.0f}")
