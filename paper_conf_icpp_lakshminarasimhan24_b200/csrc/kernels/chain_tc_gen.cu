@@ -652,7 +652,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             if (l > 0 && p.padded && wait >= 0 && warp == kLoad0) {
                 // padded: the source region is written by this CTA's epilogue of sub-task `wait`
                 if (lane == 0) {
-                    while (*reinterpret_cast<volatile int *>(&sh.done_seq) <= wait) __nanosleep(64);
+                    // atomic read of the CTA-local flag (release/acquire through fences around CTA-scope atomics)
+                    while (atomicOr_block(&sh.done_seq, 0) <= wait) __nanosleep(64);
                     __threadfence();
                 }
                 __syncwarp();
@@ -705,10 +706,16 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         for (uint32_t seq = 0;; seq++) {
             const int slot = seq % kQ;
             ptx::mbar_wait(&sh.q_full[slot], (seq / kQ) & 1);
-            const int l = sh.q_l[slot];
-            const long long t = sh.q_t[slot];
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&sh.q_empty[slot]);
+            // lane 0 reads the queue entry and releases the slot; the warp gets it by shuffle
+            int l = 0;
+            long long t = 0;
+            if (lane == 0) {
+                l = sh.q_l[slot];
+                t = sh.q_t[slot];
+                mbar_arrive(&sh.q_empty[slot]);
+            }
+            l = __shfl_sync(0xffffffff, l, 0);
+            t = __shfl_sync(0xffffffff, t, 0);
             if (l < 0) break;
             const LayerP &L = p.layer[l];
             const int nc = p.padded ? (int)((t >> 1) & 0xFF) : (int)(t % L.nnc);
@@ -874,7 +881,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             if (p.prof) web += clock64() - tb0;
             if (ew == 0 && lane == 0) {
                 __threadfence();
-                if (p.padded) *reinterpret_cast<volatile int *>(&sh.done_seq) = (int)seq + 1;
+                if (p.padded) atomicMax_block(&sh.done_seq, (int)seq + 1);
                 else if (p.only_layer < 0) st_release(status_word(p, l, t), (int)(EP | 2));
                 atomicAdd(&p.counters[0], 1ULL);
             }

@@ -10,7 +10,7 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "l1tex__throughput.avg.pct_of_peak_sustained_elapsed", "launch__registers_per_thread", "launch__grid_size",
         "launch__block_size", "launch__shared_mem_per_block_dynamic", "sm__cycles_elapsed.avg.per_second"]
 summary = {"round": R, "kernels": {}}
-for tag in ["memo_ws", "brickify", "padded", "gen_cfg5"]:
+for tag in ["memo_ws", "brickify", "padded", "gen_cfg5", "gen_cfg4"]:
     rep = os.path.join(OUT, f"{R}_{tag}.ncu-rep")
     if not os.path.exists(rep):
         continue
