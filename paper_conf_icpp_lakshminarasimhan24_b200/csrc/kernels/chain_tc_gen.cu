@@ -43,7 +43,7 @@ constexpr int kSched = 0, kLoad0 = 1, kLW = 4, kWProd = 5, kMma = 6, kEpi0 = 7, 
 constexpr int kThreads = 32 * (kEpi0 + kEpiW);
 constexpr int kLoadT = 32 * kLW;
 constexpr int kQ = 4, kRing = 16, kStack = 128;
-constexpr int kMaxIn = 4, kMaxW = 4, kMaxKs = 64;
+constexpr int kMaxIn = 4, kMaxW = 4, kMaxKs = 128;   // k-steps per layer: 3x3x3 taps x 64 channels = 108
 
 enum { AM_SW128 = 0, AM_PLANES = 1, AM_PAIR = 2 };
 
@@ -110,7 +110,7 @@ struct Shared {
     long long desc_t[kRing];
     int stk_l[kStack];
     long long stk_t[kStack];
-    uint2 ks[kMaxLayers][kMaxKs];        // per k-step: A offset (16-B units), LBO (16-B units)
+    uint32_t ks[kMaxLayers][kMaxKs];     // per k-step: A offset | LBO << 16 (both in 16-B units, < 2^14)
 };
 
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
@@ -597,7 +597,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         if (L.amode == AM_SW128) { aoff = (uint32_t)tap_px(tap) * 8 + kk * 2; lbo = 1; }
         else if (L.amode == AM_PLANES) { aoff = (uint32_t)tap_px(tap) + 2u * kk * L.rowsA; lbo = L.rowsA; }
         else { aoff = tap_px(tap); lbo = t1 >= 0 ? (uint32_t)(tap_px(t1) - tap_px(tap)) : 0u; }
-        sh.ks[l][q] = make_uint2(aoff, lbo);
+        sh.ks[l][q] = (aoff & 0xFFFF) | (lbo << 16);
     }
     if (threadIdx.x == 0) {
         for (int i = 0; i < kQ; i++) {
@@ -772,7 +772,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     const uint32_t b_base = ptx::smem_u32(w_ring + (size_t)st * p.w_stride) >> 4;
                     const int q0 = j * L.kpw, q1 = (p.dbg & 1) ? q0 + 1 : min(L.nks, q0 + L.kpw);
                     for (int q = q0; q < q1; q++) {
-                        const uint2 e = sh.ks[l][q];
+                        const uint32_t ev = sh.ks[l][q];
+                        const uint2 e = make_uint2(ev & 0xFFFF, ev >> 16);
                         const uint64_t bd = ptx::umma_desc_noswz(0, lbo_b, 128) |
                                             (uint64_t)((b_base + (q - q0) * ks_u) & 0x3FFF);
                         uint64_t ad0;

@@ -37,6 +37,10 @@ GRAPHS = {
     "planes_16_32": ([W.conv(16, 32, 3), W.conv(32, 32, 3)], 2, 16, 1, 20, 20, (1, 1, 8, 8)),
     "planes_3d": ([W.conv(32, 32, 3, nsp=3), W.conv(32, 32, 3, nsp=3)], 1, 32, 10, 12, 9, (1, 4, 4, 4)),
     "pool_tail": ([W.conv(64, 64, 3), W.conv(64, 64, 3), W.pool(64, 2, 2, 0)], 2, 64, 1, 20, 20, (1, 1, 8, 8)),
+    # 3x3x3 x 64 channels = 108 k-steps per layer (the Fig 10/11 microbenchmark layers)
+    "sw128_3d_c64": ([W.conv(64, 64, 3, nsp=3), W.conv(64, 64, 3, nsp=3)], 1, 64, 10, 12, 9, (1, 4, 4, 4)),
+    "sw128_3d_c64_valid": ([W.conv(64, 64, 3, 1, 0, nsp=3), W.conv(64, 64, 3, 1, 0, nsp=3)], 1, 64, 13, 12, 14,
+                           (1, 4, 4, 4)),
 }
 
 
