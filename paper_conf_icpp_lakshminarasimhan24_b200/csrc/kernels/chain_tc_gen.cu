@@ -45,7 +45,7 @@ constexpr int kLoadT = 32 * kLW;
 constexpr int kQ = 4, kRing = 16, kStack = 128;
 constexpr int kMaxIn = 4, kMaxW = 4, kMaxKs = 128;   // k-steps per layer: 3x3x3 taps x 64 channels = 108
 
-enum { AM_SW128 = 0, AM_PLANES = 1, AM_PAIR = 2 };
+enum { AM_SW128 = 0, AM_PLANES = 1, AM_PAIR = 2, AM_SW64 = 3 };   // AM_SW64: cin = 32, 64-B swizzled pixel rows
 
 struct LayerP {
     TView src, out, res;
@@ -61,6 +61,7 @@ struct LayerP {
     int amode, nkb, kc, nks, kpw, nws;   // kc: 16-B chunks per pixel per K-block
     int lkc;                  // log2(kc)
     int tma;                  // 1: the in-image columns of each input row arrive by one TMA box (tm_row)
+    int pxo;                  // SW64: pixel-row offset of the stage (0/1) that makes every TMA row start 128-B aligned
     int lB[3];                // log2 of the source view's brick extents (d, h, w)
     int rb, nblk, blk_px, plane_px;
     int in_rows, in_cols;
@@ -477,30 +478,34 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
         return;
     }
     if (L.tma && !T.src_scr) {
-        // stride-1 SW128 rows: the Tw in-tile columns of an in-image row by one TMA box (completion on `bar` by
-        // transaction count), halo columns by cp.async, rows outside the image zero-filled
+        // stride-1 swizzled rows (SW128: 64-channel K-block rows of 128 B; SW64: 32-channel rows of 64 B): the
+        // Tw in-tile columns of an in-image row by one TMA box (completion on `bar` by transaction count), halo
+        // columns by cp.async into the same swizzled layout, rows outside the image zero-filled
         const int l = (int)(&L - p.layer);
         const int pdw = L.pd[2];
         const int nh = L.in_cols - L.Tw;          // halo columns (k - 1)
+        const bool sw64 = L.amode == AM_SW64;
+        const int rb = sw64 ? 64 : 128, lrb = sw64 ? 6 : 7, nchr = sw64 ? 4 : 8;   // row bytes, log2, chunks / row
         for (int r2 = w; r2 < nrow; r2 += kLW) {
             const int a = r2 / L.in_rows, yy = r2 - a * L.in_rows;
             const int z = z0 + a, y = y0 + yy;
             const bool rok = z >= 0 && z < L.in_ext[0] && y >= 0 && y < L.in_ext[1];
-            const int rowpx = a * L.plane_px + yy * L.Wp;
+            const int rowpx = a * L.plane_px + yy * L.Wp + L.pxo;
             if (rok) {
                 if (lane == 0) {
-                    ptx::mbar_expect_tx(bar, (uint32_t)L.Tw * 128);
-                    const int by = y >> lBh;
-                    ptx::tma_load_5d(buf + (size_t)(rowpx + pdw) * 128, &p.tm_row[l], kb * 64, 0, T.x0 >> lBw,
-                                     y - (by << lBh), (T.n * v.nb[1] + z) * v.nb[2] + by, bar);
+                    ptx::mbar_expect_tx(bar, (uint32_t)(L.Tw * rb));
+                    const int bz = z >> lBd, by = y >> lBh;
+                    ptx::tma_load_5d(buf + ((size_t)(rowpx + pdw) << lrb), &p.tm_row[l], kb * 64, 0, T.x0 >> lBw,
+                                     ((z - (bz << lBd)) << lBh) + (y - (by << lBh)),
+                                     (T.n * v.nb[1] + bz) * v.nb[2] + by, bar);
                 }
             } else {
-                for (int q = lane; q < L.Tw * 8; q += 32)
-                    *reinterpret_cast<uint4 *>(buf + (size_t)(rowpx + pdw + (q >> 3)) * 128 + ((q & 7) << 4)) =
+                for (int q = lane; q < L.Tw * nchr; q += 32)
+                    *reinterpret_cast<uint4 *>(buf + ((size_t)(rowpx + pdw) << lrb) + ((size_t)q << 4)) =
                         make_uint4(0, 0, 0, 0);
             }
-            for (int q = lane; q < nh * 8; q += 32) {
-                const int hc = q >> 3, ch = q & 7;
+            for (int q = lane; q < nh * nchr; q += 32) {
+                const int hc = q / nchr, ch = q % nchr;
                 const int xx = hc < pdw ? hc : L.Tw + hc;
                 const int x = x0 + xx;
                 const bool ok = rok && x >= 0 && x < L.in_ext[2];
@@ -512,7 +517,9 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
                     const int in = ((((z - (bd << lBd)) << lBh) + (y - (by << lBh))) << lBw) + (x - (bx << lBw));
                     g = base + logical * v.brick_elems + (long long)in * v.Cp + kb * 64 + ch * 8;
                 }
-                ptx::cp_async16(buf + (uint32_t)px * 128 + ((ch ^ (px & 7)) << 4), g, ok ? 16u : 0u);
+                const uint32_t off = sw64 ? (uint32_t)px * 64 + ((ch ^ ((px >> 1) & 3)) << 4)
+                                          : (uint32_t)px * 128 + ((ch ^ (px & 7)) << 4);
+                ptx::cp_async16(buf + off, g, ok ? 16u : 0u);
             }
         }
         ptx::fence_proxy_async_smem();   // zero-filled rows (generic stores) -> tcgen05 operand reads
@@ -544,6 +551,10 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
             const int px = rowpx + (xx & ls2) * L.blk_px + (xx >> ls2);
             uint32_t off;
             if (L.amode == AM_SW128) off = (uint32_t)px * 128 + ((ch ^ (px & 7)) << 4);
+            else if (L.amode == AM_SW64) {
+                const int pq = px + L.pxo;
+                off = (uint32_t)pq * 64 + ((ch ^ ((pq >> 1) & 3)) << 4);
+            }
             else off = (uint32_t)ch * plane_bytes + (uint32_t)px * 16;
             const void *g = base;
             if (ok) {
@@ -582,6 +593,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         if (q >= L.nks) continue;
         int tap, kk = 0, t1 = -1;
         if (L.amode == AM_SW128) { tap = q / 4; kk = q % 4; }
+        else if (L.amode == AM_SW64) { tap = q / 2; kk = q % 2; }
         else if (L.amode == AM_PLANES) { const int kpt = (L.cin + 15) / 16; tap = q / kpt; kk = q % kpt; }
         else {   // pair taps (a, r, 2u) and (a, r, 2u+1)
             const int np = (L.k[2] + 1) / 2;
@@ -595,6 +607,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         };
         uint32_t aoff, lbo;
         if (L.amode == AM_SW128) { aoff = (uint32_t)tap_px(tap) * 8 + kk * 2; lbo = 1; }
+        else if (L.amode == AM_SW64) { aoff = (uint32_t)(tap_px(tap) + L.pxo) * 4 + kk * 2; lbo = 1; }
         else if (L.amode == AM_PLANES) { aoff = (uint32_t)tap_px(tap) + 2u * kk * L.rowsA; lbo = L.rowsA; }
         else { aoff = tap_px(tap); lbo = t1 >= 0 ? (uint32_t)(tap_px(t1) - tap_px(tap)) : 0u; }
         sh.ks[l][q] = (aoff & 0xFFFF) | (lbo << 16);
@@ -778,6 +791,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                                             (uint64_t)((b_base + (q - q0) * ks_u) & 0x3FFF);
                         uint64_t ad0;
                         if (L.amode == AM_SW128) ad0 = ptx::umma_desc_sw128(0, 1024);
+                        else if (L.amode == AM_SW64) ad0 = ptx::umma_desc_sw64(0, 512);
                         else ad0 = ptx::umma_desc_noswz(0, e.y * 16, 128);
                         for (int tl = 0; tl < L.ntl; tl++) {
                             const uint64_t ad = ad0 | (uint64_t)((a_base + e.x + tl * 128 * L.row_u) & 0x3FFF);
@@ -912,7 +926,7 @@ __global__ void pack_gen_kernel(const __nv_bfloat16 *__restrict__ w, __nv_bfloat
         const int nc = (int)(r / nkb);
         int tap, ci;
         if (amode == AM_SW128) { tap = q / 4; ci = kb * 64 + (q % 4) * 16 + j * 8 + e; }
-        else if (amode == AM_PLANES) { const int kpt = (cin + 15) / 16; tap = q / kpt; ci = (q % kpt) * 16 + j * 8 + e; }
+        else if (amode == AM_PLANES || amode == AM_SW64) { const int kpt = (cin + 15) / 16; tap = q / kpt; ci = (q % kpt) * 16 + j * 8 + e; }
         else {
             const int np = (kw + 1) / 2, u = q % np, ar = q / np;
             const int s = 2 * u + j;
@@ -929,9 +943,14 @@ __global__ void pack_gen_kernel(const __nv_bfloat16 *__restrict__ w, __nv_bfloat
 }  // namespace gen
 
 // ------------------------------------------------------------------------------------------------ host
+static bool gen_sw64_ok() {   // BDL_GEN_SW64=0: cin = 32 layers use the chunk-plane layout (A/B runs)
+    static const int v = [] { const char *e = getenv("BDL_GEN_SW64"); return e ? atoi(e) : 1; }();
+    return v != 0;
+}
 static int gen_amode(int cin) {
     if (cin <= 8) return gen::AM_PAIR;
     if (cin % 64 == 0) return gen::AM_SW128;
+    if (cin == 32 && gen_sw64_ok()) return gen::AM_SW64;
     if (cin % 16 == 0 && cin < 64) return gen::AM_PLANES;
     return -1;
 }
@@ -968,6 +987,7 @@ static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out,
     const int taps = G.k[0] * G.k[1] * G.k[2];
     if (G.amode == gen::AM_SW128) { G.nkb = l.cin / 64; G.kc = 8; G.nks = taps * 4; G.row_u = 8; }
     else if (G.amode == gen::AM_PLANES) { G.nkb = 1; G.kc = l.cin / 8; G.nks = taps * ((l.cin + 15) / 16); G.row_u = 1; }
+    else if (G.amode == gen::AM_SW64) { G.nkb = 1; G.kc = 4; G.nks = taps * 2; G.row_u = 4; }
     else { G.nkb = 1; G.kc = 1; G.nks = G.k[0] * G.k[1] * ((G.k[2] + 1) / 2); G.row_u = 1; }
     // the loader's address arithmetic uses shifts: power-of-two chunk counts and brick extents
     auto lg = [](int v) { int r = 0; while ((1 << r) < v) r++; return (1 << r) == v ? r : -1; };
@@ -1009,8 +1029,11 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
             int rows = std::max(G.k[0] * cand.plane_px, max_tap + cand.ntl * 128);
             rows = (rows + 7) / 8 * 8;
             if (G.amode == gen::AM_PLANES) rows += 1;   // odd plane stride: conflict-free loader stores
+            if (G.amode == gen::AM_SW64) rows = (rows + 1 + 7) / 8 * 8;   // room for the alignment offset pxo
             cand.rowsA = rows;
-            cand.stage_bytes = G.amode == gen::AM_SW128 ? rows * 128 : (G.amode == gen::AM_PLANES ? G.kc * rows * 16 : rows * 16);
+            cand.stage_bytes = G.amode == gen::AM_SW128 ? rows * 128
+                               : G.amode == gen::AM_SW64  ? rows * 64
+                               : (G.amode == gen::AM_PLANES ? G.kc * rows * 16 : rows * 16);
             cand.stage_bytes = (cand.stage_bytes + 1023) / 1024 * 1024;
             if (cand.stage_bytes * 2 > kGenInBudget) continue;
             const int nty = (cover_h + Tb - 1) / Tb, ntx = (cover_w + Tw - 1) / Tw;
@@ -1040,7 +1063,7 @@ static bool gen_tma_ok() {
 }
 // 5-D view of a 2-D bricked bf16 tensor (identity BrickMap): (channel, x in brick, brick column, y in brick,
 // brick row over (n, by)); box = 64 channels x Bw x nseg bricks x 1 x 1, 128-B swizzled (the SW128 A layout).
-static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int xstride = 1) {
+static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int xstride = 1, int box_ch = 64) {
     static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
     if (!enc) {
         cudaDriverEntryPointQueryResult qr;
@@ -1049,14 +1072,16 @@ static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int xs
             return false;
     }
     const cuuint64_t px = (cuuint64_t)v.Cp * 2, brick = (cuuint64_t)v.brick_elems * 2;
-    cuuint64_t dims[5] = {(cuuint64_t)v.Cp, (cuuint64_t)v.B[3], (cuuint64_t)v.nb[3], (cuuint64_t)v.B[2],
+    // dim 3 = row inside the brick (zin * Bh + yin: linear, stride one brick row of pixels), dim 4 = brick row
+    // over (n, bz, by)
+    cuuint64_t dims[5] = {(cuuint64_t)v.Cp, (cuuint64_t)v.B[3], (cuuint64_t)v.nb[3], (cuuint64_t)v.B[1] * v.B[2],
                           (cuuint64_t)v.nb[0] * v.nb[1] * v.nb[2]};
     cuuint64_t strides[4] = {px, brick, px * v.B[3], brick * v.nb[3]};
-    cuuint32_t box[5] = {64, (cuuint32_t)v.B[3], (cuuint32_t)nseg, 1, 1};
+    cuuint32_t box[5] = {(cuuint32_t)box_ch, (cuuint32_t)v.B[3], (cuuint32_t)nseg, 1, 1};
     cuuint32_t es[5] = {1, (cuuint32_t)xstride, 1, 1, 1};   // xstride 2: every other pixel of a brick row
     return enc(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, v.ptr, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-               CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) ==
-           CUDA_SUCCESS;
+               box_ch == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 // Debug profiler buffer (BDL_GEN_PROF=1): 16 x u64 per CTA, zeroed before each launch.
@@ -1268,10 +1293,20 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
         G.src = j == 0 ? in : outs[j - 1];
         G.out = outs[j];
         G.tma = 0;
+        G.pxo = 0;
         if (!padded && G.amode == gen::AM_SW128 && G.s[1] == 1 && G.s[2] == 1 && G.k[0] == 1 && nsp == 2 &&
             !G.src.bmap && G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
             gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw))
             G.tma = 1;
+        else if (!padded && G.amode == gen::AM_SW64 && G.s[0] == 1 && G.s[1] == 1 && G.s[2] == 1 && !G.src.bmap &&
+                 G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 && G.src.Cp == 32 &&
+                 G.Wp % 2 == 0 && G.plane_px % 2 == 0 && p->in_layout.Bd * p->in_layout.Bh <= 256 && gen_tma_ok() &&
+                 gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw, 1, 32)) {
+            // TMA destinations must be 128-B aligned: with even row pitches, shift the stage by one 64-B row when
+            // the first in-tile column (pd) is odd
+            G.tma = 1;
+            G.pxo = G.pd[2] & 1;
+        }
         else if (!padded && G.amode == gen::AM_SW128 && G.k[0] == 1 && G.k[1] == 1 && G.k[2] == 1 && G.s[1] == 2 &&
                  G.s[2] == 2 && G.pd[1] == 0 && G.pd[2] == 0 && nsp == 2 && !G.src.bmap && p->in_layout.Bw % 2 == 0 &&
                  G.Tw % p->in_layout.Bw == 0 && 2 * G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&

@@ -190,6 +190,17 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr, uint32_t sbo
     d |= (uint64_t)2 << 61;                              // SWIZZLE_128B
     return d;
 }
+// K-major SWIZZLE_64B descriptor: rows of 64 B (32 bf16), 8-row groups SBO apart; like SWIZZLE_128B the
+// swizzle is on absolute address bits, so any row offset is a plain start address (tools/swizzle64_test.cu).
+__device__ __forceinline__ uint64_t umma_desc_sw64(uint32_t saddr, uint32_t sbo_bytes) {
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+    d |= (uint64_t)1 << 16;
+    d |= (uint64_t)((sbo_bytes >> 4) & 0x3FFF) << 32;
+    d |= (uint64_t)1 << 46;
+    d |= (uint64_t)4 << 61;                              // SWIZZLE_64B
+    return d;
+}
 // Instruction descriptor kind::f16: D f32, A/B bf16, both K-major, shape M x N.
 __host__ __device__ constexpr uint32_t idesc_bf16_f32(int M, int N) {
     return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
