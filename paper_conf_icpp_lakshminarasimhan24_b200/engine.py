@@ -183,3 +183,72 @@ def plan_from_workload(wl, device="cuda", **opt_kw):
     opts = default_opts(**opt_kw) if opt_kw else None
     return Plan(wl["layers"], wl["weights"], wl["biases"], wl["N"], wl["C"], wl["D"], wl["H"], wl["W"],
                 wl["nsp"], wl["dtype"], wl["brick"], opts=opts, device=device)
+
+
+class HostPipeline:
+    """Pipelined host-to-host inference through a Plan (serving path).
+
+    Each request is a dense NC(D)HW tensor in pinned HOST memory.  Request k runs H2D copy -> brickify ->
+    merged subgraphs -> unbrickify -> D2H copy; the H2D of request k+1 and the D2H of request k-1 overlap
+    the merged execution of request k on three CUDA streams, with `slots` device/host buffer pairs.  All
+    computation is the plan's own kernels; PyTorch provides the streams, events and pinned buffers.
+    """
+
+    def __init__(self, plan, slots=2):
+        self.plan = plan
+        self.slots = slots
+        dev = plan.device
+        lo, li = plan.out_layout, plan.in_layout
+        self.in_shape = (li.N, li.C, li.D, li.H, li.W)
+        self.out_shape = (lo.N, lo.C, lo.D, lo.H, lo.W)
+        self.x_dev = [torch.empty(self.in_shape, dtype=plan.tdtype, device=dev) for _ in range(slots)]
+        self.y_dev = [torch.empty(self.out_shape, dtype=plan.tdtype, device=dev) for _ in range(slots)]
+        self.y_host = [torch.empty(self.out_shape, dtype=plan.tdtype).pin_memory() for _ in range(slots)]
+        self.xb = plan.alloc_bricked(li)
+        self.yb = plan.alloc_bricked(lo)
+        self.s_h2d, self.s_cmp, self.s_d2h = (torch.cuda.Stream(dev) for _ in range(3))
+
+    def run(self, inputs, on_output=None):
+        """Process the pinned host tensors `inputs` in order.  After request k's D2H completes, calls
+        on_output(k, y_host) (y_host is valid until the callback returns; its slot is then reused), or, with
+        on_output=None, returns the list of output copies.  Returns when everything is done."""
+        n, S = len(inputs), self.slots
+        h2d_done = [torch.cuda.Event() for _ in range(S)]
+        x_free = [torch.cuda.Event() for _ in range(S)]
+        cmp_done = [torch.cuda.Event() for _ in range(S)]
+        d2h_done = [torch.cuda.Event() for _ in range(S)]
+        used = [False] * S
+        outs = []
+
+        def drain(k):   # hand request k's output to the caller (waits for its D2H)
+            d2h_done[k % S].synchronize()
+            if on_output is not None:
+                on_output(k, self.y_host[k % S])
+            else:
+                outs.append(self.y_host[k % S].clone())
+
+        for k in range(n):
+            sl = k % S
+            if used[sl]:
+                drain(k - S)                                   # the host slot is reused by request k
+            with torch.cuda.stream(self.s_h2d):
+                if used[sl]:
+                    self.s_h2d.wait_event(x_free[sl])          # brickify of request k - S has read x_dev[sl]
+                self.x_dev[sl].copy_(inputs[k], non_blocking=True)
+                h2d_done[sl].record(self.s_h2d)
+            self.s_cmp.wait_event(h2d_done[sl])
+            if used[sl]:
+                self.s_cmp.wait_event(d2h_done[sl])            # D2H of request k - S has read y_dev[sl]
+            self.plan.brickify(self.x_dev[sl], out=self.xb, stream=self.s_cmp)
+            x_free[sl].record(self.s_cmp)
+            self.plan.run(self.xb, self.yb, stream=self.s_cmp)
+            self.plan.unbrickify(self.yb, out=self.y_dev[sl], stream=self.s_cmp)
+            cmp_done[sl].record(self.s_cmp)
+            with torch.cuda.stream(self.s_d2h):
+                self.s_d2h.wait_event(cmp_done[sl])
+                self.y_host[sl].copy_(self.y_dev[sl], non_blocking=True)
+                d2h_done[sl].record(self.s_d2h)
+            used[sl] = True
+        for k in range(max(0, n - S), n):
+            drain(k)
+        return None if on_output is not None else outs
