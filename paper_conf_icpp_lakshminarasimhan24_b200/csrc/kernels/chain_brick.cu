@@ -335,25 +335,56 @@ __global__ void __launch_bounds__(256) layer_kernel(GChain g, int l) {
 // 16-B store into the bricked output (consecutive threads -> consecutive 16-B chunks of a brick, so
 // loads and stores are coalesced along the channels-innermost brick rows).  Masked positions of
 // partial bricks and padded channels are written as 0 (Q11).
-template <typename T>
-__global__ void __launch_bounds__(256) pool_vec_kernel(GLayer ly, TView in, unsigned long long *counter) {
+// Element offset of channel 0 at (n, d, h, w) for power-of-two brick extents (log2 in lB[0..3]).
+__device__ __forceinline__ long long tv_off_p2(const TView &v, const int *lB, int n, int d, int h, int w) {
+    const int bn = n >> lB[0], bd = d >> lB[1], bh = h >> lB[2], bw = w >> lB[3];
+    const long long logical = (((long long)bn * v.nb[1] + bd) * v.nb[2] + bh) * v.nb[3] + bw;
+    const int in = ((((((n - (bn << lB[0])) << lB[1]) + (d - (bd << lB[1]))) << lB[2]) + (h - (bh << lB[2])))
+                    << lB[3]) + (w - (bw << lB[3]));
+    return tv_phys(v, logical) * v.brick_elems + (long long)in * v.Cp;
+}
+
+template <typename T, bool P2>
+__global__ void __launch_bounds__(256) pool_vec_kernel(GLayer ly, TView in, unsigned long long *counter, int4 lb4) {
+    const int lB[4] = {lb4.x, lb4.y, lb4.z, lb4.w};
     constexpr int V = 16 / sizeof(T);
     const TView &o = ly.out;
     const int nvec = o.Cp / V;
     const int bpx = o.B[0] * o.B[1] * o.B[2] * o.B[3];
     const long long nbr = (long long)o.nb[0] * o.nb[1] * o.nb[2] * o.nb[3];
     const long long total = nbr * bpx * nvec;
+    int lnv = 0, lbpx = lB[0] + lB[1] + lB[2] + lB[3];
+    while ((1 << lnv) < nvec) lnv++;
+    if ((1 << lnv) != nvec) lnv = -1;
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
-        const int cv = (int)(i % nvec);
-        long long r = i / nvec;
-        int inner = (int)(r % bpx);
-        long long b = r / bpx;   // logical brick
+        int cv, inner, inner0;
+        long long b;   // logical brick
+        if (P2 && lnv >= 0) {   // shifts only (power-of-two vectors per pixel and pixels per brick)
+            cv = (int)(i & (nvec - 1));
+            const long long r = i >> lnv;
+            inner = (int)(r & (bpx - 1));
+            b = r >> lbpx;
+        } else {
+            cv = (int)(i % nvec);
+            const long long r = i / nvec;
+            inner = (int)(r % bpx);
+            b = r / bpx;
+        }
+        inner0 = inner;
         int lo[4], ext[4];
         brick_region(o, b, lo, ext);
-        const int w = lo[3] + inner % o.B[3]; inner /= o.B[3];
-        const int h = lo[2] + inner % o.B[2]; inner /= o.B[2];
-        const int d = lo[1] + inner % o.B[1];
-        const int n = lo[0] + inner / o.B[1];
+        int w, h, d, n;
+        if (P2) {
+            w = lo[3] + (inner & ((1 << lB[3]) - 1)); inner >>= lB[3];
+            h = lo[2] + (inner & ((1 << lB[2]) - 1)); inner >>= lB[2];
+            d = lo[1] + (inner & ((1 << lB[1]) - 1));
+            n = lo[0] + (inner >> lB[1]);
+        } else {
+            w = lo[3] + inner % o.B[3]; inner /= o.B[3];
+            h = lo[2] + inner % o.B[2]; inner /= o.B[2];
+            d = lo[1] + inner % o.B[1];
+            n = lo[0] + inner / o.B[1];
+        }
         float m[V];
 #pragma unroll
         for (int j = 0; j < V; j++) m[j] = -INFINITY;
@@ -366,8 +397,8 @@ __global__ void __launch_bounds__(256) pool_vec_kernel(GLayer ly, TView in, unsi
                     for (int tw = 0; tw < ly.k[3]; tw++) {
                         const int iw = w * ly.s[3] - ly.p[3] + tw;
                         if (!inside4(ly.in_ext, n, id, ih, iw)) continue;
-                        const uint4 q = __ldg(reinterpret_cast<const uint4 *>(
-                            reinterpret_cast<const T *>(in.ptr) + tv_off(in, n, id, ih, iw) + cv * V));
+                        const long long eo = P2 ? tv_off_p2(in, lB, n, id, ih, iw) : tv_off(in, n, id, ih, iw);
+                        const uint4 q = __ldg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(in.ptr) + eo + cv * V));
                         const T *e = reinterpret_cast<const T *>(&q);
 #pragma unroll
                         for (int j = 0; j < V; j++) m[j] = fmaxf(m[j], to_f(e[j]));
@@ -385,7 +416,7 @@ __global__ void __launch_bounds__(256) pool_vec_kernel(GLayer ly, TView in, unsi
             oe[j] = from_f<T>(v);
         }
         *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(o.ptr) + tv_phys(o, b) * o.brick_elems +
-                                   (long long)(r % bpx) * o.Cp + cv * V) = outv;
+                                   (long long)inner0 * o.Cp + cv * V) = outv;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(counter, (unsigned long long)nbr);
 }
@@ -482,8 +513,16 @@ bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &i
             if (G.kind == BDL_OP_MAXPOOL && !G.res_ext && (G.out.Cp * esz) % 16 == 0 && (src.Cp * esz) % 16 == 0) {
                 const long long threads = nb * G.out.B[0] * G.out.B[1] * G.out.B[2] * G.out.B[3] * (G.out.Cp * esz / 16);
                 const int gp = (int)std::min<long long>((threads + 255) / 256, 148LL * 64);
-                if (g.bf16) pool_vec_kernel<__nv_bfloat16><<<gp, 256, 0, s>>>(G, src, g.counters);
-                else pool_vec_kernel<float><<<gp, 256, 0, s>>>(G, src, g.counters);
+                auto lg = [](int v) { int r = 0; while ((1 << r) < v) r++; return (1 << r) == v ? r : -1; };
+                const int4 lb4 = make_int4(lg(src.B[0]), lg(src.B[1]), lg(src.B[2]), lg(src.B[3]));
+                const bool p2 = lb4.x >= 0 && lb4.y >= 0 && lb4.z >= 0 && lb4.w >= 0;
+                if (g.bf16) {
+                    if (p2) pool_vec_kernel<__nv_bfloat16, true><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);
+                    else pool_vec_kernel<__nv_bfloat16, false><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);
+                } else {
+                    if (p2) pool_vec_kernel<float, true><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);
+                    else pool_vec_kernel<float, false><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);
+                }
                 *launches += 1;
                 continue;
             }
