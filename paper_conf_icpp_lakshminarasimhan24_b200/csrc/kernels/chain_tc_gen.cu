@@ -1120,9 +1120,23 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
         if (!gen_layer_static(ly, nsp, lo, g.layer[j])) return false;
     }
     if (padded && nconv > 1) {
-        // blocks of the planner's brick edge (rho/tau model, L649-658) over the last layer's grid
+        // CTA blocks over the last layer's grid.  The planner's brick edge (rho/tau model, L649-658) sizes the
+        // layout; a CTA's padded block is a band of bricks: start from the brick edge and double
+        // while at least one block per SM remains, so small maps (7x7, 14x14) do not end up with 4x4 blocks whose
+        // 128-row MMA tiles are mostly empty and whose halos are recomputed four times per image.
         const gen::LayerP &last = g.layer[nconv - 1];
-        const int B = std::max(1, sg.model_brick);
+        int B = std::max(1, sg.model_brick);
+        const long long nimg = p->layers[sg.first].in_ext[0];
+        auto nblocks = [&](int b) {
+            long long n = nimg;
+            for (int d = 0; d < 3; d++)
+                if (d > 0 || nsp == 3) n *= (last.grid[d] + b - 1) / b;
+            return n;
+        };
+        int maxg = 1;
+        for (int d = 0; d < 3; d++)
+            if (d > 0 || nsp == 3) maxg = std::max(maxg, last.grid[d]);
+        while (B < maxg && B < 64 && nblocks(2 * B) >= (long long)p->num_sms) B *= 2;
         for (int d = 0; d < 3; d++) {
             const bool spatial = d > 0 || nsp == 3;
             g.PB[d] = spatial ? std::min(B, last.grid[d]) : 1;
