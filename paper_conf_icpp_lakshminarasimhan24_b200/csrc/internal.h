@@ -86,7 +86,6 @@ struct Subgraph {
     int64_t norder = 0;
     std::vector<int> order_host;
     // tap-shared tcgen05 kernel: per-layer ticket counter bases (advanced deterministically every run)
-    std::vector<uint64_t> ts_tbase;
 };
 
 }  // namespace bdl

@@ -93,13 +93,8 @@ struct Params {
     int only_layer;
     unsigned long long *trace;      // debug: 8 x u64 per task, or null
     int trace_cap;
-    // tap-shared kernel (memo_ts_kernel): per-layer task queues
-    long long ts_nper;                // tasks per layer (order[l * ts_nper + k] = k-th task of layer l)
-    int ts_batch;                     // tickets drawn per atomic (same-address atomics serialize in L2)
-    unsigned long long ts_tbase[kMaxLayers];   // ticket counter base of each layer's queue (counters[8 + l])
     int dbg;                        // debug timing knobs (BDL_WS_DBG): 1 = no MMA, 2 = no epilogue math/stores,
-                                    // 4 = direct (unstaged) epilogue stores, 8 = weights not re-streamed,
-                                    // 16 = residual not fetched; results are wrong for 1, 2, 8, 16
+                                    // 8 = weights not re-streamed, 16 = residual not fetched (all give wrong results)
 };
 
 struct Shared {
@@ -809,533 +804,6 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
     if (warp == kMmaWarp) ptx::tmem_dealloc(sh.tmem_base, p.tmem_cols);
 }
 
-// ============================================================================================== tap-shared
-// C = 64 chains, MEMOIZED / unmerged (§3.2.2).  One tcgen05.mma per (kernel row r, 16-channel
-// k-step) with N = 192: the three column taps s = 0, 1, 2 of row r are stacked along N and share one A
-// operand -- the input tile rows starting at r * Wt, no column shift.  Accumulator block s then holds in
-// TMEM lane m the tap-(r, s) partial sums of output row m - s, and the epilogue forms
-//     out[i] = D0[i] + D1[i + 1] + D2[i + 2]          (i < 126 = rows per M tile)
-// with warp shuffles; the lanes that cross a 32-lane TMEM quadrant come through shared memory.  Each
-// A byte read from shared memory now feeds three taps: per 128 x 64 x 16 MAC block the SS-MMA reads
-// 3.3 KB instead of 6 KB, so the MMA is tensor-bound (96 cycles per 3 taps) instead of shared-memory
-// bound (3 x 48 cycles).
-//
-// Memo protocol (L513-531): every task (layer, band) is claimed by CAS 0 -> 1 from its layer's queue and
-// released 1 -> 2 after its global stores.  Each CTA keeps ONE layer's weights resident (72 KB) and
-// drains that layer's queue (CTA c starts on layer c % L and moves on to the next layer when its queue is
-// empty); a task whose dependencies are not complete waits for them -- the paper's "moves on ... and
-// revisits" (L523-525) -- instead of computing them with another layer's weights.  Layer l never waits
-// on layers >= l and the grid is co-resident, so the schedule cannot deadlock.
-//
-// Roles: warp 0 scheduler, warp 1 loader (dependency wait + TMA input tile), warp 2 MMA issuer (also
-// (re)loads the resident weights), warps 3-18 epilogue (TMEM -> shifted tap sum -> bias/residual/ReLU ->
-// bf16 -> direct 32-B global stores -> publication).
-
-// Input tile of a task into one (128-B swizzled) buffer without waiting on any copy: in-image rows by one
-// 5-D TMA box each (completion on `bar` by transaction count), rows outside the image zeroed with
-// shared-memory stores.  Full-width bands (ntx == 1) have both halo columns outside the image; they are
-// zeroed once at kernel start (TMA never writes them).  Otherwise the halo pixels are copied with cp.async
-// and waited for.
-__device__ __forceinline__ void ts_load_tile(const Params &p, int src_l, const TView &src, int n, int y0, int x0,
-                                             uint8_t *buf, uint64_t *bar, int lane) {
-    const int R = p.Tb + 2, Wt = p.Wt, Bh = 1 << p.lBh;
-    const uint32_t bytes = (uint32_t)p.Tw * 128;
-    for (int a = lane; a < R; a += 32) {
-        const int y = y0 - 1 + a;
-        uint8_t *dst = buf + (size_t)(a * Wt + 1) * 128;
-        if (y >= 0 && y < p.H) {
-            const int by = y >> p.lBh;
-            ptx::mbar_expect_tx(bar, bytes);
-            ptx::tma_load_5d(dst, &p.tm_row[src_l], 0, 0, x0 >> p.lBw, y - by * Bh, n * src.nb[2] + by, bar);
-        }
-    }
-    for (int a = 0; a < R; a++) {
-        const int y = y0 - 1 + a;
-        if (y >= 0 && y < p.H) continue;
-        uint4 *dst = reinterpret_cast<uint4 *>(buf + (size_t)(a * Wt + 1) * 128);
-        for (int q = lane; q < p.Tw * 8; q += 32) dst[q] = make_uint4(0, 0, 0, 0);
-    }
-    if (p.ntx > 1) {
-        const __nv_bfloat16 *base = reinterpret_cast<const __nv_bfloat16 *>(src.ptr);
-        for (int it = lane; it < R * 2 * 8; it += 32) {
-            const int k = it % 8, hp = it / 8;
-            const int a = hp >> 1, side = hp & 1;
-            const int y = y0 - 1 + a, x = side ? x0 + p.Tw : x0 - 1;
-            uint8_t *row = buf + (size_t)(a * Wt + (side ? Wt - 1 : 0)) * 128;
-            const uint32_t sw = (((ptx::smem_u32(row) >> 7) & 7) ^ (k & 7)) * 16;
-            const bool ok = y >= 0 && y < p.H && x >= 0 && x < p.W;
-            const void *g = ok ? (const void *)(base + pix_off(src, p.lBh, p.lBw, n, y, x) + k * 8) : (const void *)base;
-            ptx::cp_async16(row + sw, g, ok ? 16u : 0u);
-        }
-        ptx::cp_async_wait_all();
-    }
-    ptx::fence_proxy_async_smem();
-    __syncwarp();
-}
-
-namespace ts {
-constexpr int kSched = 0, kLoad = 1, kMma = 2, kPub = 3, kEpi0 = 4, kEpiW = 16;
-constexpr int kThreads = 32 * (kEpi0 + kEpiW);
-constexpr int kRingT = 16;             // task descriptor ring (loader -> MMA -> epilogue -> publisher)
-constexpr int kRowsT = 126;             // valid output rows per M = 128 tile
-constexpr int kN = 192;                 // 3 taps x 64 output channels
-constexpr int kWBytes = 9 * 64 * 64 * 2;
-constexpr int kAccCols = 256;           // TMEM columns per accumulator (2 accumulators, 512 allocated)
-
-struct Shared {
-    uint64_t q_full[kQ], q_empty[kQ];
-    uint64_t in_full[kMaxIn], in_empty[kMaxIn], acc_full[2], acc_empty[2], desc_full[kRingT];
-    uint64_t wfull, wdrain;
-    uint32_t tmem_base;
-    int q_l[kQ];
-    long long q_t[kQ];
-    uint64_t stored[kRingT], pub_done[kRingT];   // epilogue stores of a task done (16 warps) / task published
-    int desc_l[kRingT], desc_n[kRingT], desc_y0[kRingT], desc_x0[kRingT];
-    long long desc_t[kRingT];
-    // [group][task parity within group][channel half][chunk][quadrant][D1 lane0, D2 lane0, D2 lane1][16 ch]
-    float xch[2][2][2][2][4][3][16];
-    unsigned long long tr[kRingT][8];    // debug trace timestamps per task slot
-};
-
-// debug (p.trace with BDL_TSPROF): cycles each role spends blocked in mbarrier waits
-__device__ __forceinline__ void twait(uint64_t *bar, uint32_t parity, unsigned long long &acc) {
-    const unsigned long long t0 = clock64();
-    ptx::mbar_wait(bar, parity);
-    acc += clock64() - t0;
-}
-__device__ __forceinline__ void prof_out(const Params &p, int role, unsigned long long wait, unsigned long long t_start) {
-    if (p.dbg & 256) {
-        unsigned long long *rec = p.trace + ((size_t)blockIdx.x * 8 + role) * 2;
-        rec[0] = wait;
-        rec[1] = clock64() - t_start;
-    }
-}
-
-__device__ void scheduler(const Params &p, Shared &sh) {
-    const int lane = threadIdx.x % 32;
-    const unsigned EP = p.epoch << 2;
-    const bool unmerged = p.only_layer >= 0;
-    int l = unmerged ? p.only_layer : (int)(blockIdx.x % p.L);
-    unsigned long long oks = 0, wcyc = 0;
-    const unsigned long long t_start = clock64();
-    uint32_t qseq = 0;
-    auto emit = [&](int el, long long t) {
-        const int slot = qseq % kQ;
-        if (qseq >= (uint32_t)kQ) twait(&sh.q_empty[slot], ((qseq / kQ) - 1) & 1, wcyc);
-        if (lane == 0) {
-            sh.q_l[slot] = el;
-            sh.q_t[slot] = t;
-            mbar_arrive(&sh.q_full[slot]);
-        }
-        __syncwarp();
-        qseq++;
-    };
-    const int B = p.ts_batch;
-    for (;;) {
-        // draw B consecutive tickets with one atomic; lanes 0..B-1 claim them in parallel (CAS 0 -> 1)
-        unsigned long long tk = 0;
-        if (lane == 0) tk = atomicAdd(&p.counters[8 + l], (unsigned long long)B) - p.ts_tbase[l];
-        tk = __shfl_sync(0xffffffff, tk, 0);
-        if ((long long)tk < 0) __trap();   // ticket accounting broken: fail loudly
-        if ((long long)tk >= p.ts_nper) {
-            if (unmerged || l == p.L - 1) break;
-            l++;                            // this layer's queue is drained: move on to the next layer
-            continue;
-        }
-        const long long rem = p.ts_nper - (long long)tk;
-        const int cnt = rem < B ? (int)rem : B;
-        long long t = 0;
-        if (lane < cnt) {
-            t = p.order ? (long long)p.order[(long long)l * p.ts_nper + (long long)tk + lane] : (long long)tk + lane;
-            if (!unmerged) {
-                int *sw = status_word(p, l, t);
-                const int cur = ld_acquire(sw);
-                const bool ok = tag_state(cur, EP) == 0 && atomicCAS(sw, cur, (int)(EP | 1)) == cur;
-                if (!ok) __trap();          // every task sits in exactly one queue: a failed claim is a bug
-            }
-        }
-        if (!unmerged) oks += cnt;
-        for (int k = 0; k < cnt; k++) emit(l, __shfl_sync(0xffffffff, t, k));
-    }
-    emit(-1, 0);
-    if (lane == 0 && oks) atomicAdd(&p.counters[1], oks);
-    if (lane == 0) prof_out(p, 0, wcyc, t_start);
-}
-
-__global__ void __launch_bounds__(kThreads, 1) memo_ts_kernel(const __grid_constant__ Params p) {
-    constexpr int C = 64;
-    extern __shared__ __align__(1024) uint8_t smem[];
-    __shared__ Shared sh;
-    const int warp = __shfl_sync(0xffffffff, (int)threadIdx.x / 32, 0), lane = threadIdx.x % 32;
-    const size_t in_bytes = (size_t)p.rowsA * 128;
-    uint8_t *wbuf = smem + in_bytes * p.nin;                                   // [3 r][8 k-chunks][192 n][16 B]
-    float *bias_s = reinterpret_cast<float *>(wbuf + kWBytes);                 // [L][64]
-    for (int i = threadIdx.x; i < p.L * C; i += kThreads) bias_s[i] = p.layer[i / C].bias[i % C];
-    if (ptx::smem_u32(smem) & 1023) __trap();
-    if (p.ntx == 1) {   // halo columns of full-width bands lie outside the image: zero once, never written again
-        const int R = p.Tb + 2;
-        for (int i = threadIdx.x; i < p.nin * R * 2 * 8; i += kThreads) {
-            const int k = i % 8, hp = (i / 8) % (2 * R), b = i / (16 * R);
-            const int a = hp >> 1, side = hp & 1;
-            *reinterpret_cast<uint4 *>(smem + in_bytes * b + (size_t)(a * p.Wt + (side ? p.Wt - 1 : 0)) * 128 + k * 16) =
-                make_uint4(0, 0, 0, 0);
-        }
-    }
-
-    if (threadIdx.x == 0) {
-        for (int i = 0; i < kQ; i++) {
-            ptx::mbar_init(&sh.q_full[i], 1);
-            ptx::mbar_init(&sh.q_empty[i], 1);
-        }
-        for (int i = 0; i < kMaxIn; i++) {
-            ptx::mbar_init(&sh.in_full[i], 1);
-            ptx::mbar_init(&sh.in_empty[i], 1);
-        }
-        for (int i = 0; i < 2; i++) {
-            ptx::mbar_init(&sh.acc_full[i], 1);
-            ptx::mbar_init(&sh.acc_empty[i], kEpiW / 2);   // one epilogue group (8 warps) per accumulator
-        }
-        for (int i = 0; i < kRingT; i++) {
-            ptx::mbar_init(&sh.desc_full[i], 1);
-            ptx::mbar_init(&sh.stored[i], kEpiW / 2);
-            ptx::mbar_init(&sh.pub_done[i], 1);
-        }
-        ptx::mbar_init(&sh.wfull, 1);
-        ptx::mbar_init(&sh.wdrain, 1);
-        ptx::fence_barrier_init();
-    }
-    if (warp == kMma) {
-        ptx::tmem_alloc(&sh.tmem_base, 2 * kAccCols);
-        ptx::tmem_relinquish();
-    }
-    ptx::fence_proxy_async_smem();
-    ptx::tc_fence_before();
-    __syncthreads();
-    ptx::tc_fence_after();
-    pdl_launch_dependents();
-    // PDL: the loader and epilogue read the previous kernel's output; the scheduler rewrites memo tags that the
-    // previous run of this subgraph may still be waiting on -- all wait for the previous grid.  Only the MMA
-    // warp's weight load (prepared buffers) starts early.
-    if (warp != kMma) pdl_wait();
-
-    const unsigned EP = p.epoch << 2;
-    if (warp == kSched) {
-        scheduler(p, sh);
-    } else if (warp == kLoad) {
-        // ------------------------------------------------------------------ loader
-        unsigned long long spins_total = 0, wcyc = 0, dcyc = 0;
-        const unsigned long long t_start = clock64();
-        for (uint32_t seq = 0;; seq++) {
-            const int slot = seq % kQ;
-            twait(&sh.q_full[slot], (seq / kQ) & 1, wcyc);
-            const int l = sh.q_l[slot];
-            const long long t = sh.q_t[slot];
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&sh.q_empty[slot]);
-            const int b = seq % p.nin;
-            const unsigned long long t_q = gtime();
-            if (seq >= (uint32_t)p.nin) twait(&sh.in_empty[b], ((seq / p.nin) - 1) & 1, wcyc);
-            const unsigned long long t_buf = gtime();
-            int n = 0, ty = 0, tx = 0;
-            if (l >= 0) decode(p, t, n, ty, tx);
-            if (l >= 0) {
-                if (l > 0 && p.only_layer < 0) {
-                    long long dt;
-                    unsigned long long spins = 0;
-                    if (dep_of(p, t, lane, dt)) {
-                        const int *dw = status_word(p, l - 1, dt);
-                        while (ld_acquire(dw) != (int)(EP | 2)) {
-                            spins++;
-                            __nanosleep(64);
-                        }
-                    }
-                    __syncwarp();
-                    spins_total += spins;
-                    ptx::fence_proxy_async();   // acquired data is read by TMA (async proxy)
-                }
-                const TView &src = l == 0 ? p.in : p.layer[l - 1].out;
-                ts_load_tile(p, l, src, n, ty * p.Tb, tx * p.Tw, smem + in_bytes * b, &sh.in_full[b], lane);
-            }
-            // descriptor ring slot reuse: the task kRingT back must be published
-            if (seq >= (uint32_t)kRingT) twait(&sh.pub_done[seq % kRingT], ((seq / kRingT) - 1) & 1, wcyc);
-            if (lane == 0) {
-                sh.desc_l[seq % kRingT] = l;
-                sh.desc_t[seq % kRingT] = t;
-                sh.desc_n[seq % kRingT] = n;
-                sh.desc_y0[seq % kRingT] = ty * p.Tb;
-                sh.desc_x0[seq % kRingT] = tx * p.Tw;
-                sh.tr[seq % kRingT][0] = t_q;
-                sh.tr[seq % kRingT][1] = t_buf;
-                sh.tr[seq % kRingT][2] = gtime();
-                mbar_arrive(&sh.desc_full[seq % kRingT]);
-                mbar_arrive(&sh.in_full[b]);
-            }
-            __syncwarp();
-            if (l < 0) {
-                // the two epilogue groups take alternate tasks: the other group needs its own end marker
-                const uint32_t s2 = seq + 1;
-                if (s2 >= (uint32_t)kRingT) ptx::mbar_wait(&sh.pub_done[s2 % kRingT], ((s2 / kRingT) - 1) & 1);
-                if (lane == 0) {
-                    sh.desc_l[s2 % kRingT] = -1;
-                    mbar_arrive(&sh.desc_full[s2 % kRingT]);
-                }
-                __syncwarp();
-                break;
-            }
-        }
-        for (int o = 16; o; o >>= 1) spins_total += __shfl_xor_sync(0xffffffff, spins_total, o);
-        if (lane == 0 && spins_total) atomicAdd(&p.counters[3], spins_total);
-        if (lane == 0) prof_out(p, 1, wcyc, t_start);
-    } else if (warp == kMma) {
-        // ------------------------------------------------------------------ MMA issuer
-        constexpr uint32_t IDESC = ptx::idesc_bf16_f32(128, kN);
-        constexpr uint32_t LBO_B = kN * 16;                     // between the two 8-channel chunks of a k-step
-        const uint64_t adesc0 = ptx::umma_desc_sw128(0, 1024);
-        const uint64_t bdesc0 = ptx::umma_desc_noswz(0, LBO_B, 128);
-        const uint32_t tmem_base = __shfl_sync(0xffffffff, sh.tmem_base, 0);
-        const uint32_t w_u = ptx::smem_u32(wbuf) >> 4;
-        int cur_l = -1;
-        uint32_t wphase = 0;
-        unsigned long long wcyc = 0, wcyc2 = 0;
-        const unsigned long long t_start = clock64();
-        for (uint32_t seq = 0;; seq++) {
-            const int b = seq % p.nin, a = seq & 1;
-            twait(&sh.in_full[b], (seq / p.nin) & 1, wcyc);
-            const int l = sh.desc_l[seq % kRingT];
-            if (seq >= 2) twait(&sh.acc_empty[a], ((seq >> 1) - 1) & 1, wcyc2);
-            if (l < 0) {
-                if (lane == 0) mbar_arrive(&sh.acc_full[a]);
-                break;
-            }
-            if (l != cur_l) {
-                // (re)load this layer's weights: [tap][8 chunks][64 co][8] -> [r][chunk][s*64 + co][8]
-                if (cur_l >= 0) {   // wait until every MMA that reads the old weights has completed
-                    ptx::mma_commit_elect(&sh.wdrain);
-                    ptx::mbar_wait(&sh.wdrain, (wphase - 1) & 1);   // drain k precedes weight load k+1
-                }
-                const uint8_t *wg = reinterpret_cast<const uint8_t *>(p.layer[l].w);
-                if (lane == 0) ptx::mbar_arrive_expect_tx(&sh.wfull, kWBytes);
-                __syncwarp();
-                for (int piece = lane; piece < 72; piece += 32) {
-                    const int tap = piece / 8, ch = piece % 8, r = tap / 3, s = tap % 3;
-                    ptx::bulk_g2s(wbuf + ((size_t)(r * 8 + ch) * kN + s * 64) * 16, wg + (size_t)piece * 1024, 1024,
-                                  &sh.wfull);
-                }
-                ptx::mbar_wait(&sh.wfull, wphase & 1);
-                wphase++;
-                cur_l = l;
-            }
-            ptx::tc_fence_after();
-            if (lane == 0) sh.tr[seq % kRingT][3] = gtime();
-            const uint32_t a_u = ptx::smem_u32(smem + in_bytes * b) >> 4;
-            const uint32_t d = tmem_base + a * kAccCols;
-            if (!(p.dbg & 1)) {
-#pragma unroll
-                for (int r = 0; r < 3; r++) {
-#pragma unroll
-                    for (int kk = 0; kk < 4; kk++) {
-                        const uint64_t ad = adesc0 | (uint64_t)((a_u + (uint32_t)(r * p.Wt) * 8 + kk * 2) & 0x3FFF);
-                        const uint64_t bd = bdesc0 | (uint64_t)((w_u + (uint32_t)(r * 8 + 2 * kk) * kN) & 0x3FFF);
-                        ptx::mma_bf16_elect(d, ad, bd, IDESC, (r | kk) != 0);
-                    }
-                }
-            }
-            if (lane == 0) sh.tr[seq % kRingT][4] = gtime();
-            ptx::mma_commit_elect(&sh.in_empty[b]);
-            ptx::mma_commit_elect(&sh.acc_full[a]);
-            __syncwarp();
-        }
-        if (lane == 0) {
-            prof_out(p, 2, wcyc, t_start);
-            prof_out(p, 5, wcyc2, t_start);
-        }
-    } else if (warp == kPub) {
-        // ------------------------------------------------------------------ publisher
-        // memo state 2 once all 16 epilogue warps' global stores of the task are done (their mbarrier arrivals
-        // release them at CTA scope; the GPU-scope fence + release store make them visible to other CTAs).
-        // Every task already stored when the publisher gets to it shares one fence.
-        unsigned long long computed = 0, wcyc = 0;
-        const unsigned long long t_start = clock64();
-        uint32_t seq = 0;
-        for (bool done = false; !done;) {
-            uint32_t s1 = seq;   // [seq, s1): tasks stored and ready to publish
-            for (;;) {
-                const int slot = s1 % kRingT;
-                if (s1 == seq) {
-                    twait(&sh.desc_full[slot], (s1 / kRingT) & 1, wcyc);
-                } else if (s1 - seq >= (uint32_t)kRingT / 2 || !ptx::mbar_test(&sh.desc_full[slot], (s1 / kRingT) & 1)) {
-                    break;
-                }
-                if (sh.desc_l[slot] < 0) {
-                    done = true;
-                    break;
-                }
-                if (s1 == seq) twait(&sh.stored[slot], (s1 / kRingT) & 1, wcyc);
-                else if (!ptx::mbar_test(&sh.stored[slot], (s1 / kRingT) & 1)) break;
-                s1++;
-            }
-            if (s1 == seq) continue;
-            if (lane == 0) {
-                const unsigned long long t_sync = gtime();
-                if (p.only_layer < 0 && !(p.dbg & 32)) __threadfence();   // debug 32: no fence (timing only)
-                for (uint32_t k = seq; k < s1; k++) {
-                    const int slot = k % kRingT;
-                    const int l = sh.desc_l[slot];
-                    const long long t = sh.desc_t[slot];
-                    if (p.only_layer < 0) st_release(status_word(p, l, t), (int)(EP | 2));
-                    if (p.trace && !(p.dbg & 256)) {
-                        const unsigned long long r = atomicAdd(&p.counters[5], 1ULL);
-                        if (r < (unsigned long long)p.trace_cap) {
-                            unsigned smid;
-                            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-                            unsigned long long *rec = p.trace + r * 12;
-                            rec[0] = ((unsigned long long)smid << 40) | ((unsigned long long)blockIdx.x << 8) | (unsigned)l;
-                            rec[1] = (unsigned long long)t;
-                            for (int f = 0; f < 7; f++) rec[2 + f] = sh.tr[slot][f];
-                            rec[9] = t_sync;
-                            rec[10] = gtime();
-                            rec[11] = gtime();
-                        }
-                    }
-                    mbar_arrive(&sh.pub_done[slot]);
-                }
-            }
-            computed += s1 - seq;
-            seq = s1;
-            __syncwarp();
-        }
-        if (lane == 0 && computed) atomicAdd(&p.counters[0], computed);
-        if (lane == 0) prof_out(p, 3, wcyc, t_start);
-    } else {
-        // ------------------------------------------------------------------ epilogue
-        // Two groups of 8 warps; group g takes the tasks with seq % 2 == g (= accumulator g), so two tasks'
-        // epilogues run concurrently.  Within a group, warp (q = warp % 4, h) reads TMEM lane quadrant q (tile rows
-        // 32q..32q+31) and output channels 32h..32h+31 in two 16-channel chunks.
-        const int ew = warp - kEpi0, q = warp % 4, g = ew / 8, h = (ew / 4) % 2;
-        const int Hg = p.layer[0].out.nb[2] << p.lBh, Wg = p.layer[0].out.nb[3] << p.lBw;
-        const int i = q * 32 + lane;                 // tile row of this thread
-        const int ii = i / p.Wt, jj = i - ii * p.Wt;
-        const int mh = (1 << p.lBh) - 1, mw = (1 << p.lBw) - 1;
-        const int nb2 = p.layer[0].out.nb[2], nb3 = p.layer[0].out.nb[3];
-        const long long be = p.layer[0].out.brick_elems;   // every tensor of the chain shares the bricked geometry
-        const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(p.res.ptr);
-        const bool fix = q < 3 && lane >= 30;        // D1 / D2 rows of the next quadrant (shared memory)
-        unsigned long long wcyc = 0, bcyc = 0;
-        const unsigned long long t_start = clock64();
-        for (uint32_t seq = g;; seq += 2) {
-            const int a = g, slot = seq % kRingT;
-            twait(&sh.desc_full[slot], (seq / kRingT) & 1, wcyc);
-            const int l = sh.desc_l[slot];
-            if (l < 0) break;
-            const Layer &ly = p.layer[l];
-            const int n = sh.desc_n[slot], y = sh.desc_y0[slot] + ii, x = sh.desc_x0[slot] + jj;
-            int kind = 0;   // 0 skip (garbage column / outside tile or grid), 1 zero (masked), 2 value
-            if (ii < p.Tb && jj < p.Tw && y < Hg && x < Wg) kind = (y < p.H && x < p.W) ? 2 : 1;
-            const long long off = (long long)((n * nb2 + (y >> p.lBh)) * nb3 + (x >> p.lBw)) * be +
-                                  ((((y & mh) << p.lBw) | (x & mw)) << 6) + h * 32;
-            const bool res = kind == 2 && ly.res && !(p.dbg & 16);   // debug 16: residual skipped (timing only)
-            uint4 rr[4];
-            if (res) {   // issued before the accumulator wait: the L2 latency overlaps the MMAs
-                const uint4 *rs = reinterpret_cast<const uint4 *>(resp + off);
-#pragma unroll
-                for (int k = 0; k < 4; k++) rr[k] = __ldcg(rs + k);
-            }
-            twait(&sh.acc_full[a], (seq >> 1) & 1, wcyc);
-            ptx::tc_fence_after();
-            if (ew == 0 && lane == 0) sh.tr[slot][5] = gtime();
-            uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(ly.out.ptr) + off);
-#pragma unroll
-            for (int c = 0; c < 2; c++) {
-                uint32_t d0[16], d1[16], d2[16];
-                const uint32_t taddr = sh.tmem_base + a * kAccCols + ((uint32_t)(q * 32) << 16) + h * 32 + c * 16;
-                ptx::tmem_ld16(taddr, d0);
-                ptx::tmem_ld16(taddr + 64, d1);
-                ptx::tmem_ld16(taddr + 128, d2);
-                ptx::tmem_ld_wait();
-                ptx::reg_fence16(d0);
-                ptx::reg_fence16(d1);
-                ptx::reg_fence16(d2);
-                if (c == 1) {
-                    ptx::tc_fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&sh.acc_empty[a]);
-                    if (ew == 0 && lane == 0) sh.tr[slot][6] = gtime();   // TMEM read out
-                }
-                float (*xw)[3][16] = sh.xch[g][(seq >> 1) & 1][h][c];
-                if (q > 0 && lane < 2) {   // rows 32q, 32q+1 feed output rows 32q-1, 32q-2 of quadrant q-1
-#pragma unroll
-                    for (int e = 0; e < 16; e++) {
-                        if (lane == 0) {
-                            xw[q][0][e] = __uint_as_float(d1[e]);
-                            xw[q][1][e] = __uint_as_float(d2[e]);
-                        } else {
-                            xw[q][2][e] = __uint_as_float(d2[e]);
-                        }
-                    }
-                }
-                {
-                    const unsigned long long tb = clock64();
-                    asm volatile("bar.sync %0, 128;" ::"r"(3 + 2 * g + h) : "memory");
-                    bcyc += clock64() - tb;
-                }
-                float v[16];
-#pragma unroll
-                for (int e = 0; e < 16; e++) {
-                    float s1 = __shfl_down_sync(0xffffffff, __uint_as_float(d1[e]), 1);
-                    float s2 = __shfl_down_sync(0xffffffff, __uint_as_float(d2[e]), 2);
-                    if (fix) {
-                        if (lane == 31) s1 = xw[q + 1][0][e];
-                        s2 = lane == 31 ? xw[q + 1][2][e] : xw[q + 1][1][e];
-                    }
-                    v[e] = __uint_as_float(d0[e]) + s1 + s2;
-                }
-                if (kind && !(p.dbg & 2)) {
-                    uint4 o[2] = {make_uint4(0, 0, 0, 0), make_uint4(0, 0, 0, 0)};
-                    if (kind == 2) {
-                        const float4 *bl = reinterpret_cast<const float4 *>(bias_s + l * C + h * 32 + c * 16);
-#pragma unroll
-                        for (int c4 = 0; c4 < 4; c4++) {
-                            const float4 b = bl[c4];
-                            v[4 * c4] += b.x;
-                            v[4 * c4 + 1] += b.y;
-                            v[4 * c4 + 2] += b.z;
-                            v[4 * c4 + 3] += b.w;
-                        }
-                        if (res) {
-                            const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr[2 * c]);
-#pragma unroll
-                            for (int e = 0; e < 8; e++) {
-                                const float2 f2 = __bfloat1622float2(h2[e]);
-                                v[2 * e] += f2.x;
-                                v[2 * e + 1] += f2.y;
-                            }
-                        }
-                        if (ly.relu) {
-#pragma unroll
-                            for (int e = 0; e < 16; e++) v[e] = fmaxf(v[e], 0.f);
-                        }
-                        o[0] = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
-                        o[1] = make_uint4(pack2(v[8], v[9]), pack2(v[10], v[11]), pack2(v[12], v[13]), pack2(v[14], v[15]));
-                    }
-                    if (!(p.dbg & 64)) {   // debug 64: no output stores (timing only)
-                        dst[2 * c] = o[0];
-                        dst[2 * c + 1] = o[1];
-                    }
-                }
-            }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&sh.stored[slot]);
-        }
-        if (ew == 0 && lane == 0) {
-            prof_out(p, 4, wcyc, t_start);
-            prof_out(p, 6, bcyc, t_start);
-        }
-    }
-    ptx::tc_fence_before();
-    __syncthreads();
-    if (warp == kMma) ptx::tmem_dealloc(sh.tmem_base, 2 * kAccCols);
-}
-}  // namespace ts
 
 }  // namespace ws
 
@@ -1405,67 +873,6 @@ bool ws_geometry(const bdl_plan *p, const Subgraph &sg, WsGeom &g) {
     return best > 0;
 }
 
-// Tap-shared kernel geometry (C = 64 chains): bands of Tb rows x Tw columns with Tb * (Tw + 2) <= 126, so
-// one M = 128 tile per task; input buffers as deep as shared memory allows next to the resident weights.
-// Experimental (BDL_TS=1): the shorter MMA does not pay yet -- per-task epilogue latency (three accumulator
-// blocks per output, shuffles, 1-tile tasks) makes it slower end to end than the N = 64 kernel.
-static bool ts_enabled() {
-    static const int on = [] { const char *e = getenv("BDL_TS"); return e ? atoi(e) : 0; }();
-    return on != 0;
-}
-bool ts_geometry(const bdl_plan *p, const Subgraph &sg, WsGeom &g) {
-    if (!ts_enabled()) return false;
-    const Layer &f = p->layers[sg.first];
-    const int L = sg.last - sg.first + 1;
-    if (f.L.cin != 64 || p->in_layout.nsp != 2 || p->in_layout.brickmap) return false;
-    for (int j = sg.first; j <= sg.last; j++)
-        if (p->layers[j].L.cin != 64 || p->layers[j].L.cout != 64) return false;
-    const int Bh = p->in_layout.Bh, Bw = p->in_layout.Bw;
-    if (ilog2(Bh) < 0 || ilog2(Bw) < 0 || L > kMaxLayers) return false;
-    const int H = f.in_ext[2], W = f.in_ext[3];
-    const int Wfull = (W + Bw - 1) / Bw * Bw;
-    const int limit = 227 * 1024 - (int)sizeof(ws::ts::Shared) - 1024;
-    const int fixed = ws::ts::kWBytes + L * 64 * 4;
-    double best = -1;
-    for (int Tw = Wfull; Tw >= Bw; Tw -= Bw) {
-        WsGeom c;
-        c.Tw = Tw;
-        c.Wt = Tw + 2;
-        if (c.Wt > ws::ts::kRowsT) continue;
-        c.Tb = std::min(H, ws::ts::kRowsT / c.Wt);
-        c.ntl = 1;
-        c.rowsA = (std::max((c.Tb + 2) * c.Wt, 2 * c.Wt + 128) + 7) / 8 * 8;
-        const int inb = c.rowsA * 128;
-        c.nin = std::min(ws::kMaxIn, (limit - fixed) / inb);
-        if (c.nin < 2) continue;
-        c.nacc = 2;
-        c.tmem_cols = 2 * ws::ts::kAccCols;
-        c.smem = c.nin * inb + fixed;
-        const int nty = (H + c.Tb - 1) / c.Tb, ntx = (W + Tw - 1) / Tw;
-        const double score = (double)H * W / ((double)nty * ntx * 128.0) + (c.nin >= 3 ? 0.01 : 0.0);
-        if (score > best) {
-            best = score;
-            g = c;
-        }
-    }
-    return best > 0;
-}
-
-// Per-layer queues of the tap-shared kernel: each layer's tasks band-major over the images (band b of every
-// image before band b+1), so layer l+1's first bands become ready while layer l is still running.
-static std::vector<int> ts_order(const bdl_plan *p, const Subgraph &sg, const WsGeom &g) {
-    const Layer &f = p->layers[sg.first];
-    const int L = sg.last - sg.first + 1;
-    const int N = f.in_ext[0], H = f.in_ext[2], W = f.in_ext[3];
-    const int nty = (H + g.Tb - 1) / g.Tb, ntx = (W + g.Tw - 1) / g.Tw;
-    std::vector<int> ord;
-    for (int l = 0; l < L; l++)
-        for (int b = 0; b < nty; b++)
-            for (int n = 0; n < N; n++)
-                for (int tx = 0; tx < ntx; tx++) ord.push_back((int)(((long long)n * nty + b) * ntx + tx));
-    return ord;
-}
-
 // Locality-aware wavefront order (host): step s, image n, layer l -> tile row b = s - lag*l.
 std::vector<int> ws_order(const bdl_plan *p, const Subgraph &sg, const WsGeom &g, int lag) {
     const Layer &f = p->layers[sg.first];
@@ -1515,47 +922,6 @@ static bdl_status launch_ws_C(bdl_plan *p, Subgraph &sg, ws::Params &P, const Ws
 bdl_status launch_tc_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out, const TView *res,
                               unsigned char *ws, cudaStream_t s, int *launches);
 
-static bdl_status launch_ts(bdl_plan *p, Subgraph &sg, ws::Params &P, bool unmerged, cudaStream_t s, int *launches) {
-    WsGeom g;
-    ts_geometry(p, sg, g);
-    auto k = ws::ts::memo_ts_kernel;
-    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
-    const long long nper = (long long)P.nty * P.ntx * p->layers[sg.first].in_ext[0];
-    P.ts_nper = nper;
-    // tickets per draw: enough to keep same-address atomics off the critical path, small enough that the
-    // dynamic balance at the end of a queue stays fine (>= ~8 draws per CTA)
-    const int gl = std::max(1, std::min<int>(p->num_sms, (int)nper) / (unmerged ? 1 : P.L));
-    P.ts_batch = (int)std::max<long long>(1, std::min<long long>(4, nper / ((long long)gl * 8)));
-    if (const char *e = getenv("BDL_TS_BATCH")) P.ts_batch = std::max(1, atoi(e));
-    const long long B = P.ts_batch, draws_ok = (nper + B - 1) / B;
-    if (sg.ts_tbase.size() < (size_t)kMaxLayers) sg.ts_tbase.assign(kMaxLayers, 0);
-    if (!unmerged) {
-        const int grid = (int)std::min<long long>(nper * P.L, (long long)p->num_sms);
-        P.only_layer = -1;
-        for (int l = 0; l < P.L; l++) {
-            P.ts_tbase[l] = sg.ts_tbase[l];
-            // draws on queue l: ceil(nper / B) successful + one failing draw per CTA that starts on a layer <= l
-            long long drawers = 0;
-            for (int c = 0; c < grid; c++) drawers += (c % P.L) <= l;
-            sg.ts_tbase[l] += (unsigned long long)(B * (draws_ok + drawers));
-        }
-        launch_pdl(k, dim3(grid), dim3(ws::ts::kThreads), g.smem, s, P);
-        *launches += 1;
-    } else {
-        P.order = nullptr;
-        const int grid = (int)std::min<long long>(nper, (long long)p->num_sms);
-        for (int l = 0; l < P.L; l++) {
-            P.only_layer = l;
-            P.ts_tbase[l] = sg.ts_tbase[l];
-            sg.ts_tbase[l] += (unsigned long long)(B * (draws_ok + grid));
-            launch_pdl(k, dim3(grid), dim3(ws::ts::kThreads), g.smem, s, P);
-            *launches += 1;
-        }
-    }
-    BDL_CUDA_CHECK_LAUNCH("tcgen05 tap-shared memo kernel");
-    return BDL_OK;
-}
-
 // TMA descriptor of a bricked bf16 tensor viewed as 2-D [pixels][Cp]: box = 64 channels x box_px pixels,
 // 128-B swizzle (matches the UMMA SWIZZLE_128B A-operand layout).
 static bool encode_pixel_map(CUtensorMap *tm, const TView &v, int box_px) {
@@ -1597,13 +963,10 @@ static bool encode_row_map(CUtensorMap *tm, const TView &v, int nseg) {
     return r == CUDA_SUCCESS;
 }
 
-bool ts_geometry(const bdl_plan *p, const Subgraph &sg, WsGeom &g);
-
 bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out, const TView *res,
                               unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged) {
     WsGeom g;
-    const bool ts = ts_geometry(p, sg, g) && !in.bmap && !out.bmap && !(res && res->bmap);
-    if (!ts && !ws_geometry(p, sg, g))  // wide channel counts: the synchronous band kernel
+    if (!ws_geometry(p, sg, g))  // wide channel counts: the synchronous band kernel
         return launch_tc_subgraph(p, sg, in, out, res, wsp, s, launches);
     ws::Params P;
     memset(&P, 0, sizeof(P));
@@ -1686,7 +1049,6 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
             ws_trace_cap = cap;
         }
     }
-    if (ts) return launch_ts(p, sg, P, unmerged, s, launches);
     switch (P.C) {
         case 16: return launch_ws_C<16>(p, sg, P, g, unmerged, s, launches);
         case 32: return launch_ws_C<32>(p, sg, P, g, unmerged, s, launches);
@@ -1701,15 +1063,6 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
 namespace bdl {
 std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg) {
     WsGeom g;
-    if (ts_geometry(p, sg, g)) {
-        std::vector<int> ord = ts_order(p, sg, g);
-        if (p->opts.schedule_seed) {   // any order within a layer's queue is valid (dependencies are waited for)
-            const size_t per = ord.size() / (size_t)(sg.last - sg.first + 1);
-            std::mt19937 rng((unsigned)p->opts.schedule_seed);
-            for (size_t o = 0; o < ord.size(); o += per) std::shuffle(ord.begin() + o, ord.begin() + o + per, rng);
-        }
-        return ord;
-    }
     if (!ws_geometry(p, sg, g)) return {};
     // lag: how many band rows layer l trails layer l-1.  Larger = fewer dependency waits but a larger
     // live intermediate; take the largest lag whose live intermediate (lag band rows of every image of
@@ -1743,7 +1096,6 @@ namespace bdl {
 // Band height of the warp-specialized kernel for subgraph sg (0 if it cannot run it).
 int ws_band_rows(const bdl_plan *p, const Subgraph &sg) {
     WsGeom g;
-    if (ts_geometry(p, sg, g)) return g.Tb;
     return ws_geometry(p, sg, g) ? g.Tb : 0;
 }
 }  // namespace bdl

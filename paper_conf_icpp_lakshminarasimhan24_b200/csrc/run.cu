@@ -63,7 +63,6 @@ bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream) {
         cudaMemsetAsync(ws + sg.status_off, 0, sg.ntasks_total * 4, s);
         cudaMemsetAsync(ws + sg.counter_off, 0, 128, s);
         sg.ticket_base = 0;
-        sg.ts_tbase.assign(kMaxLayers, 0);
         sg.epoch = 0;
     }
     cudaError_t e = cudaGetLastError();
