@@ -41,6 +41,10 @@ GRAPHS = {
     "sw128_3d_c64": ([W.conv(64, 64, 3, nsp=3), W.conv(64, 64, 3, nsp=3)], 1, 64, 10, 12, 9, (1, 4, 4, 4)),
     "sw128_3d_c64_valid": ([W.conv(64, 64, 3, 1, 0, nsp=3), W.conv(64, 64, 3, 1, 0, nsp=3)], 1, 64, 13, 12, 14,
                            (1, 4, 4, 4)),
+    # 32-channel layers on the 64-B swizzled layout: valid padding (no stage offset) and a 1x1 layer, ragged extents
+    "sw64_3d_valid_1x1": ([W.conv(32, 32, 3, 1, 0, nsp=3), W.conv(32, 32, 1, nsp=3)], 1, 32, 11, 13, 14,
+                          (1, 4, 4, 4)),
+    "sw64_2d_chain": ([W.conv(32, 64, 3), W.conv(64, 32, 1)], 2, 32, 1, 19, 21, (1, 1, 8, 8)),
 }
 
 
