@@ -95,7 +95,9 @@ typedef struct bdl_layer {
 
 /* Static-analysis knobs (§3.3); bdl_plan_opts_default gives the paper's values. */
 typedef struct bdl_plan_opts {
-    double delta_threshold;      /* 0.15: memoized when padding data growth Delta > 15% (L644) */
+    double delta_threshold;      /* 0.15: memoized when padding data growth Delta > 15% (L644).  On B200 our
+                                    memoized kernels measured faster than padded on every subgraph tried
+                                    (DESIGN.md §7); a negative value selects memoized everywhere. */
     int64_t tau;                 /* 4096: rho threshold, "tau = 2^12" (L656, printed "212") */
     int32_t bcand[4];            /* {4, 8, 16, 32} brick edge candidates (L654) */
     int64_t onchip_budget;       /* bytes a merged subgraph's footprint may use; 0 = device L2 size (L611-614) */
@@ -145,7 +147,8 @@ int32_t bdl_plan_num_subgraphs(const bdl_plan *p);
 
 /* Subgraph i: layers [first, last], mode (bdl_mode, never AUTO), brick edge chosen by the model
  * (rho/tau; the executed brick is the layout's), Delta (padding data growth, SURVEY Q6 reading),
- * and the executing kernel (0 = CUDA-core brick kernel, 1 = tcgen05 band kernel). */
+ * and the executing kernel (0 = CUDA-core brick kernel, 1 = tcgen05 band kernel for C = 64/128 3x3
+ * chains, 2 = generic tcgen05 kernel for every other bf16 shape). */
 bdl_status bdl_plan_subgraph(const bdl_plan *p, int32_t i, int32_t *first, int32_t *last,
                              int32_t *mode, int32_t *model_brick, double *delta, int32_t *kernel);
 
@@ -189,7 +192,7 @@ void bdl_plan_destroy(bdl_plan *p);
 
 /* Subgraph i's model details: Delta under the first-layer-only reading (SURVEY Q6 alternative),
  * rho of the model's brick (L653), the mode the Delta rule chose before any override, and the
- * tcgen05 band height (0 = CUDA-core brick kernel). */
+ * tcgen05 band height (0 = not the band kernel). */
 bdl_status bdl_plan_subgraph_model(const bdl_plan *p, int32_t i, double *delta_first, int64_t *rho,
                                    int32_t *mode_model, int32_t *tc_band);
 
