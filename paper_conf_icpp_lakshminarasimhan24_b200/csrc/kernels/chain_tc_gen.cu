@@ -62,6 +62,8 @@ struct LayerP {
     int lkc;                  // log2(kc)
     int tma;                  // 1: the in-image columns of each input row arrive by one TMA box (tm_row)
     int pxo;                  // SW64: pixel-row offset of the stage (0/1) that makes every TMA row start 128-B aligned
+    int xal;                  // padded mode, first layer: tiles start at the region's x rounded down to a brick
+                              // boundary, so their in-tile columns are whole brick-row segments (TMA boxes)
     int lB[3];                // log2 of the source view's brick extents (d, h, w)
     int rb, nblk, blk_px, plane_px;
     int in_rows, in_cols;
@@ -218,8 +220,12 @@ __host__ __device__ inline void region_of(const LayerP *ly, int L, const int PB[
         }
     }
 }
+// first tile column of a padded-mode region (aligned down to a brick edge for xal layers)
+__host__ __device__ inline int region_x0(const LayerP &L, int lo2) {
+    return L.xal ? (lo2 >> L.lB[2]) << L.lB[2] : lo2;
+}
 __host__ __device__ inline int region_subtiles(const LayerP &L, const int lo[3], const int hi[3]) {
-    const int a = hi[0] - lo[0], b = hi[1] - lo[1], c = hi[2] - lo[2];
+    const int a = hi[0] - lo[0], b = hi[1] - lo[1], c = hi[2] - region_x0(L, lo[2]);
     if (a <= 0 || b <= 0 || c <= 0) return 0;
     return a * ((b + L.Tb - 1) / L.Tb) * ((c + L.Tw - 1) / L.Tw) * L.nnc;
 }
@@ -257,11 +263,12 @@ __device__ __forceinline__ Tile make_tile(const Params &p, int l, long long t) {
     T.n = (int)(P / p.npb[0]);
     int lo[3], hi[3];
     region_of(p.layer, p.L, p.PB, blk, l, lo, hi);
-    const int nty = (hi[1] - lo[1] + L.Tb - 1) / L.Tb, ntx = (hi[2] - lo[2] + L.Tw - 1) / L.Tw;
+    const int xs = region_x0(L, lo[2]);
+    const int nty = (hi[1] - lo[1] + L.Tb - 1) / L.Tb, ntx = (hi[2] - xs + L.Tw - 1) / L.Tw;
     const int kx = k % ntx; k /= ntx;
     const int ky = k % nty;
     const int kd = k / nty;
-    T.d = lo[0] + kd; T.y0 = lo[1] + ky * L.Tb; T.x0 = lo[2] + kx * L.Tw;
+    T.d = lo[0] + kd; T.y0 = lo[1] + ky * L.Tb; T.x0 = xs + kx * L.Tw;
     for (int d = 0; d < 3; d++) { T.hi[d] = hi[d]; T.dlo[d] = lo[d]; }
     T.dst_scr = l < p.L - 1;
     T.src_scr = l > 0;
@@ -846,7 +853,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 const int i = m / L.Wp, j = m - i * L.Wp;
                 const int y = T.y0 + i, x = T.x0 + j;
                 int kind = 0;   // 0 skip, 1 zero (masked), 2 value
-                if (i < L.Tb && j < L.Tw && d < T.hi[0] && y < T.hi[1] && x < T.hi[2])
+                if (i < L.Tb && j < L.Tw && d < T.hi[0] && y < T.hi[1] && x < T.hi[2] && (!p.padded || x >= T.dlo[2]))
                     kind = (d < L.out_ext[0] && y < L.out_ext[1] && x < L.out_ext[2]) ? 2 : 1;
                 const int ch0 = T.nc * L.Nc + cb * CB;
                 uint32_t r[2][16];
@@ -998,6 +1005,9 @@ static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out,
     // the loader's address arithmetic uses shifts: power-of-two chunk counts and brick extents
     auto lg = [](int v) { int r = 0; while ((1 << r) < v) r++; return (1 << r) == v ? r : -1; };
     G.lkc = lg(G.kc);
+    G.xal = 0;
+    G.tma = 0;
+    G.pxo = 0;
     G.lB[0] = lg(lo_out.Bd);
     G.lB[1] = lg(lo_out.Bh);
     G.lB[2] = lg(lo_out.Bw);
@@ -1067,6 +1077,13 @@ static bool gen_tma_ok() {
     static const int v = [] { const char *e = getenv("BDL_GEN_TMA"); return e ? atoi(e) : 1; }();
     return v != 0;
 }
+// Padded-mode first layer eligible for TMA rows (stride 1, swizzled A layout, 2-D or SW64 3-D)?
+static bool gen_pad_tma_ok(const gen::LayerP &G, int nsp, int Bw) {
+    if (!gen_tma_ok() || G.s[0] != 1 || G.s[1] != 1 || G.s[2] != 1 || Bw > 256) return false;
+    if (G.amode == gen::AM_SW128) return G.k[0] == 1 && nsp == 2;
+    return G.amode == gen::AM_SW64;
+}
+
 // 5-D view of a 2-D bricked bf16 tensor (identity BrickMap): (channel, x in brick, brick column, y in brick,
 // brick row over (n, by)); box = 64 channels x Bw x nseg bricks x 1 x 1, 128-B swizzled (the SW128 A layout).
 static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int xstride = 1, int box_ch = 64) {
@@ -1156,7 +1173,11 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
                 }
                 G.pR[d] = std::max(1, mx);
             }
-            if (!gen_layer_tiles(G, G.pR[1], G.pR[2], 1)) return false;
+            // first layer (reads the bricked subgraph input): brick-aligned tiles so its rows arrive by TMA
+            const int Bw = p->in_layout.Bw;
+            const bool xal = j == 0 && gen_pad_tma_ok(G, nsp, Bw);
+            G.xal = xal ? 1 : 0;
+            if (!gen_layer_tiles(G, G.pR[1], xal ? G.pR[2] + Bw - 1 : G.pR[2], xal ? Bw : 1)) return false;
             if (j < nconv - 1) {
                 G.scr_off = g.scr_slot;
                 g.scr_slot += ((long long)G.pR[0] * G.pR[1] * G.pR[2] * G.cout * 2 + 255) / 256 * 256;
@@ -1314,11 +1335,12 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
         G.out = outs[j];
         G.tma = 0;
         G.pxo = 0;
-        if (!padded && G.amode == gen::AM_SW128 && G.s[1] == 1 && G.s[2] == 1 && G.k[0] == 1 && nsp == 2 &&
+        // (padded mode: only the first layer, whose tiles are brick-aligned (xal); later layers read CTA scratch)
+        if ((!padded || G.xal) && G.amode == gen::AM_SW128 && G.s[1] == 1 && G.s[2] == 1 && G.k[0] == 1 && nsp == 2 &&
             !G.src.bmap && G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
             gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw))
             G.tma = 1;
-        else if (!padded && G.amode == gen::AM_SW64 && G.s[0] == 1 && G.s[1] == 1 && G.s[2] == 1 && !G.src.bmap &&
+        else if ((!padded || G.xal) && G.amode == gen::AM_SW64 && G.s[0] == 1 && G.s[1] == 1 && G.s[2] == 1 && !G.src.bmap &&
                  G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 && G.src.Cp == 32 &&
                  G.Wp % 2 == 0 && G.plane_px % 2 == 0 && p->in_layout.Bd * p->in_layout.Bh <= 256 && gen_tma_ok() &&
                  gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw, 1, 32)) {
