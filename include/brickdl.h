@@ -166,7 +166,14 @@ int64_t bdl_plan_workspace_bytes(const bdl_plan *p);
  * >= bdl_plan_workspace_bytes, 256-byte aligned, caller-owned, reused by every bdl_run. */
 bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream);
 
-/* Run subgraph i (its input/residual tensors must already hold data: for i = 0 `in_bricked`,
+/* Streams and replays: a plan's workspace (memo tables, run state) serves one stream at a time -- do not
+ * run the same plan/workspace on two streams concurrently.  The per-run state (ticket counter, memo-tag
+ * epoch) lives in the workspace and is advanced by the kernels themselves (the last CTA of a launch
+ * rewinds the ticket and bumps the epoch), so bdl_run / bdl_run_subgraph launches may be captured in a
+ * CUDA graph and replayed.  A launch that fails mid-run leaves that state undefined: call
+ * bdl_plan_prepare again.
+ *
+ * Run subgraph i (its input/residual tensors must already hold data: for i = 0 `in_bricked`,
  * otherwise earlier subgraphs' outputs in the workspace).  in_bricked / out_bricked: DEVICE,
  * bricked per the plan's input / output layouts. */
 bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void *out_bricked,

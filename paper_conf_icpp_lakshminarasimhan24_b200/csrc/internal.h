@@ -62,21 +62,25 @@ struct Subgraph {
     int kernel;                 // KernelKind the subgraph is able to run on
     int gen_layers = 0;         // generic tcgen05 kernel: leading conv layers it runs (a pool tail follows)
     int64_t gen_scr_off = -1;   // generic tcgen05 kernel, padded mode: per-CTA region scratch
-    int in_tensor;              // index into Plan::tensors
+    int in_tensor;              // index into Plan::tensors (the first layer's input)
     int out_tensor;
+    bool chain = true;          // every layer reads the previous one (padded mode and the band / CUDA-core
+                                // kernels need this; DAG subgraphs run memoized or unmerged on the generic kernel)
+    std::vector<int> src_local;    // per layer: index (within the subgraph) of the layer it reads, or -1 = external
+    std::vector<int> src_tensor;   // per layer: tensor index of an external input, or -1
+    std::vector<int> res_local;    // per layer: index (within the subgraph) of the residual's producer, or -1
     std::vector<int> res_tensor;   // per layer in subgraph: tensor index of external residual, or -1
     // memoized mode
-    std::vector<int64_t> memo_off; // per layer (except last): bricked intermediate buffer offsets
+    std::vector<int64_t> memo_off; // per layer (except last): bricked intermediate buffer offsets (a live-out
+                                   // layer's buffer is the tensor later subgraphs read)
     int64_t status_off = -1;       // int32 [L][tasks]
     std::vector<int64_t> task_base;// per layer offset into the status table (in words)
     int64_t ntasks_total = 0;
-    int64_t counter_off = -1;      // uint64 [4] + ticket counter
+    int64_t counter_off = -1;      // uint64 run-state block (kernels/common.cuh: counters, ticket, epoch)
     // padded mode scratch (CUDA-core kernel)
     int64_t scratch_off = -1;
     int64_t scratch_slot_floats = 0;
     int grid = 0;                  // persistent grid size
-    uint64_t ticket_base = 0;      // memo ticket counter offset for the next run
-    unsigned epoch = 0;            // memo tag epoch (bumped every run; tags of older epochs read as state 0)
     // tcgen05 band kernel parameters
     int tc_band = 0;               // band rows
     int tc_smem = 0;
@@ -85,7 +89,6 @@ struct Subgraph {
     int64_t order_off = -1;
     int64_t norder = 0;
     std::vector<int> order_host;
-    // tap-shared tcgen05 kernel: per-layer ticket counter bases (advanced deterministically every run)
 };
 
 }  // namespace bdl
@@ -97,7 +100,6 @@ struct bdl_plan {
     bdl_layout in_layout, out_layout;
     bdl_plan_opts opts;
     int64_t ws_bytes = 0;
-    uint32_t epoch = 0;
     int num_sms = 148;
     int64_t l2_bytes = 0;
     bool prepared = false;

@@ -31,9 +31,7 @@ struct GChain {
     long long slot_floats;
     int *status;
     long long task_base[kMaxLayers];
-    unsigned epoch;
-    unsigned long long *counters;   // [0] computed [1] cas_ok [2] cas_fail [3] spins [4] ticket
-    unsigned long long ticket_base;
+    unsigned long long *counters;   // run state (common.cuh run_epoch / run_exit)
     long long ntop;                 // bricks of the last layer's output
 };
 
@@ -242,10 +240,10 @@ __global__ void __launch_bounds__(256) memo_chain_kernel(GChain g) {
     __shared__ long long s_task;
     __shared__ int s_cmd_l;
     __shared__ long long s_cmd_b;
-    const unsigned EP = g.epoch << 2;
+    const unsigned EP = run_epoch(g.counters) << 2;
     for (;;) {
         if (threadIdx.x == 0) {
-            unsigned long long tk = atomicAdd(&g.counters[4], 1ULL) - g.ticket_base;
+            unsigned long long tk = atomicAdd(&g.counters[4], 1ULL);
             s_task = (long long)tk;
             if ((long long)tk < g.ntop) {
                 // top-level brick: claim it (always succeeds: only tickets reach last-layer bricks)
@@ -317,6 +315,7 @@ __global__ void __launch_bounds__(256) memo_chain_kernel(GChain g) {
             if (s_sp == 0) break;
         }
     }
+    if (threadIdx.x == 0) run_exit(g.counters);
 }
 
 // ---------------------------------------------------------------------------------------------- unmerged
@@ -488,7 +487,6 @@ bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &i
     g.slot_floats = sg.scratch_slot_floats;
     g.status = (int *)(ws + sg.status_off);
     for (int j = 0; j < g.L; j++) g.task_base[j] = sg.task_base[j];
-    g.epoch = sg.epoch;
     g.counters = (unsigned long long *)(ws + sg.counter_off);
     int grid = (int)std::min<long long>(g.ntop, sg.grid);
     int mode = sg.mode;
@@ -498,8 +496,6 @@ bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &i
         else padded_chain_kernel<float><<<grid, 256, 0, s>>>(g);
         *launches += 1;
     } else if (mode == BDL_MODE_MEMOIZED) {
-        g.ticket_base = const_cast<Subgraph &>(sg).ticket_base;
-        const_cast<Subgraph &>(sg).ticket_base += (unsigned long long)g.ntop + grid;
         if (g.bf16) memo_chain_kernel<__nv_bfloat16><<<grid, 256, 0, s>>>(g);
         else memo_chain_kernel<float><<<grid, 256, 0, s>>>(g);
         *launches += 1;

@@ -55,9 +55,7 @@ struct TcParams {
     TView in, res;
     int *status;
     long long task_base[kMaxLayers];
-    unsigned epoch;
-    unsigned long long *counters;  // [0] computed [1] cas_ok [2] cas_fail [3] spins [4] ticket
-    unsigned long long ticket_base;
+    unsigned long long *counters;  // [0] tiles computed (common.cuh counter block)
     long long ntiles;              // tiles per layer = N * nty * ntx
     int only_layer;                // >= 0: unmerged launch of that layer
     unsigned long long *trace;     // debug: per task [smid|l, tile, t0..t4] (globaltimer ns), or null
@@ -319,135 +317,6 @@ __global__ void __launch_bounds__(kTcThreads, 1) tc_padded_kernel(const __grid_c
     teardown<C>(sh, p.tmem_cols);
 }
 
-// ------------------------------------------------------------------------------------------------ memoized
-struct TcFrame {
-    int l, phase, k;
-    long long t;
-};
-
-__device__ __forceinline__ int *tc_status(const TcParams &p, int l, long long t) { return p.status + p.task_base[l] + t; }
-
-template <int C>
-__global__ void __launch_bounds__(kTcThreads, 1) tc_memo_kernel(const __grid_constant__ TcParams p) {
-    extern __shared__ __align__(1024) uint8_t smem[];
-    __shared__ TcShared sh;
-    __shared__ TcFrame stk[kMaxLayers + 1];
-    constexpr int KC = C / 8;
-    uint8_t *bufA = smem;
-    uint8_t *wst = bufA + (size_t)KC * p.rowsA * 16;
-    setup<C>(sh, smem, KC * p.rowsA * 16, p.tmem_cols);
-    uint32_t wq = 0, done_phase = 0;
-    const unsigned EP = p.epoch << 2;
-    const bool unmerged = p.only_layer >= 0;
-    const int top = unmerged ? p.only_layer : p.L - 1;
-    const int Mrows = p.Tb * p.Wt;
-    const int ntl = (Mrows + 127) / 128;
-    for (;;) {
-        if (threadIdx.x == 0) {
-            unsigned long long tk = atomicAdd(&p.counters[4], 1ULL) - p.ticket_base;
-            sh.task = (long long)tk;
-            if ((long long)tk < p.ntiles) {
-                if (!unmerged) {
-                    int *sw = tc_status(p, top, (long long)tk);
-                    int cur = ld_acquire(sw);
-                    atomicCAS(sw, cur, (int)(EP | 1));
-                    atomicAdd(&p.counters[1], 1ULL);
-                }
-                stk[0] = TcFrame{top, unmerged ? 1 : 0, unmerged ? 9 : 0, (long long)tk};
-                sh.sp = 1;
-            }
-        }
-        __syncthreads();
-        if (sh.task >= p.ntiles) break;
-        for (;;) {
-            unsigned long long t0 = gtime();
-            if (threadIdx.x == 0) {
-                sh.cmd_l = -1;
-                unsigned long long spins = 0, fails = 0, oks = 0;
-                while (sh.cmd_l < 0) {
-                    TcFrame &f = stk[sh.sp - 1];
-                    if (f.l == 0 || unmerged) { sh.cmd_l = f.l; sh.cmd_t = f.t; break; }
-                    if (f.k >= 9) {
-                        if (f.phase == 0) { f.phase = 1; f.k = 0; continue; }
-                        sh.cmd_l = f.l; sh.cmd_t = f.t;
-                        break;
-                    }
-                    int n, ty, tx;
-                    decode_tile(p, f.t, n, ty, tx);
-                    int dy = f.k / 3 - 1, dx = f.k % 3 - 1;
-                    int qy = ty + dy, qx = tx + dx;
-                    if (qy < 0 || qy >= p.nty || qx < 0 || qx >= p.ntx) { f.k++; continue; }
-                    long long dt = ((long long)n * p.nty + qy) * p.ntx + qx;
-                    int *sw = tc_status(p, f.l - 1, dt);
-                    int cur = ld_acquire(sw);
-                    int st = ((cur & ~3) == (int)EP) ? (cur & 3) : 0;
-                    if (f.phase == 0) {
-                        f.k++;
-                        if (st == 2) continue;
-                        if (st == 0 && atomicCAS(sw, cur, (int)(EP | 1)) == cur) {
-                            oks++;
-                            stk[sh.sp] = TcFrame{f.l - 1, 0, 0, dt};
-                            sh.sp++;
-                            continue;
-                        }
-                        fails++;
-                    } else {
-                        if (st == 2) { f.k++; continue; }
-                        spins++;
-                        __nanosleep(100);
-                    }
-                }
-                if (oks) atomicAdd(&p.counters[1], oks);
-                if (fails) atomicAdd(&p.counters[2], fails);
-                if (spins) atomicAdd(&p.counters[3], spins);
-                __threadfence();
-            }
-            __syncthreads();
-            const int l = sh.cmd_l;
-            const long long tt = sh.cmd_t;
-            int n, ty, tx;
-            decode_tile(p, tt, n, ty, tx);
-            const int y0 = ty * p.Tb, x0 = tx * p.Tw;
-            const TView &src = l == 0 ? p.in : p.layer[l - 1].out;
-            unsigned long long t1 = gtime();
-            load_tile<C>(src, n, y0 - 1, x0 - 1, p.Tb + 2, p.Wt, bufA, p.rowsA);
-            ptx::tc_fence_before();
-            __syncthreads();
-            ptx::tc_fence_after();
-            unsigned long long t2 = gtime();
-            if (threadIdx.x == 0) issue_layer<C>(p, sh, p.layer[l].w, bufA, p.rowsA, ntl, wst, wq);
-            ptx::mbar_wait(&sh.mma_done, done_phase);
-            done_phase ^= 1;
-            ptx::tc_fence_after();
-            unsigned long long t3 = gtime();
-            epilogue_global<C>(p, sh, p.layer[l], ntl, n, y0, x0, p.layer[l].res);
-            ptx::tc_fence_before();
-            __syncthreads();
-            if (threadIdx.x == 0 && p.trace) {
-                unsigned long long t4 = gtime();
-                unsigned long long k = atomicAdd(&p.counters[5], 1ULL);
-                if (k < (unsigned long long)p.trace_cap) {
-                    unsigned long long *r = p.trace + k * 7;
-                    r[0] = ((unsigned long long)smid() << 32) | ((unsigned)blockIdx.x << 8) | (unsigned)l;
-                    r[1] = (unsigned long long)tt;
-                    r[2] = t0; r[3] = t1; r[4] = t2; r[5] = t3; r[6] = t4;
-                }
-            }
-            if (threadIdx.x == 0) {
-                if (!unmerged) {
-                    __threadfence();
-                    st_release(tc_status(p, l, tt), (int)(EP | 2));
-                }
-                atomicAdd(&p.counters[0], 1ULL);
-                sh.sp--;
-            }
-            __syncthreads();
-            if (sh.sp == 0) break;
-        }
-    }
-    teardown<C>(sh, p.tmem_cols);
-}
-
 // weights [cout][3][3][cin] (bf16) -> [tap][cin/8][cout][8]
 __global__ void pack_tc_kernel(const __nv_bfloat16 *__restrict__ w, __nv_bfloat16 *__restrict__ out, int C, int taps) {
     long long total = (long long)C * taps * C;
@@ -541,24 +410,7 @@ static bdl_status launch_tc_C(bdl_plan *p, Subgraph &sg, TcParams &P, const TcGe
         k<<<grid, kTcThreads, g.smem, s>>>(P);
         *launches += 1;
     } else {
-        auto k = tc_memo_kernel<C>;
-        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
-        int grid = (int)std::min<long long>(P.ntiles, (long long)p->num_sms * ctas_per_sm);
-        if (mode == BDL_MODE_MEMOIZED) {
-            P.only_layer = -1;
-            P.ticket_base = sg.ticket_base;
-            sg.ticket_base += (unsigned long long)P.ntiles + grid;
-            k<<<grid, kTcThreads, g.smem, s>>>(P);
-            *launches += 1;
-        } else {
-            for (int l = 0; l < P.L; l++) {
-                P.only_layer = l;
-                P.ticket_base = sg.ticket_base;
-                sg.ticket_base += (unsigned long long)P.ntiles + grid;
-                k<<<grid, kTcThreads, g.smem, s>>>(P);
-                *launches += 1;
-            }
-        }
+        return fail(BDL_EUNSUPPORTED, "tc band kernel: memoized / unmerged modes run on the warp-specialized kernel");
     }
     BDL_CUDA_CHECK_LAUNCH("tc chain kernel");
     return BDL_OK;
@@ -608,7 +460,6 @@ bdl_status launch_tc_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
         P.task_base[j] = sg.task_base[j];
     }
     P.status = (int *)(ws + sg.status_off);
-    P.epoch = sg.epoch;
     P.counters = (unsigned long long *)(ws + sg.counter_off);
     P.ntiles = (long long)P.N * P.nty * P.ntx;
     {

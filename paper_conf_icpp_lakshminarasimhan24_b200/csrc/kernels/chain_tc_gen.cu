@@ -24,6 +24,7 @@
 //                then release-publish the tile (state 2)
 #include <algorithm>
 #include <cstdio>
+#include <random>
 #include <cstdlib>
 #include <cstring>
 #include <string>
@@ -44,12 +45,14 @@ constexpr int kThreads = 32 * (kEpi0 + kEpiW);
 constexpr int kLoadT = 32 * kLW;
 constexpr int kQ = 4, kRing = 16, kStack = 128;
 constexpr int kMaxIn = 4, kMaxW = 4, kMaxKs = 128;   // k-steps per layer: 3x3x3 taps x 64 channels = 108
+constexpr int kTaskBits = 26;   // order entry = (layer << kTaskBits) | task
 
 enum { AM_SW128 = 0, AM_PLANES = 1, AM_PAIR = 2, AM_SW64 = 3 };   // AM_SW64: cin = 32, 64-B swizzled pixel rows
 
 struct LayerP {
     TView src, out, res;
     const __nv_bfloat16 *w;   // packed [nc][kb][ks][2][Nc][8]
+    int srcl, resl;           // producer (index in the subgraph) of the input / of the residual, -1 = external
     const float *bias;        // [cout]
     int relu, has_res;
     int cin, cout;
@@ -82,9 +85,7 @@ struct Params {
     int nin, nw, in_stride, w_stride;    // ring depths and slot strides (bytes)
     int nacc, acc_stride, tmem_cols;
     int *status;
-    unsigned epoch;
-    unsigned long long *counters;        // [0] computed [1] cas_ok [2] cas_fail [3] spins [4] ticket
-    unsigned long long ticket_base;
+    unsigned long long *counters;        // run state (common.cuh run_epoch / run_exit)
     const int *order;                    // (l << 26) | task, or null (unmerged)
     long long norder;
     int only_layer;
@@ -135,7 +136,7 @@ __device__ __forceinline__ int *status_word(const Params &p, int l, long long t)
 }
 
 struct TaskC { int n, d, ty, tx, nc; };
-__device__ __forceinline__ TaskC decode(const LayerP &L, long long t) {
+__host__ __device__ __forceinline__ TaskC decode(const LayerP &L, long long t) {
     TaskC c;
     c.nc = (int)(t % L.nnc); t /= L.nnc;
     c.tx = (int)(t % L.ntx); t /= L.ntx;
@@ -164,13 +165,14 @@ __device__ __forceinline__ long long pix(const TView &v, int n, int d, int y, in
     return phys * v.brick_elems + (long long)in * v.Cp;
 }
 
-// Dependencies of task t of layer l (l >= 1): the layer l-1 tiles covering its input window.
-struct DepRange { int n, d0, nd, b0, nb, x0, nx, nnc; };
-__device__ __forceinline__ DepRange dep_range(const Params &p, int l, long long t) {
-    const LayerP &C = p.layer[l], &P = p.layer[l - 1];
+// Dependencies of task t of layer C: the tiles of its input producer P covering its input window (every channel
+// chunk of P), and the tiles of its residual producer R covering its output tile (the same channel chunk).
+struct DepRange { int n, d0, nd, b0, nb, x0, nx, c0, nnc; };
+__host__ __device__ __forceinline__ DepRange dep_range_src(const LayerP &C, const LayerP &P, long long t) {
     const TaskC c = decode(C, t);
     DepRange r;
     r.n = c.n;
+    r.c0 = 0;
     r.nnc = P.nnc;
     int lo, hi;
     lo = max(0, c.d * C.s[0] - C.pd[0]);
@@ -187,14 +189,60 @@ __device__ __forceinline__ DepRange dep_range(const Params &p, int l, long long 
     r.nx = hi >= lo ? hi / P.Tw - r.x0 + 1 : 0;
     return r;
 }
-__device__ __forceinline__ int dep_count(const DepRange &r) { return r.nd * r.nb * r.nx * r.nnc; }
-__device__ __forceinline__ long long dep_task(const Params &p, int l, const DepRange &r, int i) {
-    const LayerP &P = p.layer[l - 1];
-    const int c = i % r.nnc; i /= r.nnc;
+__host__ __device__ __forceinline__ DepRange dep_range_res(const LayerP &C, const LayerP &R, long long t) {
+    const TaskC c = decode(C, t);
+    DepRange r;
+    r.n = c.n;
+    r.c0 = c.nc;     // same cout, same Nc: the same channel chunk
+    r.nnc = 1;
+    r.d0 = c.d;
+    r.nd = c.d < C.out_ext[0] ? 1 : 0;
+    int lo = c.ty * C.Tb, hi = min(C.out_ext[1], lo + C.Tb) - 1;
+    r.b0 = lo / R.Tb;
+    r.nb = hi >= lo ? hi / R.Tb - r.b0 + 1 : 0;
+    lo = c.tx * C.Tw;
+    hi = min(C.out_ext[2], lo + C.Tw) - 1;
+    r.x0 = lo / R.Tw;
+    r.nx = hi >= lo ? hi / R.Tw - r.x0 + 1 : 0;
+    return r;
+}
+__host__ __device__ __forceinline__ int dep_count(const DepRange &r) { return r.nd * r.nb * r.nx * r.nnc; }
+__host__ __device__ __forceinline__ long long dep_task(const LayerP &P, const DepRange &r, int i) {
+    const int c = r.c0 + i % r.nnc; i /= r.nnc;
     const int x = r.x0 + i % r.nx; i /= r.nx;
     const int b = r.b0 + i % r.nb; i /= r.nb;
     const int d = r.d0 + i;
     return ((((long long)r.n * P.ntd + d) * P.nty + b) * P.ntx + x) * P.nnc + c;
+}
+// All dependencies of (l, t) as one index space: [0, ns) on the input producer, [ns, ns + nr) on the residual's.
+struct Deps {
+    DepRange s, r;
+    int ns, nr, ls, lr;
+};
+__host__ __device__ __forceinline__ Deps deps_of(const LayerP *ly, int l, long long t) {
+    Deps D;
+    const LayerP &C = ly[l];
+    D.ls = C.srcl;
+    D.lr = C.resl;
+    D.ns = D.nr = 0;
+    if (C.srcl >= 0) {
+        D.s = dep_range_src(C, ly[C.srcl], t);
+        D.ns = dep_count(D.s);
+    }
+    if (C.resl >= 0) {
+        D.r = dep_range_res(C, ly[C.resl], t);
+        D.nr = dep_count(D.r);
+    }
+    return D;
+}
+// i-th dependency: its layer and task
+__host__ __device__ __forceinline__ long long dep_at(const LayerP *ly, const Deps &D, int i, int &dl) {
+    if (i < D.ns) {
+        dl = D.ls;
+        return dep_task(ly[D.ls], D.s, i);
+    }
+    dl = D.lr;
+    return dep_task(ly[D.lr], D.r, i - D.ns);
 }
 
 // Padded mode: region of layer l's output needed for block (bd, by, bx) of the last layer (Fig 4:
@@ -299,14 +347,12 @@ __device__ void scheduler_padded(const Params &p, Shared &sh) {
     for (;;) {
         // two blocks at a time: their layers interleave (A.l0, B.l0, A.l1, B.l1, ...) so that a layer's
         // loads wait for the previous layer of the same block while the other block's MMAs run
-        // one ticket draw per pair, so every CTA overshoots by exactly one draw and the counter
-        // advance per run is deterministic (2*ceil(norder/2) + 2*grid; the host offsets ticket_base)
+        // one ticket draw per pair
         long long P[2];
         int np = 0;
         unsigned long long tk = 0;
-        if (lane == 0) tk = atomicAdd(&p.counters[4], 2ULL) - p.ticket_base;
+        if (lane == 0) tk = atomicAdd(&p.counters[4], 2ULL);
         tk = __shfl_sync(0xffffffff, tk, 0);
-        if ((long long)tk < 0) __trap();   // ticket accounting broken: fail loudly
         for (int i = 0; i < 2; i++)
             if ((long long)(tk + i) < p.norder) P[np++] = (long long)(tk + i);
         if (np == 0) break;
@@ -338,7 +384,7 @@ __device__ void scheduler_padded(const Params &p, Shared &sh) {
 
 __device__ void scheduler(const Params &p, Shared &sh) {
     const int lane = threadIdx.x % 32;
-    const unsigned EP = p.epoch << 2;
+    const unsigned EP = run_epoch(p.counters) << 2;
     const bool unmerged = p.only_layer >= 0;
     unsigned long long oks = 0, fails = 0;
     int sp = 0;
@@ -357,10 +403,9 @@ __device__ void scheduler(const Params &p, Shared &sh) {
     };
     for (;;) {
         unsigned long long tk = 0;
-        if (lane == 0) tk = atomicAdd(&p.counters[4], 1ULL) - p.ticket_base;
+        if (lane == 0) tk = atomicAdd(&p.counters[4], 1ULL);
         tk = __shfl_sync(0xffffffff, tk, 0);
         if ((long long)tk >= p.norder) break;
-        if ((long long)tk < 0) __trap();   // ticket accounting broken: fail loudly
         int l;
         long long t;
         if (unmerged) {
@@ -368,8 +413,8 @@ __device__ void scheduler(const Params &p, Shared &sh) {
             t = (long long)tk;
         } else {
             const int e = p.order[tk];
-            l = e >> 26;
-            t = e & ((1 << 26) - 1);
+            l = e >> kTaskBits;
+            t = e & ((1 << kTaskBits) - 1);
             int ok = 0;
             if (lane == 0) {
                 int *sw = status_word(p, l, t);
@@ -386,21 +431,21 @@ __device__ void scheduler(const Params &p, Shared &sh) {
         }
         sp = 1;
         if (!unmerged) {
-            // recursion (Fig 2d): claim not-started dependencies, deepest first in the emit order
+            // recursion (Fig 2d): claim not-started dependencies (input and residual producers), deepest first
+            // in the emit order
             for (int s = 0; s < sp; s++) {
                 __syncwarp();
                 const int sl = sh.stk_l[s];
                 const long long st = sh.stk_t[s];
-                if (sl == 0) continue;
-                const DepRange r = dep_range(p, sl, st);
-                const int nd = dep_count(r);
+                const Deps D = deps_of(p.layer, sl, st);
+                const int nd = D.ns + D.nr;
                 for (int i0 = 0; i0 < nd; i0 += 32) {
                     const int i = i0 + lane;
-                    int claimed = 0, busy = 0;
+                    int claimed = 0, busy = 0, dl = 0;
                     long long dt = 0;
                     if (i < nd && sp < kStack - 32) {
-                        dt = dep_task(p, sl, r, i);
-                        int *dw = status_word(p, sl - 1, dt);
+                        dt = dep_at(p.layer, D, i, dl);
+                        int *dw = status_word(p, dl, dt);
                         const int cur = ld_acquire(dw);
                         const int s2 = tag_state(cur, EP);
                         if (s2 == 0 && atomicCAS(dw, cur, (int)(EP | 1)) == cur) claimed = 1;
@@ -411,7 +456,7 @@ __device__ void scheduler(const Params &p, Shared &sh) {
                     oks += __popc(cm);
                     if (claimed) {
                         const int pos = sp + __popc(cm & ((1u << lane) - 1));
-                        sh.stk_l[pos] = sl - 1;
+                        sh.stk_l[pos] = dl;
                         sh.stk_t[pos] = dt;
                     }
                     sp += __popc(cm);
@@ -657,9 +702,10 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
     pdl_launch_dependents();
     // loaders / epilogue read the previous kernel's output; the scheduler rewrites memo tags that a previous
     // run of this subgraph may still be waiting on
-    if ((warp >= kLoad0 && warp < kLoad0 + kLW) || warp >= kEpi0 || warp == kSched) pdl_wait();
+    const bool waits = (warp >= kLoad0 && warp < kLoad0 + kLW) || warp >= kEpi0 || warp == kSched;
+    if (waits) pdl_wait();
 
-    const unsigned EP = p.epoch << 2;
+    const unsigned EP = waits ? run_epoch(p.counters) << 2 : 0u;
     if (warp == kSched) {
         if (p.padded) scheduler_padded(p, sh);
         else scheduler(p, sh);
@@ -683,14 +729,16 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     __threadfence();
                 }
                 __syncwarp();
-            } else if (l > 0 && !p.padded && p.only_layer < 0 && warp == kLoad0) {
-                // wait for the dependency tiles (state 2 of this epoch)
-                const DepRange r = dep_range(p, l, t);
-                const int nd = dep_count(r);
+            } else if (l >= 0 && !p.padded && p.only_layer < 0 && warp == kLoad0) {
+                // wait for the dependency tiles of the input and residual producers (state 2 of this epoch)
+                const Deps D = deps_of(p.layer, l, t);
+                const int nd = D.ns + D.nr;
                 unsigned long long spins = 0;
                 const unsigned long long td0 = clock64();
                 for (int i = lane; i < nd; i += 32) {
-                    const int *dw = status_word(p, l - 1, dep_task(p, l, r, i));
+                    int dl;
+                    const long long dt = dep_at(p.layer, D, i, dl);
+                    const int *dw = status_word(p, dl, dt);
                     while (ld_acquire(dw) != (int)(EP | 2)) {
                         spins++;
                         __nanosleep(32);
@@ -922,6 +970,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
     ptx::tc_fence_before();
     __syncthreads();
     if (warp == kMma) ptx::tmem_dealloc(sh.tmem_base, p.tmem_cols);
+    if (threadIdx.x == 0) run_exit(p.counters);
 }
 
 // weights [cout][kd][kh][kw][cin] bf16 -> [nc][kb][ks][2][Nc][8] per the layer's A mode
@@ -1135,8 +1184,12 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
         bdl_layout_init(&lo, nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
                         p->in_layout.Bn, p->in_layout.Bd, p->in_layout.Bh, p->in_layout.Bw, BDL_BF16);
         if (!gen_layer_static(ly, nsp, lo, g.layer[j])) return false;
+        g.layer[j].srcl = j < (int)sg.src_local.size() ? sg.src_local[j] : j - 1;
+        g.layer[j].resl = j < (int)sg.res_local.size() ? sg.res_local[j] : -1;
+        if (g.layer[j].resl >= 0 && g.layer[g.layer[j].resl].Nc != g.layer[j].Nc) return false;
     }
     if (padded && nconv > 1) {
+        if (!sg.chain) return false;   // padded mode: chains only (partition)
         // CTA blocks over the last layer's grid.  The planner's brick edge (rho/tau model, L649-658) sizes the
         // layout; a CTA's padded block is a band of bricks: start from the brick edge and double
         // while at least one block per SM remains, so small maps (7x7, 14x14) do not end up with 4x4 blocks whose
@@ -1178,6 +1231,10 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
             const bool xal = j == 0 && gen_pad_tma_ok(G, nsp, Bw);
             G.xal = xal ? 1 : 0;
             if (!gen_layer_tiles(G, G.pR[1], xal ? G.pR[2] + Bw - 1 : G.pR[2], xal ? Bw : 1)) return false;
+            // padded sub-task ids pack (sub-tile << 8 | channel chunk): 16 + 8 bits
+            const int xs = xal ? G.pR[2] + Bw - 1 : G.pR[2];
+            const long long nsub = (long long)G.pR[0] * ((G.pR[1] + G.Tb - 1) / G.Tb) * ((xs + G.Tw - 1) / G.Tw);
+            if (nsub >= (1LL << 16) || G.nnc >= (1 << 8)) return false;
             if (j < nconv - 1) {
                 G.scr_off = g.scr_slot;
                 g.scr_slot += ((long long)G.pR[0] * G.pR[1] * G.pR[2] * G.cout * 2 + 255) / 256 * 256;
@@ -1191,6 +1248,7 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
             G.nty = (G.grid[1] + G.Tb - 1) / G.Tb;
             G.ntx = (G.grid[2] + G.Tw - 1) / G.Tw;
             G.ntasks = (long long)p->layers[sg.first + j].out_ext[0] * G.ntd * G.nty * G.ntx * G.nnc;
+            if (G.ntasks >= (1LL << gen::kTaskBits)) return false;   // order entries: (layer << 26) | task
         }
     }
     int in_stride = 0, w_stride = 0, acc = 0;
@@ -1221,13 +1279,26 @@ int gen_conv_layers(const bdl_plan *p, const Subgraph &sg) {
     if (L < 1 || L > kMaxLayers) return 0;
     for (int j = 0; j < L; j++) {
         if (p->layers[sg.first + j].L.kind != BDL_OP_CONV) return 0;
-        int rt = sg.res_tensor[j];
-        if (p->layers[sg.first + j].L.residual != BDL_NO_RESIDUAL && rt < 0) return 0;
+        const bool res = p->layers[sg.first + j].L.residual != BDL_NO_RESIDUAL;
+        if (res && sg.res_tensor[j] < 0 && sg.res_local[j] < 0) return 0;
     }
+    if (L < sg.last - sg.first + 1 && p->layers[sg.last].L.input != sg.first + L - 1) return 0;   // pool tail: last conv
     GenGeom g;
     if (!gen_geometry(p, sg, L, false, g)) return 0;
-    if (L > 1 && !gen_geometry(p, sg, L, true, g)) return 0;
+    if (L > 1 && sg.chain && !gen_geometry(p, sg, L, true, g)) return 0;
     return L;
+}
+
+// Can layer `li` of the plan run on the generic kernel (the planner's test for branched subgraphs)?
+bool gen_layer_supported(const bdl_plan *p, int li) {
+    if (p->in_layout.dtype != BDL_BF16 || p->in_layout.Bn != 1) return false;
+    const Layer &ly = p->layers[li];
+    bdl_layout lo;
+    bdl_layout_init(&lo, p->in_layout.nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
+                    p->in_layout.Bn, p->in_layout.Bd, p->in_layout.Bh, p->in_layout.Bw, BDL_BF16);
+    gen::LayerP G;
+    memset(&G, 0, sizeof(G));
+    return gen_layer_static(ly, p->in_layout.nsp, lo, G) && gen_layer_tiles(G, G.grid[1], G.grid[2], p->in_layout.Bw);
 }
 
 // Tasks (memo status words) of conv layer j of the generic kernel's subgraph.
@@ -1257,8 +1328,17 @@ size_t gen_packed_bytes(const bdl_plan *p, const Subgraph &sg, int j) {
     return (size_t)G.nnc * G.nkb * G.nks * 2 * G.Nc * 8 * 2;
 }
 
-// Topological task order: images in groups (enough tiles in flight to fill the GPU, intermediates of a
-// group L2-resident), layer by layer within a group.
+// Memo task order (host, uploaded at prepare).  Tickets are drawn along it; any order is correct (the scheduler
+// claims missing dependencies first), the order only decides locality and waiting.
+//  * default: locality-aware wavefront (the paper's future work, L1785-1791).  Images run in groups large
+//    enough to keep every SM busy; inside a group each task gets a scan key: a task that reads only external
+//    tensors is keyed by the fraction of its input frame (d, y, x raster order) its window reaches, and a task
+//    with producers inside the subgraph by the largest key among its dependencies plus a lag of about two
+//    waves of that layer's tasks.  Sorting by key interleaves the layers as a wavefront that streams each image
+//    top to bottom: a layer's tiles are consumed shortly after they are produced, while they are still in L2,
+//    instead of layer by layer (3-D volumes: 402 MB of cfg5 intermediates would not fit).
+//  * schedule_seed != 0: a seeded random topological order (Kahn's algorithm drawing uniformly from the ready
+//    set), for schedule-invariance tests.
 std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
     const int L = gen_conv_layers(p, sg);
     std::vector<int> ord;
@@ -1266,15 +1346,84 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
     GenGeom g;
     gen_geometry(p, sg, L, false, g);
     const int N = p->layers[sg.first].in_ext[0];
+    std::vector<long long> base(L + 1, 0);
+    for (int j = 0; j < L; j++) base[j + 1] = base[j] + g.layer[j].ntasks;
+    const long long total = base[L];
+    auto enc = [&](int j, long long t) { return (j << gen::kTaskBits) | (int)t; };
+    if (p->opts.schedule_seed) {
+        // dependents lists + in-degrees, then Kahn with a seeded uniform pick from the ready set
+        std::vector<int> indeg(total, 0);
+        std::vector<std::vector<int>> out(total);
+        for (int j = 0; j < L; j++)
+            for (long long t = 0; t < g.layer[j].ntasks; t++) {
+                const gen::Deps D = gen::deps_of(g.layer, j, t);
+                for (int i = 0; i < D.ns + D.nr; i++) {
+                    int dl;
+                    const long long dt = gen::dep_at(g.layer, D, i, dl);
+                    out[base[dl] + dt].push_back((int)(base[j] + t));
+                    indeg[base[j] + t]++;
+                }
+            }
+        std::vector<int> ready;
+        for (long long u = 0; u < total; u++)
+            if (!indeg[u]) ready.push_back((int)u);
+        std::mt19937 rng((unsigned)p->opts.schedule_seed);
+        while (!ready.empty()) {
+            const size_t k = std::uniform_int_distribution<size_t>(0, ready.size() - 1)(rng);
+            const int u = ready[k];
+            ready[k] = ready.back();
+            ready.pop_back();
+            const int j = (int)(std::upper_bound(base.begin(), base.end(), (long long)u) - base.begin()) - 1;
+            ord.push_back(enc(j, u - base[j]));
+            for (int v : out[u])
+                if (--indeg[v] == 0) ready.push_back(v);
+        }
+        return ord;
+    }
+    static const bool layer_major = [] { const char *e = getenv("BDL_GEN_ORDER"); return e && !strcmp(e, "layer"); }();
     long long per_img0 = g.layer[0].ntasks / N;
     int G = (int)std::max<long long>(1, (2LL * p->num_sms + per_img0 - 1) / std::max<long long>(1, per_img0));
     G = std::min(G, N);
-    for (int n0 = 0; n0 < N; n0 += G)
-        for (int j = 0; j < L; j++) {
-            const long long per = g.layer[j].ntasks / N;
-            for (int n = n0; n < std::min(N, n0 + G); n++)
-                for (long long t = 0; t < per; t++) ord.push_back((j << 26) | (int)(n * per + t));
+    std::vector<double> key(total, 0.0);
+    for (int j = 0; j < L; j++) {
+        const gen::LayerP &C = g.layer[j];
+        const double per_img = (double)C.ntasks / N;
+        // BDL_GEN_ORDER=layer (A/B runs): layer by layer inside each image group
+        const double lag = layer_major ? 2.0 : std::min(1.0, 2.0 * p->num_sms / (G * per_img));
+        const double frame = (double)C.in_ext[0] * C.in_ext[1] * C.in_ext[2];
+        for (long long t = 0; t < C.ntasks; t++) {
+            const gen::Deps D = gen::deps_of(g.layer, j, t);
+            double k = -1.0;
+            for (int i = 0; i < D.ns + D.nr; i++) {
+                int dl;
+                const long long dt = gen::dep_at(g.layer, D, i, dl);
+                k = std::max(k, key[base[dl] + dt]);
+            }
+            if (D.ns == 0) {   // reads an external tensor: how far down its input frame the window reaches
+                const gen::TaskC c = gen::decode(C, t);
+                const int z = std::min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.k[0] - 1);
+                const int y = std::min(C.in_ext[1] - 1, (c.ty * C.Tb + C.Tb - 1) * C.s[1] - C.pd[1] + C.k[1] - 1);
+                const int x = std::min(C.in_ext[2] - 1, (c.tx * C.Tw + C.Tw - 1) * C.s[2] - C.pd[2] + C.k[2] - 1);
+                k = std::max(k, ((double)std::max(z, 0) * C.in_ext[1] + std::max(y, 0)) * C.in_ext[2] + std::max(x, 0)) /
+                    frame;
+            }
+            if (D.ns + D.nr > 0) k += lag;
+            key[base[j] + t] = k;
         }
+    }
+    struct E { int grp; double key; int j; long long t; };
+    std::vector<E> es;
+    es.reserve(total);
+    for (int j = 0; j < L; j++) {
+        const long long per = g.layer[j].ntasks / N;
+        for (long long t = 0; t < g.layer[j].ntasks; t++) es.push_back({(int)(t / per) / G, key[base[j] + t], j, t});
+    }
+    std::stable_sort(es.begin(), es.end(), [](const E &a, const E &b) {
+        if (a.grp != b.grp) return a.grp < b.grp;
+        if (a.key != b.key) return a.key < b.key;
+        return a.j < b.j;
+    });
+    for (const E &e : es) ord.push_back(enc(e.j, e.t));
     return ord;
 }
 
@@ -1295,7 +1444,7 @@ bdl_status launch_pack_gen(const bdl_plan *p, const Subgraph &sg, int j, void *w
 bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &in, const TView &out,
                                  const std::vector<TView> &res_views, unsigned char *ws, cudaStream_t s, int *launches);
 
-bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out,
+bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TView> &srcv, const TView &out,
                                const std::vector<TView> &res, unsigned char *wsp, cudaStream_t s, int *launches) {
     const int L = gen_conv_layers(p, sg);
     if (L <= 0) return fail(BDL_EUNSUPPORTED, "generic tcgen05 kernel: subgraph not supported");
@@ -1307,7 +1456,9 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
     memset(&P, 0, sizeof(P));
     P.L = L;
     P.prof = gen_prof_buffer(s);
+#ifdef BDL_DEBUG   // timing knobs that deliberately skip work (wrong results): debug builds only
     if (const char *e = getenv("BDL_GEN_DBG")) P.dbg = atoi(e);
+#endif
     if (getenv("BDL_GEN_GEOM")) {
         for (int j = 0; j < L; j++) {
             const gen::LayerP &G = g.layer[j];
@@ -1331,7 +1482,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
                             p->in_layout.Bn, p->in_layout.Bd, p->in_layout.Bh, p->in_layout.Bw, BDL_BF16);
             outs[j] = make_view(lo, wsp + sg.memo_off[j]);
         }
-        G.src = j == 0 ? in : outs[j - 1];
+        G.src = G.srcl >= 0 ? outs[G.srcl] : srcv[j];
         G.out = outs[j];
         G.tma = 0;
         G.pxo = 0;
@@ -1354,8 +1505,9 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
                  G.Tw % p->in_layout.Bw == 0 && 2 * G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
                  gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, 2 * G.Tw / p->in_layout.Bw, 2))
             G.tma = 2;
-        G.has_res = sg.res_tensor[j] >= 0;
-        if (G.has_res) G.res = res[j];
+        G.has_res = sg.res_tensor[j] >= 0 || G.resl >= 0;
+        if (sg.res_tensor[j] >= 0) G.res = res[j];
+        else if (G.resl >= 0) G.res = outs[G.resl];
         G.relu = ly.L.relu;
         G.w = (const __nv_bfloat16 *)(wsp + ly.tc_w_off);
         G.bias = (const float *)(wsp + ly.b_off);
@@ -1369,7 +1521,6 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
     P.acc_stride = g.acc_stride;
     P.tmem_cols = g.tmem_cols;
     P.status = (int *)(wsp + sg.status_off);
-    P.epoch = sg.epoch;
     P.counters = (unsigned long long *)(wsp + sg.counter_off);
     cudaFuncSetAttribute(gen::gen_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
     const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;
@@ -1384,8 +1535,6 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
         P.scr_slot = g.scr_slot;
         P.norder = (long long)p->layers[sg.first].in_ext[0] * g.npb[0] * g.npb[1] * g.npb[2];
         const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-        P.ticket_base = sg.ticket_base;
-        sg.ticket_base += 2 * (((unsigned long long)P.norder + 1) / 2) + 2 * grid;
         launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
         *launches += 1;
     } else if (!unmerged) {
@@ -1393,8 +1542,6 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
         P.order = (const int *)(wsp + sg.order_off);
         P.norder = sg.norder;
         const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-        P.ticket_base = sg.ticket_base;
-        sg.ticket_base += (unsigned long long)P.norder + grid;
         launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
         *launches += 1;
     } else {
@@ -1403,8 +1550,6 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const
             P.only_layer = j;
             P.norder = P.layer[j].ntasks;
             const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-            P.ticket_base = sg.ticket_base;
-            sg.ticket_base += (unsigned long long)P.norder + grid;
             launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
             *launches += 1;
         }

@@ -85,9 +85,7 @@ struct Params {
     TView in, res;
     int *status;
     long long task_base[kMaxLayers];
-    unsigned epoch;
-    unsigned long long *counters;   // [0] computed [1] cas_ok [2] cas_fail [3] spins [4] ticket [5] trace idx
-    unsigned long long ticket_base;
+    unsigned long long *counters;   // run state (common.cuh run_epoch / run_exit); [7] debug trace index
     const int *order;               // encoded (l << 24) | tile, or null (unmerged: identity over only_layer)
     long long norder;
     int only_layer;
@@ -207,7 +205,7 @@ __device__ __forceinline__ void load_tile(const Params &p, const TView &src_in, 
 // CAS-ed by 9 lanes at once -- and hands claimed tasks to the loaders, dependencies first.
 __device__ void scheduler(const Params &p, Shared &sh) {
     const int lane = threadIdx.x % 32;
-    const unsigned EP = p.epoch << 2;
+    const unsigned EP = run_epoch(p.counters) << 2;
     const bool unmerged = p.only_layer >= 0;
     unsigned long long oks = 0, fails = 0;
     int sp = 0;
@@ -226,7 +224,7 @@ __device__ void scheduler(const Params &p, Shared &sh) {
     for (;;) {
         if (sp == 0) {
             unsigned long long tk = 0;
-            if (lane == 0) tk = atomicAdd(&p.counters[4], 1ULL) - p.ticket_base;
+            if (lane == 0) tk = atomicAdd(&p.counters[4], 1ULL);
             tk = __shfl_sync(0xffffffff, tk, 0);
             if ((long long)tk >= p.norder) break;
             int l;
@@ -477,7 +475,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
     } else if (warp < RL::WPROD) {
         // ------------------------------------------------------------------ loaders
         const int tidl = threadIdx.x - 32 * kLoadWarp0;
-        const unsigned EP = p.epoch << 2;
+        const unsigned EP = run_epoch(p.counters) << 2;
         for (uint32_t seq = 0;; seq++) {
             const int slot = seq % kQ;
             ptx::mbar_wait(&sh.q_full[slot], (seq / kQ) & 1);
@@ -599,14 +597,15 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
             long long prev_t = 0;
             uint32_t prev_seq = 0;
             unsigned long long prev_sync = 0, prev_read = 0;
+            const unsigned EPs = run_epoch(p.counters) << 2;
             auto publish = [&](int l, long long t, uint32_t sq, unsigned long long t_sync, unsigned long long t_read) {
                 if (p.only_layer < 0) {
                     __threadfence();
-                    st_release(status_word(p, l, t), (int)((p.epoch << 2) | 2));
+                    st_release(status_word(p, l, t), (int)(EPs | 2));
                 }
                 atomicAdd(&p.counters[0], 1ULL);
                 if (p.trace) {
-                    unsigned long long k = atomicAdd(&p.counters[5], 1ULL);
+                    unsigned long long k = atomicAdd(&p.counters[7], 1ULL);
                     if (k < (unsigned long long)p.trace_cap) {
                         unsigned smid;
                         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
@@ -802,6 +801,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
     ptx::tc_fence_before();
     __syncthreads();
     if (warp == kMmaWarp) ptx::tmem_dealloc(sh.tmem_base, p.tmem_cols);
+    if (threadIdx.x == 0) run_exit(p.counters);
 }
 
 
@@ -870,7 +870,10 @@ bool ws_geometry(const bdl_plan *p, const Subgraph &sg, WsGeom &g) {
             break;  // widest fitting Tw for this Tb
         }
     }
-    return best > 0;
+    if (best <= 0) return false;
+    // task ids are packed as (layer << 24) | tile in the order list: the tile index must fit 24 bits
+    const long long ntiles = (long long)f.in_ext[0] * ((H + g.Tb - 1) / g.Tb) * ((W + g.Tw - 1) / g.Tw);
+    return ntiles < (1LL << 24);
 }
 
 // Locality-aware wavefront order (host): step s, image n, layer l -> tile row b = s - lag*l.
@@ -899,8 +902,6 @@ static bdl_status launch_ws_C(bdl_plan *p, Subgraph &sg, ws::Params &P, const Ws
     int grid = (int)std::min<long long>(ntiles * (unmerged ? 1 : P.L), (long long)p->num_sms);
     if (!unmerged) {
         P.only_layer = -1;
-        P.ticket_base = sg.ticket_base;
-        sg.ticket_base += (unsigned long long)P.norder + grid;
         launch_pdl(k, dim3(grid), dim3(ws::Roles<C>::THREADS), g.smem, s, P);
         *launches += 1;
     } else {
@@ -909,8 +910,6 @@ static bdl_status launch_ws_C(bdl_plan *p, Subgraph &sg, ws::Params &P, const Ws
         grid = (int)std::min<long long>(ntiles, (long long)p->num_sms);
         for (int l = 0; l < P.L; l++) {
             P.only_layer = l;
-            P.ticket_base = sg.ticket_base;
-            sg.ticket_base += (unsigned long long)P.norder + grid;
             launch_pdl(k, dim3(grid), dim3(ws::Roles<C>::THREADS), g.smem, s, P);
             *launches += 1;
         }
@@ -1026,11 +1025,12 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
         }
     }
     P.status = (int *)(wsp + sg.status_off);
-    P.epoch = sg.epoch;
     P.counters = (unsigned long long *)(wsp + sg.counter_off);
     P.order = sg.order_off >= 0 ? (const int *)(wsp + sg.order_off) : nullptr;
     P.norder = sg.norder;
+#ifdef BDL_DEBUG   // timing knobs that deliberately skip work (wrong results): debug builds only
     if (const char *e = getenv("BDL_WS_DBG")) P.dbg = atoi(e);
+#endif
     if (const char *e = getenv("BDL_TRACE")) {
         static unsigned long long *tbuf = nullptr;
         static int tcap = 0;

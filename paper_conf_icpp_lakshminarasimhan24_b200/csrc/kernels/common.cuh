@@ -44,6 +44,30 @@ __device__ __forceinline__ void st_release(int *p, int v) {
     asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
+// ---- per-run state of a persistent memo kernel, kept on the device (no host-side counters, so a plan's
+// launches can be replayed from a CUDA graph).  Counter block of a subgraph (workspace, zeroed by
+// bdl_plan_prepare):
+//   [0] tasks computed  [1] successful CAS claims  [2] failed claims / busy deps  [3] spin polls
+//       (accumulated since prepare, read by bdl_plan_counters)
+//   [4] ticket counter of the running launch (starts at 0)
+//   [5] memo-tag epoch of the running launch
+//   [6] CTAs of the running launch that have exited
+// A launch reads its epoch after pdl_wait(); the last CTA to exit rewinds the ticket counter and advances the
+// epoch, so tags written by this launch read as state 0 ("not started") in the next one.
+__device__ __forceinline__ unsigned run_epoch(const unsigned long long *c) {
+    return (unsigned)*reinterpret_cast<const volatile unsigned long long *>(c + 5);
+}
+// Thread 0 of every CTA, after the CTA's last use of the ticket counter and of the epoch.
+__device__ __forceinline__ void run_exit(unsigned long long *c) {
+    __threadfence();
+    if (atomicAdd(&c[6], 1ULL) == (unsigned long long)(gridDim.x * gridDim.y * gridDim.z) - 1) {
+        atomicExch(&c[4], 0ULL);
+        atomicExch(&c[6], 0ULL);
+        __threadfence();
+        atomicAdd(&c[5], 1ULL);
+    }
+}
+
 // Programmatic dependent launch (PDL): a kernel launched with launch_pdl() may start while the previous
 // kernel in the stream drains; it must call pdl_wait() before touching that kernel's outputs.
 __device__ __forceinline__ void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }

@@ -21,21 +21,49 @@ static int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 // ---------------------------------------------------------------------------------------------
 // Region analysis (Fig 4): reverse traversal from an output brick region [a, b) of the
 // subgraph's last layer; returns per layer the INPUT region of that layer (unclipped) along one dim.
-// in_lo[j], in_hi[j] for j = 0..L-1 (layer first+j).
-static void regions_1d(const std::vector<Layer> &ly, int first, int last, int dim, int64_t a, int64_t b,
-                       std::vector<int64_t> &in_lo, std::vector<int64_t> &in_hi) {
+// in_lo[j], in_hi[j] for j = 0..L-1 (layer first+j).  The traversal follows the graph, not the listing:
+// a layer's input region is added to the output region needed of the layer it reads, and its output
+// region to that of its residual's producer (branches merge by interval hull), so a projection
+// shortcut or a skip connection inside the subgraph is sized by its real consumers.  For a chain this
+// is the paper's Fig 4 recursion I = s(O-1) + k.  halo = false: the halo-free region s(O-1) + min(k, s) (windows
+// that do not overlap: a pool of k = s needs B x s without padding, L456-458), so Delta >= 0.
+static void regions_dag(const std::vector<Layer> &ly, int first, int last, int dim, int64_t a, int64_t b, bool halo,
+                        std::vector<int64_t> &in_lo, std::vector<int64_t> &in_hi) {
     int L = last - first + 1;
+    std::vector<int64_t> olo(L, INT64_MAX), ohi(L, INT64_MIN);
+    olo[L - 1] = a;
+    ohi[L - 1] = b;
     in_lo.assign(L, 0);
     in_hi.assign(L, 0);
     for (int j = L - 1; j >= 0; j--) {
+        if (olo[j] >= ohi[j]) continue;   // output not needed inside the subgraph (a live-out only)
         const bdl_layer &l = ly[first + j].L;
         int k = dim == 0 ? 1 : l.k[dim - 1], s = dim == 0 ? 1 : l.stride[dim - 1], p = dim == 0 ? 0 : l.pad[dim - 1];
-        int64_t lo = a * s - p, hi = (b - 1) * s - p + k;  // input extent I = s(O-1) + k (Q19)
+        int64_t lo, hi;
+        if (halo) {
+            lo = olo[j] * s - p;               // input extent I = s(O-1) + k (Q19)
+            hi = (ohi[j] - 1) * s - p + k;
+        } else {                               // halo-free: non-overlapping windows of the same stride
+            lo = olo[j] * s;
+            hi = (ohi[j] - 1) * s + std::min(k, s);
+        }
         in_lo[j] = lo;
         in_hi[j] = hi;
-        a = lo;
-        b = hi;
+        const int src = l.input - first;
+        if (src >= 0) {
+            olo[src] = std::min(olo[src], lo);
+            ohi[src] = std::max(ohi[src], hi);
+        }
+        if (l.residual != BDL_NO_RESIDUAL && l.residual >= first) {
+            const int r = l.residual - first;
+            olo[r] = std::min(olo[r], olo[j]);
+            ohi[r] = std::max(ohi[r], ohi[j]);
+        }
     }
+}
+static void regions_1d(const std::vector<Layer> &ly, int first, int last, int dim, int64_t a, int64_t b,
+                       std::vector<int64_t> &in_lo, std::vector<int64_t> &in_hi) {
+    regions_dag(ly, first, last, dim, a, b, true, in_lo, in_hi);
 }
 
 // Delta: sum over layers and bricks of the padded input region (clipped at the feature
@@ -51,19 +79,9 @@ double compute_delta(const std::vector<Layer> &ly, int first, int last, const in
         std::vector<double> ps(L, 0.0), es(L, 0.0);
         for (int64_t i = 0; i < nb; i++) {
             int64_t a = i * B[dim], b = std::min<int64_t>(a + B[dim], ext_out);
-            std::vector<int64_t> lo, hi;
-            regions_1d(ly, first, last, dim, a, b, lo, hi);
-            // halo-free region: strides only
-            int64_t ea = a, eb = b;
-            std::vector<int64_t> elo(L), ehi(L);
-            for (int j = L - 1; j >= 0; j--) {
-                const bdl_layer &l = ly[first + j].L;
-                int s = dim == 0 ? 1 : l.stride[dim - 1];
-                ea *= s;
-                eb *= s;
-                elo[j] = ea;
-                ehi[j] = eb;
-            }
+            std::vector<int64_t> lo, hi, elo, ehi;
+            regions_dag(ly, first, last, dim, a, b, true, lo, hi);
+            regions_dag(ly, first, last, dim, a, b, false, elo, ehi);
             for (int j = 0; j < L; j++) {
                 int64_t I = ly[first + j].in_ext[dim];
                 ps[j] += (double)std::max<int64_t>(0, std::min(hi[j], I) - std::max<int64_t>(lo[j], 0));
@@ -124,6 +142,7 @@ size_t gen_packed_bytes(const bdl_plan *p, const Subgraph &sg, int j);
 std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg);
 
 int64_t gen_scratch_bytes(const bdl_plan *p, const Subgraph &sg);
+bool gen_layer_supported(const bdl_plan *p, int layer);
 
 int effective_kernel(const Subgraph &sg) { return sg.kernel; }
 }
@@ -135,7 +154,7 @@ using namespace bdl;
 
 static bool tc_eligible(const bdl_plan *p, const Subgraph &sg) {
     if (p->in_layout.dtype != BDL_BF16) return false;
-    if (p->in_layout.Bn != 1) return false;
+    if (p->in_layout.Bn != 1 || !sg.chain) return false;
     const Layer &f = p->layers[sg.first];
     int C = f.L.cin;
     if (!(C == 16 || C == 32 || C == 64 || C == 128)) return false;
@@ -154,7 +173,8 @@ static bool tc_eligible(const bdl_plan *p, const Subgraph &sg) {
         if (l.residual != BDL_NO_RESIDUAL && rt < 0) return false;
     }
     int smem = 0;
-    return tc_band_rows(p, sg, &smem) > 0;
+    // memoized / unmerged run on the warp-specialized kernel (C <= 64); wider chains go to the generic kernel
+    return tc_band_rows(p, sg, &smem) > 0 && ws_band_rows(p, sg) > 0;
 }
 
 extern "C" {
@@ -252,19 +272,26 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             if (p->layers[j].L.input == m || p->layers[j].L.residual == m) return true;
         return false;
     };
+    // DAG subgraphs (a layer reading a non-previous layer, a residual produced inside the subgraph, or an inner
+    // layer read by a later subgraph) run on the generic tcgen05 kernel, which tracks per-layer producers; the
+    // paper ends subgraphs only at pools and normalisations (L620-626), not at branches.
+    const bool dag_ok = in->dtype == BDL_BF16 && in->Bn == 1;
     auto range_ok = [&](int first, int end) {
         if (p->opts.max_subgraph_layers > 0 && end - first + 1 > p->opts.max_subgraph_layers) return false;
         if (end - first + 1 > kMaxLayers) return false;
+        bool branch = false, all_gen = true;
         for (int j = first; j <= end; j++) {
             if (!fits_brick(j)) return false;
-            if (j > first && p->layers[j].L.input != j - 1) return false;      // a chain
             if (j < end && is_pool(p->layers[j])) return false;                 // pool ends a subgraph (L620-626)
-            int r = p->layers[j].L.residual;
-            if (r != BDL_NO_RESIDUAL && r >= first) return false;                // residual must be materialized
-            if (j < end && consumed_after(j, end)) return false;               // no live-out inside
+            const int r = p->layers[j].L.residual;
+            branch = branch || (j > first && p->layers[j].L.input != j - 1) || (r != BDL_NO_RESIDUAL && r >= first) ||
+                     (j < end && consumed_after(j, end));
+            if (!(j == end && is_pool(p->layers[j]))) all_gen = all_gen && gen_layer_supported(p, j);
         }
-        // footprint (L605-614): concurrently resident bricks x padded regions (+ memo tags)
-        int nconc = 2 * p->num_sms;
+        if (branch && !(dag_ok && all_gen)) return false;
+        // footprint (L605-614): concurrently resident bricks x padded regions + weights.  The persistent kernels hold
+        // one tile's region per SM at a time, so the resident bricks are one per SM.
+        int nconc = p->num_sms;
         int64_t fp = 0;
         std::vector<int64_t> lo, hi;
         int64_t vol_sum = 0;
@@ -316,6 +343,39 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             bdl_plan_destroy(p);
             return fail(BDL_EINVAL, "partition: subgraph input is not materialized (internal error)");
         }
+        bool liveout = false;
+        for (int j = sg.first; j <= sg.last; j++) {
+            const bdl_layer &l = p->layers[j].L;
+            const int src = l.input >= sg.first ? l.input - sg.first : -1;
+            sg.src_local.push_back(src);
+            int st = -1;
+            if (src < 0) {
+                st = tensor_of(l.input);
+                if (st < 0) {
+                    bdl_plan_destroy(p);
+                    return fail(BDL_EINVAL, "partition: layer " + std::to_string(j) + " input is not materialized");
+                }
+            }
+            sg.src_tensor.push_back(st);
+            if (j > sg.first && src != j - 1 - sg.first) sg.chain = false;
+            const int r2 = l.residual;
+            if (r2 != BDL_NO_RESIDUAL && r2 >= sg.first) {
+                sg.res_local.push_back(r2 - sg.first);
+                sg.res_tensor.push_back(-1);
+                sg.chain = false;
+            } else if (r2 != BDL_NO_RESIDUAL) {
+                int t2 = tensor_of(r2);
+                if (t2 < 0) {
+                    bdl_plan_destroy(p);
+                    return fail(BDL_EUNSUPPORTED, "layer " + std::to_string(j) + ": residual source is not materialized");
+                }
+                sg.res_local.push_back(-1);
+                sg.res_tensor.push_back(t2);
+            } else {
+                sg.res_local.push_back(-1);
+                sg.res_tensor.push_back(-1);
+            }
+        }
         const Layer &ll = p->layers[sg.last];
         Tensor t;
         t.producer = sg.last;
@@ -326,19 +386,19 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             t.layout.brickmap = in->brickmap;  // same grid: keep the caller's BrickMap
         p->tensors.push_back(t);
         sg.out_tensor = (int)p->tensors.size() - 1;
-        for (int j = sg.first; j <= sg.last; j++) {
-            int r2 = p->layers[j].L.residual;
-            if (r2 == BDL_NO_RESIDUAL) {
-                sg.res_tensor.push_back(-1);
-            } else {
-                int t2 = tensor_of(r2);
-                if (t2 < 0) {
-                    bdl_plan_destroy(p);
-                    return fail(BDL_EUNSUPPORTED, "layer " + std::to_string(j) + ": residual source is not a subgraph output");
-                }
-                sg.res_tensor.push_back(t2);
-            }
+        // inner layers read by later subgraphs: their memo buffers are materialized tensors
+        for (int j = sg.first; j < sg.last; j++) {
+            if (!consumed_after(j, sg.last)) continue;
+            const Layer &ly = p->layers[j];
+            Tensor lt;
+            lt.producer = j;
+            bdl_layout_init(&lt.layout, nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
+                            in->Bn, in->Bd, in->Bh, in->Bw, in->dtype);
+            lt.ws_off = 0;
+            p->tensors.push_back(lt);
+            liveout = true;
         }
+        if (liveout) sg.chain = false;
         // ---- models
         int ext_in[4];
         for (int d = 0; d < 4; d++) ext_in[d] = fl.in_ext[d];
@@ -356,14 +416,22 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
         if (sg.last == sg.first) sg.mode_model = BDL_MODE_UNMERGED;
         else if (rho_exec < (double)bn) sg.mode_model = BDL_MODE_UNMERGED;
         else sg.mode_model = sg.delta > p->opts.delta_threshold ? BDL_MODE_MEMOIZED : BDL_MODE_PADDED;
+        // padded mode recomputes a chain per CTA block and materializes only the last layer: a DAG subgraph
+        // (branches, inner live-outs) executes memoized instead
+        if (!sg.chain && sg.mode_model == BDL_MODE_PADDED) sg.mode_model = BDL_MODE_MEMOIZED;
         sg.mode = p->opts.force_mode != BDL_MODE_AUTO ? p->opts.force_mode : sg.mode_model;
+        if (!sg.chain && sg.mode == BDL_MODE_PADDED) sg.mode = BDL_MODE_MEMOIZED;
         p->sgs.push_back(sg);
     }
-    p->tensors.back().ws_off = -1;  // graph output is the user's buffer
-    p->out_layout = p->tensors.back().layout;
+    p->tensors[p->sgs.back().out_tensor].ws_off = -1;  // graph output is the user's buffer
+    p->out_layout = p->tensors[p->sgs.back().out_tensor].layout;
     for (auto &sg : p->sgs) {
         sg.kernel = tc_eligible(p, sg) ? KERNEL_TC_BAND : KERNEL_BRICK;
         if (sg.kernel == KERNEL_BRICK && (sg.gen_layers = gen_conv_layers(p, sg)) > 0) sg.kernel = KERNEL_TC_GEN;
+        if (!sg.chain && sg.kernel != KERNEL_TC_GEN) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EUNSUPPORTED, "partition: a branched subgraph cannot run on the generic kernel");
+        }
     }
 
     // ---- workspace layout
@@ -388,7 +456,8 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             }
         else if (sg.kernel == KERNEL_TC_GEN)
             for (int j = 0; j < sg.gen_layers; j++) p->layers[sg.first + j].tc_w_off = take(gen_packed_bytes(p, sg, j));
-    for (size_t t = 1; t + 1 < p->tensors.size(); t++) p->tensors[t].ws_off = take(p->tensors[t].layout.total_bytes);
+    for (size_t t = 1; t < p->tensors.size(); t++)
+        if (p->tensors[t].ws_off == 0) p->tensors[t].ws_off = take(p->tensors[t].layout.total_bytes);
     for (auto &sg : p->sgs) {
         int L = sg.last - sg.first + 1;
         sg.memo_off.assign(L, -1);
@@ -399,7 +468,10 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             bdl_layout lo;
             bdl_layout_init(&lo, nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
                             in->Bn, in->Bd, in->Bh, in->Bw, in->dtype);
-            if (j < L - 1) sg.memo_off[j] = take(lo.total_bytes);
+            if (j < L - 1) {
+                const int lt = tensor_of(sg.first + j);   // a live-out's buffer is its tensor
+                sg.memo_off[j] = lt >= 0 ? p->tensors[lt].ws_off : take(lo.total_bytes);
+            }
             sg.task_base[j] = words;
             // memo tags: one per brick, or per band task of the tcgen05 kernels (bands of >= 1 row)
             int64_t w = std::max<int64_t>(lo.nbricks, lo.N * lo.D * lo.H * lo.nb[3]);
@@ -461,6 +533,7 @@ bdl_status bdl_plan_set_mode(bdl_plan *p, int32_t i, int32_t mode) {
     if (!p || i < 0 || i >= (int)p->sgs.size()) return fail(BDL_EINVAL, "bdl_plan_set_mode: bad index");
     if (mode == BDL_MODE_AUTO) mode = p->sgs[i].mode_model;
     if (mode < BDL_MODE_PADDED || mode > BDL_MODE_UNMERGED) return fail(BDL_EINVAL, "bdl_plan_set_mode: bad mode");
+    if (mode == BDL_MODE_PADDED && !p->sgs[i].chain) mode = BDL_MODE_MEMOIZED;   // DAG subgraph: see partition
     p->sgs[i].mode = mode;
     p->prepared = false;
     return BDL_OK;

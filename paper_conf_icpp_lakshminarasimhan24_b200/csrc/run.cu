@@ -21,7 +21,7 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
                               unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged);
 int tc_launches(const bdl_plan *p, const Subgraph &sg);
 bdl_status launch_pack_gen(const bdl_plan *p, const Subgraph &sg, int j, void *w_out, cudaStream_t s);
-bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out,
+bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TView> &srcv, const TView &out,
                                const std::vector<TView> &res, unsigned char *wsp, cudaStream_t s, int *launches);
 int gen_launches(const bdl_plan *p, const Subgraph &sg);
 
@@ -62,8 +62,6 @@ bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream) {
             cudaMemcpyAsync(ws + sg.order_off, sg.order_host.data(), sg.norder * 4, cudaMemcpyHostToDevice, s);
         cudaMemsetAsync(ws + sg.status_off, 0, sg.ntasks_total * 4, s);
         cudaMemsetAsync(ws + sg.counter_off, 0, 128, s);
-        sg.ticket_base = 0;
-        sg.epoch = 0;
     }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return fail(BDL_ECUDA, std::string("bdl_plan_prepare: ") + cudaGetErrorString(e));
@@ -81,7 +79,6 @@ bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void
     unsigned char *ws = (unsigned char *)workspace;
     cudaStream_t s = (cudaStream_t)stream;
     Subgraph &sg = p->sgs[i];
-    sg.epoch++;
     const Tensor &tin = p->tensors[sg.in_tensor];
     const Tensor &tout = p->tensors[sg.out_tensor];
     TView vin = make_view(tin.layout, tensor_ptr(p, sg.in_tensor, in_bricked, out_bricked, ws));
@@ -96,12 +93,17 @@ bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void
     }
     int launches = 0;
     const int kern = effective_kernel(sg);
-    if (kern == KERNEL_TC_GEN) return launch_gen_subgraph(p, sg, vin, vout, res, ws, s, &launches);
+    if (kern == KERNEL_TC_GEN) {
+        std::vector<TView> srcv(sg.last - sg.first + 1);   // external inputs per layer (graph branches)
+        for (size_t j = 0; j < srcv.size(); j++) {
+            const int t = sg.src_tensor[j];
+            if (t >= 0) srcv[j] = make_view(p->tensors[t].layout, tensor_ptr(p, t, in_bricked, out_bricked, ws));
+        }
+        return launch_gen_subgraph(p, sg, srcv, vout, res, ws, s, &launches);
+    }
     if (kern == KERNEL_TC_BAND) {
         const bool single = sg.first == sg.last;
         if (sg.mode == BDL_MODE_PADDED && !single) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
-        static const bool legacy = getenv("BDL_TC_LEGACY") != nullptr;  // A/B against the synchronous kernel
-        if (legacy) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
         return launch_ws_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches,
                                   sg.mode == BDL_MODE_UNMERGED || single);
     }

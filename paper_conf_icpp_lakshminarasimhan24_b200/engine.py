@@ -213,6 +213,12 @@ class HostPipeline:
         on_output(k, y_host) (y_host is valid until the callback returns; its slot is then reused), or, with
         on_output=None, returns the list of output copies.  Returns when everything is done."""
         n, S = len(inputs), self.slots
+        # the plan's weight packing / memo-table reset (bdl_plan_prepare) and any caller work were queued on the
+        # caller's current stream: every pipeline stream starts after them.  A plan's workspace is used by one
+        # stream at a time (its memo tables and run state are shared), so the merged runs stay on s_cmp.
+        cur = torch.cuda.current_stream(self.plan.device)
+        for st in (self.s_h2d, self.s_cmp, self.s_d2h):
+            st.wait_stream(cur)
         h2d_done = [torch.cuda.Event() for _ in range(S)]
         x_free = [torch.cuda.Event() for _ in range(S)]
         cmp_done = [torch.cuda.Event() for _ in range(S)]

@@ -22,7 +22,25 @@ def rel_err(y, ref):
 
 
 C3 = dict(nsp=3)
+
+
+def bottlenecks(cin, width, stride):
+    """ResNet-50 bottleneck with a projection shortcut followed by an identity bottleneck (§4.3):
+    layers read non-previous layers and add residuals produced inside the subgraph (a DAG subgraph)."""
+    return [
+        W.conv(cin, width, 1, inp=-1),                                   # 0
+        W.conv(width, width, 3, stride),                                 # 1
+        W.conv(cin, 4 * width, 1, stride, 0, relu=False, inp=-1),        # 2 projection of the block input
+        W.conv(width, 4 * width, 1, inp=1, res=2, wscale=0.5),           # 3 + projection
+        W.conv(4 * width, width, 1),                                     # 4
+        W.conv(width, width, 3),                                         # 5
+        W.conv(width, 4 * width, 1, res=3, wscale=0.5),                  # 6 + block 1 output
+    ]
+
+
 GRAPHS = {
+    "dag_bottlenecks_s1": (bottlenecks(64, 64, 1), 2, 64, 1, 16, 16, (1, 1, 8, 8)),
+    "dag_bottlenecks_s2": (bottlenecks(256, 128, 2), 2, 256, 1, 18, 14, (1, 1, 8, 8)),
     # name: (layers, N, C, D, H, W, brick)
     "pair_s1_vgg_conv1": ([W.conv(3, 64, 3)], 2, 3, 1, 20, 20, (1, 1, 8, 8)),
     "pair_s2_k7_stem": ([W.conv(3, 64, 7, 2, 3)], 2, 3, 1, 38, 38, (1, 1, 8, 8)),
@@ -106,3 +124,62 @@ def test_gen_repeat_and_masking():
     v = first.view(torch.bfloat16).view(2, 2, 2, 8, 8, 64).float()   # [n][by][bx][y][x][c]
     full = v.permute(0, 1, 3, 2, 4, 5).reshape(2, 16, 16, 64)
     assert float(full[:, 13:].abs().max()) == 0.0 and float(full[:, :, 11:].abs().max()) == 0.0
+
+
+def test_dag_subgraph_schedule_invariance():
+    """A bottleneck DAG (projection + identity block) as ONE merged memoized subgraph: any task order gives
+    bit-identical results with every task computed exactly once (computed == successful claims: 2 compulsory
+    atomics per task, L1147-1149; merged execution only reorders work, L363-365).  Seeds select random
+    topological orders; seed 0 is the locality-aware wavefront."""
+    layers, N, C, D, H, Wd, brick = GRAPHS["dag_bottlenecks_s1"]
+    wl = W.make_graph_workload(layers, N, C, D, H, Wd, 2, brick, "bf16", seed=17)
+    ref = oracle.run_graph(wl["layers"], wl["x"].numpy(), wl["weights"], wl["biases"], dtype="bf16")
+    y0, n0 = None, None
+    for seed in (0, 1, 7, 123):
+        plan = engine.plan_from_workload(wl, force_mode=2, schedule_seed=seed)
+        sgs = plan.subgraphs()
+        assert len(sgs) == 1 and sgs[0]["mode"] == "memoized" and sgs[0]["kernel"] == "tcgen05 generic", sgs
+        y = plan.forward(wl["x"]).float().cpu().numpy()
+        c = plan.counters(0)
+        assert c["computed"] == c["cas_ok"] and c["computed"] > 0, (seed, c)
+        if y0 is None:
+            y0, n0 = y, c["computed"]
+            assert rel_err(y, ref) <= TOL
+        else:
+            np.testing.assert_array_equal(y, y0)
+            assert c["computed"] == n0
+    plan.set_mode("unmerged")
+    np.testing.assert_array_equal(plan.forward(wl["x"]).float().cpu().numpy(), y0)
+
+
+@pytest.mark.parametrize("which", ["band_cfg2", "gen_dag"])
+def test_cuda_graph_replay(which):
+    """The per-run memo state (ticket counter, tag epoch) lives on the device, so a captured bdl_run replays
+    correctly: each replay recomputes from its current input."""
+    import torch
+    if which == "band_cfg2":
+        wl = W.make_workload("cfg2", N=2, H=24, W=24)
+    else:
+        layers, N, C, D, H, Wd, brick = GRAPHS["dag_bottlenecks_s1"]
+        wl = W.make_graph_workload(layers, N, C, D, H, Wd, 2, brick, "bf16", seed=19)
+    plan = engine.plan_from_workload(wl, force_mode=2)
+    xs = [wl["x"], (wl["x"] * -0.5).to(torch.bfloat16).float(), (wl["x"] + 0.25).to(torch.bfloat16).float()]
+    refs = [plan.forward(x).clone() for x in xs]
+    xb = plan.brickify(xs[0])
+    yb = plan.alloc_bricked(plan.out_layout)
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        plan.run(xb, yb)
+    torch.cuda.current_stream().wait_stream(s)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        plan.run(xb, yb)
+    for rep in range(2):
+        for x, ref in zip(xs, refs):
+            plan.brickify(x, out=xb)
+            g.replay()
+            y = plan.unbrickify(yb)
+            torch.cuda.synchronize()
+            assert torch.equal(y, ref), (which, rep)

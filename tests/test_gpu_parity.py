@@ -238,3 +238,25 @@ def test_full_resolution_single_image(cfg):
     plan = engine.plan_from_workload(wl)
     y = plan.forward(wl["x"]).float().cpu().numpy()
     assert rel_err(y, ref) <= TOL["bf16"]
+
+
+@pytest.mark.parametrize("cfg", ["cfg3", "cfg4"])
+def test_full_batch_sampled(cfg):
+    """VGG-16 at N=128 / ResNet-50 at N=256: the bench's batch sizes and launch configuration (several
+    image groups in the generic kernel's task order, padded CTA blocks grown to whole-image bands).
+    Images 0 and N-1 are checked against the oracle element by element, and bit for bit against a
+    one-image plan of the same graph (merged execution only reorders work, L363-365; one K-order
+    per element in every geometry and mode)."""
+    wl = workloads.make_workload(cfg)
+    N = wl["N"]
+    plan = engine.plan_from_workload(wl)
+    y = plan.forward(wl["x"]).float().cpu().numpy()
+    del plan
+    torch.cuda.empty_cache()
+    ref = oracle_out(wl, images=[0, N - 1])
+    assert rel_err(y[[0, N - 1]], ref) <= TOL["bf16"], rel_err(y[[0, N - 1]], ref)
+    one = workloads.make_workload(cfg, N=1)
+    p1 = engine.plan_from_workload(one)
+    for n in (0, N - 1):
+        y1 = p1.forward(wl["x"][n:n + 1]).float().cpu().numpy()
+        np.testing.assert_array_equal(y[n:n + 1], y1)

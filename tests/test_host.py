@@ -173,25 +173,49 @@ def test_tiny_layer_rule_unmerged():
 
 @pytest.mark.parametrize("cfg", ["cfg3", "cfg4"])
 def test_partition_invariants(cfg):
+    """Reverse-traversal partition (L603-626): subgraphs tile the layer list, pools end subgraphs, every layer
+    reads a layer of its own subgraph or a materialized earlier one, and branched subgraphs (projection
+    shortcuts, residuals produced inside, inner live-outs) run memoized on the generic tcgen05 kernel."""
     p = _plan(cfg, N=2)
     L = workloads.make_layers(cfg)
     sgs = p.subgraphs()
     covered = []
     for sg in sgs:
-        covered += list(range(sg["first"], sg["last"] + 1))
-        for j in range(sg["first"] + 1, sg["last"] + 1):
-            assert L[j]["input"] == j - 1                   # a chain
-            assert L[j - 1]["kind"] != "maxpool"            # pools end subgraphs (L620-626)
+        f, e = sg["first"], sg["last"]
+        covered += list(range(f, e + 1))
+        assert e - f + 1 <= 16
+        branched = False
+        for j in range(f, e + 1):
+            if j < e:
+                assert L[j]["kind"] != "maxpool"            # pools end subgraphs (L620-626)
+            assert L[j]["input"] < j                         # producers come first (topological listing)
             r = L[j]["residual"]
-            assert r is None or r < sg["first"]            # residual sources are materialized
-        for j in range(sg["first"], sg["last"]):
-            for m in range(sg["last"] + 1, len(L)):        # no live-out inside a subgraph
-                assert L[m]["input"] != j and L[m]["residual"] != j
+            branched |= (j > f and L[j]["input"] != j - 1) or (r is not None and r >= f)
+            branched |= j < e and any(L[m]["input"] == j or L[m]["residual"] == j for m in range(e + 1, len(L)))
+        if branched:
+            assert sg["mode"] in ("memoized", "unmerged") and sg["kernel"] == "tcgen05 generic"
     assert covered == list(range(len(L)))
     if cfg == "cfg3":
         pools = [i for i, l in enumerate(L) if l["kind"] == "maxpool"]
         ends = {sg["last"] for sg in sgs}
         assert all(pi in ends for pi in pools)
+        assert all(sg["first"] < sg["last"] for sg in sgs)   # no pool-only subgraph
+    if cfg == "cfg4":
+        # the paper splits ResNet-50 into 7 merged subgraphs (L1130-1165); we allow branches inside subgraphs,
+        # so no projection or pool runs alone
+        assert len(sgs) <= 10
+        assert all(sg["first"] < sg["last"] for sg in sgs)
+
+
+def test_partition_chain_only_for_cuda_core_path():
+    """fp32 graphs run on the CUDA-core brick kernels, which merge chains only: branches cut subgraphs."""
+    L = workloads.make_layers("cfg4")[:9]
+    p = engine.Plan(L, None, None, 1, 3, 1, 64, 64, 2, "f32", (1, 1, 8, 8), device=None)
+    for sg in p.subgraphs():
+        for j in range(sg["first"] + 1, sg["last"] + 1):
+            assert L[j]["input"] == j - 1
+            r = L[j]["residual"]
+            assert r is None or r < sg["first"]
 
 
 def test_plan_opts_force_mode_and_budget():

@@ -291,3 +291,61 @@ def test_workload_recipe_is_seeded_and_bf16_representable():
     L = workloads.make_layers("cfg4")
     assert sum(l["kind"] == "conv" for l in L) == 53
     assert sum(l["kind"] == "maxpool" for l in workloads.make_layers("cfg3")) == 5
+
+
+# ---------------------------------------------------------------- P6 on the branched (DAG) path
+def _resnet50_prefix_torch(x, w, b):
+    """ResNet-50 v1.5 prefix written out by hand with torch fp64 (no layer indices involved): stem
+    conv7x7/2 + ReLU, maxpool 3x3/2 p1, conv2_x block 1 (projection shortcut), conv2_x blocks 2 and 3
+    (identity shortcuts), conv3_x block 1 (stride 2 on the 3x3 and on the projection).  Epilogue
+    order bias -> residual add -> ReLU.  w/b are consumed in the listed order."""
+    F = torch.nn.functional
+    it = iter(zip(w, b))
+
+    def conv(h, s=1, p=0, relu=True):
+        wi, bi = next(it)
+        y = F.conv2d(h, wi, bi, stride=s, padding=p)
+        return torch.relu(y) if relu else y
+
+    h = conv(x, s=2, p=3)
+    next(it)                                   # the pool has no weights
+    h = F.max_pool2d(h, 3, 2, 1)
+    for stage_stride, nblocks in ((1, 3), (2, 1)):
+        for blk in range(nblocks):
+            s = stage_stride if blk == 0 else 1
+            a = conv(h)
+            a = conv(a, s=s, p=1)
+            if blk == 0:
+                proj = conv(h, s=s, relu=False)
+                wi, bi = next(it)
+                h = torch.relu(F.conv2d(a, wi, bi) + proj)
+            else:
+                wi, bi = next(it)
+                h = torch.relu(F.conv2d(a, wi, bi) + h)
+    return h
+
+
+def test_p6_dag_resnet50_prefix_vs_torch():
+    """Pins run_graph's branch semantics (a layer reading a non-previous layer; a residual taken from
+    a layer OUTPUT, the projection) and make_layers('cfg4')'s input/residual indices: the first 16
+    layers of the cfg4 graph against the hand-written torch fp64 forward (§4.3 ResNet-50,
+    L1130-1165; merged execution reproduces exactly this layer-by-layer result, L363-365)."""
+    layers = workloads.make_layers("cfg4")[:16]
+    assert [l["kind"] for l in layers].count("maxpool") == 1
+    wl = workloads.make_graph_workload(layers, 2, 3, 1, 40, 36, 2, (1, 1, 8, 8), "f64", seed=41)
+    y = oracle.run_graph(wl["layers"], wl["x"].numpy(), wl["weights"], wl["biases"], dtype="f64")
+    ws = [t.double()[:, :, 0] for t in wl["weights"] if t is not None]
+    bs = [t.double() for t in wl["biases"] if t is not None]
+    ws.insert(1, None)
+    bs.insert(1, None)
+    ref = _resnet50_prefix_torch(wl["x"].double()[:, :, 0], ws, bs)
+    assert y.shape[1:] == (512, 1, 5, 5)
+    np.testing.assert_allclose(y[:, :, 0], ref.numpy(), rtol=1e-12, atol=1e-12)
+    # the pin discriminates: block 2 adding the projection output (layer 4) instead of block 1's output
+    # (layer 5) -- same shape, wrong index -- must fail it
+    assert wl["layers"][8]["residual"] == 5 and wl["layers"][5]["residual"] == 4
+    bad = [dict(l) for l in wl["layers"]]
+    bad[8]["residual"] = 4
+    with pytest.raises(AssertionError):
+        yb = oracle.run_graph(bad, wl["x"].numpy(), wl["weights"], wl["biases"], dtype="f64")
+        np.testing.assert_allclose(yb[:, :, 0], ref.numpy(), rtol=1e-12, atol=1e-12)

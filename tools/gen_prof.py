@@ -7,7 +7,8 @@ import numpy as np, torch
 from paper_conf_icpp_lakshminarasimhan24_b200 import engine, workloads, lib
 cfg = sys.argv[1]
 wl = workloads.make_workload(cfg)
-plan = engine.plan_from_workload(wl)
+ml = int(os.environ.get("MAXL", "0"))
+plan = engine.plan_from_workload(wl, max_subgraph_layers=ml) if ml else engine.plan_from_workload(wl)
 xb = plan.brickify(wl["x"]); yb = plan.alloc_bricked(plan.out_layout)
 plan.run(xb, yb); torch.cuda.synchronize()
 sgs = plan.subgraphs()
