@@ -38,6 +38,9 @@ def parse():
     ap.add_argument("--mode", default="auto")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cudnn", action="store_true")
+    ap.add_argument("--no-extra", action="store_true",
+                    help="skip the other configurations (cfg3/cfg4/cfg5 and cfg2 padded) measured in the default run")
+    ap.add_argument("--micro", type=int, default=2, help="strong scaling: micro-batches per rank for the gather overlap")
     ap.add_argument("--spatial", action="store_true",
                     help="3-D configs: shard ONE volume into depth slabs with a brick-plane halo exchange "
                          "(default for 3-D configs when WORLD_SIZE > 1)")
@@ -73,6 +76,102 @@ def useful_flops(wl):
             f += 2 * wl["N"] * Do * Ho * Wo * l["cout"] * l["cin"] * kd * kh * kw
         shapes[i] = (Do, Ho, Wo)
     return f
+
+
+def subgraph_roofline(wl, sgs, peak_tflops, hbm_gbs):
+    """t_roof = sum over subgraphs of max(F_s / P_tensor, Bytes_s / HBM).  F_s = useful conv FLOPs
+    (2*MACs of layer-by-layer execution; padded recompute not credited); Bytes_s = algorithmic merged bytes: every
+    tensor the subgraph reads from outside (its input, external residuals / branch inputs) once, every tensor it
+    leaves for later subgraphs (its output, inner live-outs) once, its weights once (bf16 storage)."""
+    from paper_conf_icpp_lakshminarasimhan24_b200 import workloads
+    L = wl["layers"]
+    esz = 2 if wl["dtype"] == "bf16" else 4
+    shapes = {-1: (wl["D"], wl["H"], wl["W"])}
+    chans = {-1: wl["C"]}
+    flops = []
+    for i, l in enumerate(L):
+        D, H, W = shapes[l["input"]]
+        o = workloads.layer_out_shape(l, D, H, W)
+        shapes[i], chans[i] = o, l["cout"]
+        flops.append(2 * wl["N"] * o[0] * o[1] * o[2] * l["cout"] * l["cin"] * l["k"][0] * l["k"][1] * l["k"][2]
+                     if l["kind"] == "conv" else 0)
+    tb = lambda m: wl["N"] * chans[m] * shapes[m][0] * shapes[m][1] * shapes[m][2] * esz   # noqa: E731
+    t_roof, per = 0.0, []
+    for s in sgs:
+        f, e = s["first"], s["last"]
+        reads = set()
+        for j in range(f, e + 1):
+            for m in (L[j]["input"], L[j]["residual"]):
+                if m is not None and m < f:
+                    reads.add(m)
+        writes = {e} | {j for j in range(f, e) if any(L[m]["input"] == j or L[m]["residual"] == j
+                                                      for m in range(e + 1, len(L)))}
+        wbytes = sum(L[j]["cout"] * L[j]["cin"] * L[j]["k"][0] * L[j]["k"][1] * L[j]["k"][2] * esz
+                     for j in range(f, e + 1) if L[j]["kind"] == "conv")
+        F = sum(flops[f:e + 1])
+        B = sum(tb(m) for m in reads) + sum(tb(m) for m in writes) + wbytes
+        t = max(F / (peak_tflops * 1e12), B / (hbm_gbs * 1e9))
+        t_roof += t
+        per.append({"layers": [f, e], "gflop": F / 1e9, "mbytes": B / 1e6, "t_roof_ms": t * 1e3})
+    return t_roof * 1e3, per
+
+
+def measure_config(cfg, dev, K, flush, peaks, mode=None, cudnn=True):
+    """One more configuration measured in the same run (same contract as the headline: K steps of brickify +
+    merged subgraphs + unbrickify with inputs resident in HBM, L2 flushed between steps, events around each step;
+    a second pass with events around each subgraph for the per-subgraph times)."""
+    import torch
+    from paper_conf_icpp_lakshminarasimhan24_b200 import engine, workloads
+    wl = workloads.make_workload(cfg)
+    plan = engine.plan_from_workload(wl, device=dev)
+    if mode:
+        plan.set_mode(mode)
+    sgs = plan.subgraphs()
+    x = wl["x"].to(device=dev, dtype=plan.tdtype).contiguous()
+    xb = plan.alloc_bricked(plan.in_layout)
+    yb = plan.alloc_bricked(plan.out_layout)
+    lo = plan.out_layout
+    y = torch.empty((lo.N, lo.C, lo.D, lo.H, lo.W), dtype=plan.tdtype, device=dev)
+    for _ in range(3):
+        plan.forward_into(x, y)
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    for a, b in ev:
+        flush()
+        a.record()
+        plan.brickify(x, out=xb)
+        plan.run(xb, yb)
+        plan.unbrickify(yb, out=y)
+        b.record()
+    torch.cuda.synchronize()
+    step_ms = statistics.mean(a.elapsed_time(b) for a, b in ev)
+    sev = [[torch.cuda.Event(enable_timing=True) for _ in range(len(sgs) + 1)] for _ in range(K)]
+    for e in sev:
+        flush()
+        plan.brickify(x, out=xb)
+        e[0].record()
+        for i in range(len(sgs)):
+            plan.run_subgraph(i, xb, yb)
+            e[i + 1].record()
+    torch.cuda.synchronize()
+    sub_ms = [statistics.median(e[i].elapsed_time(e[i + 1]) for e in sev) for i in range(len(sgs))]
+    peak = float(peaks["bf16_tflops"]) if wl["dtype"] == "bf16" else None
+    out = {"workload": workload_desc(wl), "mode": "/".join(sorted({g["mode"] for g in sgs})),
+           "subgraphs": len(sgs), "ms_per_step": step_ms, "images_per_s": wl["N"] / (step_ms / 1e3),
+           "merged_ms": sum(sub_ms), "gpu_launches_per_step": 2 + plan.launches_per_run}
+    if peak:
+        flops = useful_flops(wl)
+        t_roof, per = subgraph_roofline(wl, sgs, peak, float(peaks["hbm_gbs"]))
+        out["roofline"] = {"t_roof_ms": t_roof, "frac_merged": t_roof / sum(sub_ms), "frac_step": t_roof / step_ms,
+                           "useful_tflops_merged": flops / (sum(sub_ms) / 1e3) / 1e12, "peak_tflops": peak,
+                           "how": "t_roof = sum_s max(F_s/P_bf16, Bytes_s/HBM) (SURVEY 8(d)); frac = t_roof / measured"}
+        out["per_subgraph"] = [dict(p, ms=m, mode=g["mode"], kernel=g["kernel"])
+                               for p, m, g in zip(per, sub_ms, sgs)]
+    if cudnn:
+        out["cudnn_layer_by_layer"] = cudnn_lbl(wl, dev, K, flush)
+    del plan, xb, yb, x, y
+    torch.cuda.empty_cache()
+    return out
 
 
 # ------------------------------------------------------------------------------------------ clocks
@@ -204,6 +303,8 @@ def main():
 
     if workloads.CONFIGS[args.config]["nsp"] == 3 and (world > 1 or args.spatial):
         return bench_spatial(args, world, rank, local, dev)
+    if args.config == "cfg4" and world > 1:
+        return bench_strong(args, world, rank, local, dev)
     wl = workloads.make_workload(args.config, input_seed_offset=rank)
     plan = engine.plan_from_workload(wl, device=dev)
     if args.mode != "auto":
@@ -322,12 +423,14 @@ def main():
     peaks, peak_src = load_peaks()
     flops = useful_flops(wl)
     kernel_ms = statistics.mean(run_ms)
-    traffic = None
+    traffic, traffic_src = None, None
     tp = os.path.join(ROOT, "profiles", "ncu_summary_latest.json")
     if os.path.exists(tp):
         try:
             with open(tp) as f:
                 traffic = json.load(f).get("dram_bytes_per_launch", {}).get(sg[0]["kernel"])
+            traffic_src = ("file lookup, not measured in this run: dram__bytes_read.sum + dram__bytes_write.sum of one "
+                           "launch from the committed ncu --set full capture summarised in profiles/ncu_summary_latest.json")
         except Exception:
             traffic = None
     kinds = {g["kernel"] for g in sg}
@@ -341,7 +444,7 @@ def main():
     achieved = flops / (kernel_ms / 1e3) / 1e12
     kname = sg[0]["kernel"] if len(sg) == 1 else f"{len(sg)} subgraph launches ({', '.join(sorted(kinds))})"
     roofline = {"bound": bound, "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
-                "traffic": traffic if len(sg) == 1 else None, "peak_source": peak_src,
+                "traffic": traffic if len(sg) == 1 else None, "traffic_source": traffic_src, "peak_source": peak_src,
                 "kernel": f"{kname} ({'/'.join(sorted({g['mode'] for g in sg}))})",
                 "algorithmic_flops_per_launch": flops, "kernel_ms_mean": kernel_ms, "hbm_frac_of_step_bytes": None}
     # step bytes: brickify (read+write) + subgraphs (in, out) + unbrickify (read+write)
@@ -358,6 +461,21 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(wl)
+
+    # ---- the other configurations, in the same run (driver-observed): cfg2 padded mode, cfg3, cfg4, cfg5
+    extra = None
+    if rank == 0 and world == 1 and not args.no_extra and args.config == "cfg2" and args.mode == "auto":
+        extra = {}
+        del xb, yb
+        torch.cuda.empty_cache()
+        Ke = max(3, min(K, 10))
+        for name, cfg, mode in (("cfg2_padded", "cfg2", "padded"), ("cfg3", "cfg3", None), ("cfg4", "cfg4", None),
+                                ("cfg5", "cfg5", None)):
+            try:
+                extra[name] = measure_config(cfg, dev, Ke, flush_l2, load_peaks()[0], mode=mode,
+                                             cudnn=not args.no_cudnn and name != "cfg2_padded")
+            except Exception as e:   # report, do not hide: the headline line still prints
+                extra[name] = {"error": f"{type(e).__name__}: {str(e)[:300]}"}
 
     if rank == 0:
         launches = K * (2 + plan.launches_per_run)
@@ -389,6 +507,7 @@ def main():
                              "unbrickify": statistics.mean(e[2].elapsed_time(e[3]) for e in ev),
                              "step_with_events_between_kernels": statistics.mean(e[0].elapsed_time(e[3]) for e in ev)},
             "cudnn_layer_by_layer": cudnn,
+            "other_configs": extra,
         }
         print(json.dumps(line))
     if world > 1:
@@ -512,6 +631,72 @@ def bench_spatial(args, world, rank, local, dev):
         print(json.dumps(line))
     if world > 1:
         dist.destroy_process_group()
+    return 0
+
+
+def bench_strong(args, world, rank, local, dev):
+    """Strong scaling: the global batch of 256 images is split over the ranks in
+    micro-batches; each rank runs brickify + merged subgraphs + unbrickify per micro-batch and all-gathers the
+    outputs over NCCL on a communication stream while its next micro-batch computes (parallel.BatchRunner).  value =
+    global images / max-over-ranks step time with the gather; sharded_value = the same with outputs left sharded."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_lakshminarasimhan24_b200 import engine, parallel, workloads
+    full = workloads.make_workload(args.config)
+    n_total = full["N"]
+    mb, ranges = parallel.micro_batches(n_total, world, args.micro)
+    wl = workloads.make_workload(args.config, N=mb)
+    plan = engine.plan_from_workload(wl, device=dev)
+    if args.mode != "auto":
+        plan.set_mode(args.mode)
+    lo = plan.out_layout
+    run = parallel.BatchRunner(n_total, (lo.C, lo.D, lo.H, lo.W), rank, world, micro=args.micro, plan=plan, device=dev)
+    x_local = full["x"][run.global_images()].to(device=dev, dtype=plan.tdtype).contiguous()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    for _ in range(max(3, args.warmup)):
+        run.forward(x_local)
+    torch.cuda.synchronize()
+    K = args.steps
+    res = {}
+    with ClockSampler(local) as clk:
+        for gather in (True, False):
+            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+            dist.barrier()
+            torch.cuda.synchronize()
+            for a, b in ev:
+                flush.zero_()
+                a.record()
+                run.forward(x_local, gather=gather)
+                b.record()
+            torch.cuda.synchronize()
+            dist.barrier()
+            t = torch.tensor([sum(a.elapsed_time(b) for a, b in ev)], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            res[gather] = float(t.item())
+    # correctness of the gathered batch: this rank's own images equal its local results
+    y = run.forward(x_local)
+    mine = y[run.global_images()]
+    ok = bool(torch.equal(mine, run.forward(x_local, gather=False)))
+    peaks, peak_src = load_peaks()
+    if rank == 0:
+        line = {
+            "metric": "images/sec merged conv chain per B200", "value": n_total * K / (res[True] / 1e3),
+            "unit": "images/s", "n_gpus": world, "steps": K, "warmup": max(3, args.warmup),
+            "ms_per_step": res[True] / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": wl["dtype"], "data": "synthetic (seeded N(0,1) inputs, He-normal weights; workloads.py)",
+            "config": {"workload": workload_desc(full), "global_batch": n_total, "images_per_gpu": n_total // world,
+                       "micro_batches": args.micro, "micro_batch": mb,
+                       "parallelism": f"batch-sharded x{world}, outputs all-gathered (NCCL all_gather_into_tensor on a "
+                                      f"comm stream, overlapped with the next micro-batch)",
+                       "l2": "flushed between timed steps (256 MiB write, outside the events)"},
+            "sharded_value": n_total * K / (res[False] / 1e3),
+            "gather_check": ok,
+            "clocks": clk.summary(),
+            "gpu_launches": K * args.micro * (2 + plan.launches_per_run),
+        }
+        print(json.dumps(line))
+    dist.destroy_process_group()
     return 0
 
 

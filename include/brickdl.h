@@ -106,7 +106,13 @@ typedef struct bdl_plan_opts {
     int32_t max_subgraph_layers; /* 0 = unlimited */
     int32_t num_sms;             /* 0 = query the device */
     int32_t schedule_seed;       /* 0 = locality-aware wavefront task order; else a seeded random
-                                    permutation of the memo tasks (schedule-invariance testing) */
+                                    topological order of the memo tasks (schedule-invariance testing) */
+    int32_t memo_defer;          /* generic kernel, memoized: 1 = a claimed task whose dependency is in progress
+                                    elsewhere is set aside and revisited ("moves on ... revisits later", L523-525);
+                                    0 = it is handed to the CTA's in-order pipeline, which waits (default: measured
+                                    faster on B200) */
+    int32_t group_waves;         /* generic kernel, memoized: images per task-order group sized so the group's first
+                                    layer holds this many waves of tasks (0 = default 8) */
 } bdl_plan_opts;
 
 typedef struct bdl_plan bdl_plan;  /* opaque, library-owned host object */

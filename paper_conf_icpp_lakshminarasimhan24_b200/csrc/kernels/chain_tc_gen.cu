@@ -24,6 +24,7 @@
 //                then release-publish the tile (state 2)
 #include <algorithm>
 #include <cstdio>
+#include <cmath>
 #include <random>
 #include <cstdlib>
 #include <cstring>
@@ -44,6 +45,7 @@ constexpr int kSched = 0, kLoad0 = 1, kLW = 4, kWProd = 5, kMma = 6, kEpi0 = 7, 
 constexpr int kThreads = 32 * (kEpi0 + kEpiW);
 constexpr int kLoadT = 32 * kLW;
 constexpr int kQ = 4, kRing = 16, kStack = 128;
+constexpr int kPendDraw = 32, kPend = kPendDraw + kStack;   // pending (deferred) tasks: draw tickets below kPendDraw
 constexpr int kMaxIn = 4, kMaxW = 4, kMaxKs = 128;   // k-steps per layer: 3x3x3 taps x 64 channels = 108
 constexpr int kTaskBits = 26;   // order entry = (layer << kTaskBits) | task
 
@@ -85,6 +87,7 @@ struct Params {
     int nin, nw, in_stride, w_stride;    // ring depths and slot strides (bytes)
     int nacc, acc_stride, tmem_cols;
     int *status;
+    int defer;                           // bdl_plan_opts.memo_defer: 1 = hand over only ready tasks (revisit the others)
     unsigned long long *counters;        // run state (common.cuh run_epoch / run_exit)
     const int *order;                    // (l << 26) | task, or null (unmerged)
     long long norder;
@@ -114,6 +117,8 @@ struct Shared {
     long long desc_t[kRing];
     int stk_l[kStack];
     long long stk_t[kStack];
+    int pend_l[kPend];
+    long long pend_t[kPend];
     uint32_t ks[kMaxLayers][kMaxKs];     // per k-step: A offset | LBO << 16 (both in 16-B units, < 2^14)
 };
 
@@ -130,7 +135,7 @@ __device__ __forceinline__ void pwait(const Params &p, uint64_t *bar, uint32_t p
         ptx::mbar_wait(bar, parity);
     }
 }
-__device__ __forceinline__ int tag_state(int v, unsigned EP) { return ((v & ~3) == (int)EP) ? (v & 3) : 0; }
+__device__ __forceinline__ int tag_state(int v, unsigned EP) { return ((v & ~1023) == (int)EP) ? (v & 3) : 0; }
 __device__ __forceinline__ int *status_word(const Params &p, int l, long long t) {
     return p.status + p.layer[l].task_base + t;
 }
@@ -382,17 +387,27 @@ __device__ void scheduler_padded(const Params &p, Shared &sh) {
     (void)computed;
 }
 
+// Memoized scheduler (§3.2.2, Fig 2d), one warp.  Tickets are drawn along the host-built order
+// (gen_task_order); a ticket's task is claimed with CAS 0 -> 1, its not-started dependencies are claimed
+// recursively (the walk back of Fig 2d), and the bundle is handed to the loaders producers-first (layer order).
+// A task is handed over only when it is READY: every dependency is published (state 2) or was handed over by this
+// CTA earlier (state 3, ours; it completes ahead of the dependent in this CTA's in-order pipeline).  A claimed task
+// whose dependency is still in progress on another CTA is not waited for: it goes to a pending list and is
+// revisited later ("moves on ... and revisits this brick later", L523-525), so one slow tile never blocks the
+// CTA's pipeline.  Progress: the lowest-layer pending task of all CTAs only depends on handed-over tasks.
+// Tag word: (epoch << 10) | (owner CTA << 2) | state, state 0 free, 1 claimed, 3 claimed + handed over, 2 done.
 __device__ void scheduler(const Params &p, Shared &sh) {
     const int lane = threadIdx.x % 32;
-    const unsigned EP = run_epoch(p.counters) << 2;
+    const unsigned EP = run_epoch(p.counters) << 10;
+    const int MINE1 = (int)(EP | (blockIdx.x << 2) | 1), MINE3 = (int)(EP | (blockIdx.x << 2) | 3);
     const bool unmerged = p.only_layer >= 0;
-    unsigned long long oks = 0, fails = 0;
-    int sp = 0;
+    unsigned long long oks = 0, defers = 0;
     uint32_t qseq = 0;
     auto emit = [&](int l, long long t) {
         const int slot = qseq % kQ;
         if (qseq >= (uint32_t)kQ) ptx::mbar_wait(&sh.q_empty[slot], ((qseq / kQ) - 1) & 1);
         if (lane == 0) {
+            if (l >= 0 && !unmerged) atomicExch(status_word(p, l, t), MINE3);   // handed over (before any publish)
             sh.q_l[slot] = l;
             sh.q_t[slot] = t;
             sh.q_w[slot] = -1;
@@ -401,80 +416,142 @@ __device__ void scheduler(const Params &p, Shared &sh) {
         __syncwarp();
         qseq++;
     };
+    if (unmerged) {
+        for (;;) {
+            unsigned long long tk = 0;
+            if (lane == 0) tk = atomicAdd(&p.counters[4], 1ULL);
+            tk = __shfl_sync(0xffffffff, tk, 0);
+            if ((long long)tk >= p.norder) break;
+            emit(p.only_layer, (long long)tk);
+        }
+        emit(-1, 0);
+        return;
+    }
+    // every dependency published, or handed over by this CTA
+    auto ready = [&](int l, long long t) {
+        const Deps D = deps_of(p.layer, l, t);
+        const int nd = D.ns + D.nr;
+        bool ok = true;
+        for (int i0 = 0; i0 < nd; i0 += 32) {
+            const int i = i0 + lane;
+            bool mine = true;
+            if (i < nd) {
+                int dl;
+                const long long dt = dep_at(p.layer, D, i, dl);
+                const int v = ld_acquire(status_word(p, dl, dt));
+                mine = tag_state(v, EP) == 2 || v == MINE3;
+            }
+            ok = __all_sync(0xffffffff, mine) && ok;
+        }
+        return ok;
+    };
+    int np = 0;                  // pending (claimed, not handed over) tasks: sh.pend_l / sh.pend_t [0, np)
+    bool tickets = true;
+    unsigned sleep_ns = 32;
     for (;;) {
+        // revisit the pending tasks (in claim order)
+        if (np > 0) {
+            int w = 0;
+            for (int i = 0; i < np; i++) {
+                const int l = sh.pend_l[i];
+                const long long t = sh.pend_t[i];
+                __syncwarp();
+                if (ready(l, t)) {
+                    emit(l, t);
+                } else {
+                    if (lane == 0) {
+                        sh.pend_l[w] = l;
+                        sh.pend_t[w] = t;
+                    }
+                    w++;
+                }
+                __syncwarp();
+            }
+            np = w;
+        }
+        if (!tickets || np >= kPendDraw) {
+            if (!tickets && np == 0) break;
+            __nanosleep(sleep_ns);            // everything pending waits on other CTAs: back off
+            sleep_ns = min(sleep_ns * 2, 1024u);
+            continue;
+        }
+        sleep_ns = 32;
         unsigned long long tk = 0;
         if (lane == 0) tk = atomicAdd(&p.counters[4], 1ULL);
         tk = __shfl_sync(0xffffffff, tk, 0);
-        if ((long long)tk >= p.norder) break;
-        int l;
-        long long t;
-        if (unmerged) {
-            l = p.only_layer;
-            t = (long long)tk;
-        } else {
-            const int e = p.order[tk];
-            l = e >> kTaskBits;
-            t = e & ((1 << kTaskBits) - 1);
-            int ok = 0;
-            if (lane == 0) {
-                int *sw = status_word(p, l, t);
-                const int cur = ld_acquire(sw);
-                ok = tag_state(cur, EP) == 0 && atomicCAS(sw, cur, (int)(EP | 1)) == cur;
-            }
-            ok = __shfl_sync(0xffffffff, ok, 0);
-            if (!ok) continue;   // already claimed (by a dependent's recursion)
-            oks++;
+        if ((long long)tk >= p.norder) {
+            tickets = false;
+            continue;
         }
+        const int e = p.order[tk];
+        const int l0 = e >> kTaskBits;
+        const long long t0 = e & ((1 << kTaskBits) - 1);
+        int ok = 0;
         if (lane == 0) {
-            sh.stk_l[0] = l;
-            sh.stk_t[0] = t;
+            int *sw = status_word(p, l0, t0);
+            const int cur = ld_acquire(sw);
+            ok = tag_state(cur, EP) == 0 && atomicCAS(sw, cur, MINE1) == cur;
         }
-        sp = 1;
-        if (!unmerged) {
-            // recursion (Fig 2d): claim not-started dependencies (input and residual producers), deepest first
-            // in the emit order
-            for (int s = 0; s < sp; s++) {
-                __syncwarp();
-                const int sl = sh.stk_l[s];
-                const long long st = sh.stk_t[s];
-                const Deps D = deps_of(p.layer, sl, st);
-                const int nd = D.ns + D.nr;
-                for (int i0 = 0; i0 < nd; i0 += 32) {
-                    const int i = i0 + lane;
-                    int claimed = 0, busy = 0, dl = 0;
-                    long long dt = 0;
-                    if (i < nd && sp < kStack - 32) {
-                        dt = dep_at(p.layer, D, i, dl);
-                        int *dw = status_word(p, dl, dt);
-                        const int cur = ld_acquire(dw);
-                        const int s2 = tag_state(cur, EP);
-                        if (s2 == 0 && atomicCAS(dw, cur, (int)(EP | 1)) == cur) claimed = 1;
-                        else if (s2 != 2) busy = 1;
-                    }
-                    const unsigned cm = __ballot_sync(0xffffffff, claimed);
-                    fails += __popc(__ballot_sync(0xffffffff, busy));
-                    oks += __popc(cm);
-                    if (claimed) {
-                        const int pos = sp + __popc(cm & ((1u << lane) - 1));
-                        sh.stk_l[pos] = dl;
-                        sh.stk_t[pos] = dt;
-                    }
-                    sp += __popc(cm);
+        ok = __shfl_sync(0xffffffff, ok, 0);
+        if (!ok) continue;   // already claimed (by a dependent's walk back)
+        oks++;
+        if (lane == 0) {
+            sh.stk_l[0] = l0;
+            sh.stk_t[0] = t0;
+        }
+        int sp = 1;
+        // walk back (Fig 2d): claim the not-started dependencies (input and residual producers), transitively
+        for (int s = 0; s < sp; s++) {
+            __syncwarp();
+            const int sl = sh.stk_l[s];
+            const long long st = sh.stk_t[s];
+            const Deps D = deps_of(p.layer, sl, st);
+            const int nd = D.ns + D.nr;
+            for (int i0 = 0; i0 < nd; i0 += 32) {
+                const int i = i0 + lane;
+                int claimed = 0, dl = 0;
+                long long dt = 0;
+                if (i < nd && sp < kStack - 32) {
+                    dt = dep_at(p.layer, D, i, dl);
+                    int *dw = status_word(p, dl, dt);
+                    const int cur = ld_acquire(dw);
+                    if (tag_state(cur, EP) == 0 && atomicCAS(dw, cur, MINE1) == cur) claimed = 1;
                 }
+                const unsigned cm = __ballot_sync(0xffffffff, claimed);
+                oks += __popc(cm);
+                if (claimed) {
+                    const int pos = sp + __popc(cm & ((1u << lane) - 1));
+                    sh.stk_l[pos] = dl;
+                    sh.stk_t[pos] = dt;
+                }
+                sp += __popc(cm);
             }
-            __syncwarp();
         }
-        // emit dependencies before dependents (reverse stack order)
-        while (sp > 0) {
-            sp--;
-            __syncwarp();
-            emit(sh.stk_l[sp], sh.stk_t[sp]);
+        __syncwarp();
+        // hand the bundle over producers first (layers are listed topologically), deferring what is not ready
+        for (int l = 0; l < p.L; l++) {
+            for (int s = 0; s < sp; s++) {
+                if (sh.stk_l[s] != l) continue;   // (warp-uniform: every lane reads the same entry)
+                const long long t = sh.stk_t[s];
+                __syncwarp();
+                if (!p.defer || ready(l, t)) {
+                    emit(l, t);
+                } else {
+                    defers++;
+                    if (lane == 0) {
+                        sh.pend_l[np] = l;
+                        sh.pend_t[np] = t;
+                    }
+                    np++;
+                }
+                __syncwarp();
+            }
         }
     }
     emit(-1, 0);
     if (lane == 0) {
         if (oks) atomicAdd(&p.counters[1], oks);
-        if (fails) atomicAdd(&p.counters[2], fails);
+        if (defers) atomicAdd(&p.counters[2], defers);
     }
 }
 
@@ -705,7 +782,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
     const bool waits = (warp >= kLoad0 && warp < kLoad0 + kLW) || warp >= kEpi0 || warp == kSched;
     if (waits) pdl_wait();
 
-    const unsigned EP = waits ? run_epoch(p.counters) << 2 : 0u;
+    const unsigned EP = waits ? run_epoch(p.counters) << 10 : 0u;   // tag word: epoch << 10 | owner << 2 | state
     if (warp == kSched) {
         if (p.padded) scheduler_padded(p, sh);
         else scheduler(p, sh);
@@ -1382,14 +1459,18 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
     }
     static const bool layer_major = [] { const char *e = getenv("BDL_GEN_ORDER"); return e && !strcmp(e, "layer"); }();
     long long per_img0 = g.layer[0].ntasks / N;
-    int G = (int)std::max<long long>(1, (2LL * p->num_sms + per_img0 - 1) / std::max<long long>(1, per_img0));
+    // images per group: the group's first layer holds `group_waves` waves of tasks (enough ready work at every
+    // dependency level; measured on B200, cfg4: 2 waves 13.3 ms, 4 waves 11.6 ms, 8 waves 11.2 ms)
+    const double gw = p->opts.group_waves > 0 ? p->opts.group_waves : 8.0;
+    static const double lw = [] { const char *e = getenv("BDL_GEN_LAGWAVES"); return e ? atof(e) : 2.0; }();
+    int G = (int)std::max<long long>(1, (long long)std::ceil(gw * p->num_sms / std::max<long long>(1, per_img0)));
     G = std::min(G, N);
     std::vector<double> key(total, 0.0);
     for (int j = 0; j < L; j++) {
         const gen::LayerP &C = g.layer[j];
         const double per_img = (double)C.ntasks / N;
         // BDL_GEN_ORDER=layer (A/B runs): layer by layer inside each image group
-        const double lag = layer_major ? 2.0 : std::min(1.0, 2.0 * p->num_sms / (G * per_img));
+        const double lag = layer_major ? 2.0 : std::min(1.0, lw * p->num_sms / (G * per_img));
         const double frame = (double)C.in_ext[0] * C.in_ext[1] * C.in_ext[2];
         for (long long t = 0; t < C.ntasks; t++) {
             const gen::Deps D = gen::deps_of(g.layer, j, t);
@@ -1521,6 +1602,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
     P.acc_stride = g.acc_stride;
     P.tmem_cols = g.tmem_cols;
     P.status = (int *)(wsp + sg.status_off);
+    P.defer = p->opts.memo_defer;
     P.counters = (unsigned long long *)(wsp + sg.counter_off);
     cudaFuncSetAttribute(gen::gen_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
     const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;

@@ -172,6 +172,15 @@ class Plan:
         """Dense NC(D)HW -> dense output: brickify, every merged subgraph, unbrickify."""
         return self.unbrickify(self.run(self.brickify(x, stream=stream), stream=stream), stream=stream)
 
+    def forward_into(self, x, out, stream=None):
+        """forward() into a caller-owned dense output tensor (brick buffers are allocated once and reused)."""
+        if getattr(self, "_fw_xb", None) is None:
+            self._fw_xb = self.alloc_bricked(self.in_layout)
+            self._fw_yb = self.alloc_bricked(self.out_layout)
+        self.brickify(x, out=self._fw_xb, stream=stream)
+        self.run(self._fw_xb, self._fw_yb, stream=stream)
+        return self.unbrickify(self._fw_yb, out=out, stream=stream)
+
     def counters(self, i=0, stream=None):
         arr = (ctypes.c_uint64 * 4)()
         check(lib().bdl_plan_counters(self.h, i, ctypes.c_void_p(self.ws_ptr), _stream_handle(stream), arr))

@@ -1,9 +1,13 @@
-"""Multi-GPU plumbing: one process per GPU, batch sharding with no data-path collective.
+"""Multi-GPU plumbing: one process per GPU.
 
 Merged execution never crosses images (bricks block the batch only within a brick, PAPER.md
-L374-376, L738-739), so an inference batch shards trivially across ranks: rank r runs the whole
-merged plan on its contiguous slice of images.  The only collectives are the timing barrier and the
-max-over-ranks reduction in bench.py (plumbing, not the data path).
+L374-376, L738-739), so an inference batch shards trivially across ranks: each rank runs the whole
+merged plan on its share of the images.  Two ways to use that:
+  * weak scaling (bench.py default): every rank runs its own batch; no data-path collective;
+  * strong scaling (BatchRunner): a fixed global batch is split over the ranks in
+    micro-batches and the outputs are all-gathered (NCCL over NVLink) on a communication stream while the
+    next micro-batch computes -- the only data-path collective the north_star allows ("NCCL over NVLink is
+    used only to gather outputs").
 """
 from __future__ import annotations
 
@@ -18,6 +22,85 @@ def shard(n_total: int, rank: int, world: int) -> tuple[int, int]:
     lo = rank * base + min(rank, extra)
     hi = lo + base + (1 if rank < extra else 0)
     return lo, hi
+
+
+def micro_batches(n_total: int, world: int, micro: int):
+    """Global image ranges of the strong-scaling schedule: micro-batch i of rank r holds images
+    [(i*world + r)*mb, (i*world + r + 1)*mb) with mb = n_total / (world*micro).  All-gathering micro-batch i
+    over the ranks (rank-major) then yields the contiguous global images [i*world*mb, (i+1)*world*mb), so each
+    gather lands directly in its final place in the output batch.  Returns mb and, per rank, the list of ranges."""
+    if world <= 0 or micro <= 0 or n_total % (world * micro):
+        raise ValueError(f"batch {n_total} must split into {world} ranks x {micro} micro-batches")
+    mb = n_total // (world * micro)
+    return mb, [[((i * world + r) * mb, (i * world + r + 1) * mb) for i in range(micro)] for r in range(world)]
+
+
+class BatchRunner:
+    """Strong scaling over the batch with an overlapped output gather (one rank's share).
+
+    forward(x_local) takes this rank's micro-batches stacked as [micro*mb, C, D, H, W] (images in the order of
+    micro_batches()[rank]), computes micro-batch i with `compute(x_i, out=y_i)` on the current stream and
+    all-gathers y_i into the output batch on a communication stream (torch.distributed all_gather_into_tensor:
+    NCCL over NVLink/NVSwitch on GPUs, gloo on CPU) while micro-batch i+1 computes.  The result is the whole
+    global batch [n_total, ...] on every rank, in global image order.  gather=False leaves the outputs sharded
+    (the paper's per-GPU runs).  `compute` defaults to a merged-execution Plan of mb images.
+    """
+
+    def __init__(self, n_total, out_shape, rank, world, micro=2, compute=None, plan=None, device="cuda", dtype=None,
+                 group=None):
+        import torch
+        self.mb, ranges = micro_batches(n_total, world, micro)
+        self.ranges = ranges[rank]
+        self.rank, self.world, self.micro, self.group = rank, world, micro, group
+        self.plan = plan
+        if compute is None:
+            if plan is None:
+                raise ValueError("BatchRunner needs a plan or a compute function")
+            compute = lambda x, out: plan.forward_into(x, out)   # noqa: E731
+        self.compute = compute
+        dtype = dtype if dtype is not None else (plan.tdtype if plan is not None else torch.float32)
+        self.device = torch.device(device)
+        self.y_local = torch.empty((micro * self.mb,) + tuple(out_shape), dtype=dtype, device=self.device)
+        self.y_all = torch.empty((n_total,) + tuple(out_shape), dtype=dtype, device=self.device)
+        self.cuda = self.device.type == "cuda"
+        self.comm = torch.cuda.Stream(self.device) if self.cuda else None
+
+    def global_images(self):
+        """Global indices of this rank's images, in the order forward() expects them."""
+        return [n for a, b in self.ranges for n in range(a, b)]
+
+    def forward(self, x_local, gather=True):
+        import torch
+        import torch.distributed as dist
+        mb, W = self.mb, self.world
+        done = []
+        for i in range(self.micro):
+            xi = x_local[i * mb:(i + 1) * mb]
+            yi = self.y_local[i * mb:(i + 1) * mb]
+            self.compute(xi, yi)
+            if not gather:
+                continue
+            dst = self.y_all[i * W * mb:(i + 1) * W * mb]
+            if self.cuda:
+                ev = torch.cuda.Event()
+                ev.record()
+                self.comm.wait_event(ev)
+                with torch.cuda.stream(self.comm):
+                    if W > 1:
+                        dist.all_gather_into_tensor(dst, yi, group=self.group)
+                    else:
+                        dst.copy_(yi)
+                yi.record_stream(self.comm)
+            else:
+                if W > 1:
+                    done.append(dist.all_gather_into_tensor(dst, yi, group=self.group, async_op=True))
+                else:
+                    dst.copy_(yi)
+        for w in done:
+            w.wait()
+        if gather and self.cuda:
+            torch.cuda.current_stream(self.device).wait_stream(self.comm)
+        return self.y_all if gather else self.y_local
 
 
 def env_rank():

@@ -135,13 +135,15 @@ def test_dag_subgraph_schedule_invariance():
     wl = W.make_graph_workload(layers, N, C, D, H, Wd, 2, brick, "bf16", seed=17)
     ref = oracle.run_graph(wl["layers"], wl["x"].numpy(), wl["weights"], wl["biases"], dtype="bf16")
     y0, n0 = None, None
-    for seed in (0, 1, 7, 123):
-        plan = engine.plan_from_workload(wl, force_mode=2, schedule_seed=seed)
+    # memo_defer=1: the paper's "move on and revisit" hand-over (claimed tasks with in-progress dependencies are
+    # set aside); 0: in-order hand-over, the loader waits
+    for seed, defer in ((0, 0), (0, 1), (1, 0), (7, 1), (123, 0), (123, 1)):
+        plan = engine.plan_from_workload(wl, force_mode=2, schedule_seed=seed, memo_defer=defer)
         sgs = plan.subgraphs()
         assert len(sgs) == 1 and sgs[0]["mode"] == "memoized" and sgs[0]["kernel"] == "tcgen05 generic", sgs
         y = plan.forward(wl["x"]).float().cpu().numpy()
         c = plan.counters(0)
-        assert c["computed"] == c["cas_ok"] and c["computed"] > 0, (seed, c)
+        assert c["computed"] == c["cas_ok"] and c["computed"] > 0, (seed, defer, c)
         if y0 is None:
             y0, n0 = y, c["computed"]
             assert rel_err(y, ref) <= TOL

@@ -116,7 +116,9 @@ def test_cfg2_tc_modes_vs_oracle(size):
     wl = workloads.make_workload("cfg2", **size)
     ref = oracle_out(wl)
     plan = engine.plan_from_workload(wl)
-    assert plan.subgraphs()[0]["kernel"] == "tcgen05 band"
+    # C <= 64: the band kernels; C = 128 chains run on the generic kernel (the warp-specialized band kernel's
+    # weights-resident design holds C <= 64)
+    assert plan.subgraphs()[0]["kernel"] == ("tcgen05 band" if wl["C"] <= 64 else "tcgen05 generic")
     outs = {}
     for mode in ("padded", "memoized", "unmerged"):
         plan.set_mode(mode)

@@ -108,3 +108,61 @@ def test_gloo_halo_exchange(world):
     for p in procs:
         p.join(timeout=60)
     assert res == {r: True for r in range(world)}
+
+
+# ---------------------------------------------------------------- batch sharding + overlapped output gather
+@pytest.mark.parametrize("n,world,micro", [(256, 8, 2), (256, 2, 4), (12, 3, 2), (8, 1, 2)])
+def test_micro_batches_cover_batch_in_gather_order(n, world, micro):
+    mb, ranges = parallel.micro_batches(n, world, micro)
+    assert mb * world * micro == n
+    seen = sorted(i for r in range(world) for a, b in ranges[r] for i in range(a, b))
+    assert seen == list(range(n))
+    for i in range(micro):   # gathering micro-batch i rank-major gives contiguous global images
+        cat = [k for r in range(world) for k in range(*ranges[r][i])]
+        assert cat == list(range(i * world * mb, (i + 1) * world * mb))
+    with pytest.raises(ValueError):
+        parallel.micro_batches(n + 1, world, micro)
+
+
+def _layer_fn(x, out):
+    """Stand-in for the merged plan on CPU: one fixed conv + ReLU (the gather path is what is under test)."""
+    w = torch.linspace(-1, 1, 4 * 3 * 3 * 3, dtype=torch.float64).reshape(4, 3, 3, 3)
+    out.copy_(torch.relu(torch.nn.functional.conv2d(x[:, :, 0], w, padding=1))[:, :, None])
+    return out
+
+
+def _gloo_gather_worker(rank, world, port, q):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n, micro = 4 * world, 2
+    g = torch.Generator().manual_seed(5)
+    x_all = torch.randn(n, 3, 1, 6, 5, generator=g, dtype=torch.float64)
+    run = parallel.BatchRunner(n, (4, 1, 6, 5), rank, world, micro=micro, compute=_layer_fn, device="cpu",
+                               dtype=torch.float64)
+    x_local = x_all[run.global_images()].contiguous()
+    y = run.forward(x_local)
+    ref = _layer_fn(x_all, torch.empty(n, 4, 1, 6, 5, dtype=torch.float64))
+    sharded = run.forward(x_local, gather=False)
+    ok = bool(torch.equal(y, ref)) and bool(torch.equal(sharded, ref[run.global_images()]))
+    q.put((rank, ok))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_gloo_batch_gather_equals_unsharded(world):
+    """Strong scaling: every rank computes its micro-batches and all-gathers them; the gathered
+    batch equals the unsharded computation in global image order on every rank."""
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_gloo_gather_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    assert res == {r: True for r in range(world)}
