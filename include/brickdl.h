@@ -113,6 +113,9 @@ typedef struct bdl_plan_opts {
                                     faster on B200) */
     int32_t group_waves;         /* generic kernel, memoized: images per task-order group sized so the group's first
                                     layer holds this many waves of tasks (0 = default 8) */
+    int32_t fuse_pool;           /* generic kernel: a subgraph's trailing max-pool as the last conv's epilogue
+                                    (L620-626): 0 = where measured faster on B200 (memoized / unmerged, <= 128
+                                    channels), 1 = always, 2 = never (separate pool kernel) */
 } bdl_plan_opts;
 
 typedef struct bdl_plan bdl_plan;  /* opaque, library-owned host object */

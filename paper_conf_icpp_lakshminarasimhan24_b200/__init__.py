@@ -40,7 +40,8 @@ class bdl_layer(ctypes.Structure):
 class bdl_plan_opts(ctypes.Structure):
     _fields_ = [("delta_threshold", _f64), ("tau", _i64), ("bcand", _i32 * 4), ("onchip_budget", _i64),
                 ("force_mode", _i32), ("force_brick", _i32), ("max_subgraph_layers", _i32),
-                ("num_sms", _i32), ("schedule_seed", _i32), ("memo_defer", _i32), ("group_waves", _i32)]
+                ("num_sms", _i32), ("schedule_seed", _i32), ("memo_defer", _i32), ("group_waves", _i32),
+                ("fuse_pool", _i32)]
 
 
 class BrickDLError(RuntimeError):

@@ -55,6 +55,14 @@ struct LayerP {
     TView src, out, res;
     const __nv_bfloat16 *w;   // packed [nc][kb][ks][2][Nc][8]
     int srcl, resl;           // producer (index in the subgraph) of the input / of the residual, -1 = external
+    // fused max-pool (the subgraph ends in a pool of this conv, L620-626): the task grid and `out` are the POOLED
+    // output; a task is a Tpb x Tpw tile of pool outputs and computes the conv tile under its windows
+    // (Tb = (Tpb-1)*ps + pk rows, Fig 4 rule with the pool's stride as padding factor, L456-458), pools it in
+    // the epilogue and never materializes the conv output
+    int pool;
+    int pk[2], ps[2], ppd[2]; // pool window / stride / padding (h, w)
+    int pout[3];              // pooled output extents (d, h, w); out_ext stays the conv's
+    int Tpb, Tpw;
     const float *bias;        // [cout]
     int relu, has_res;
     int cin, cout;
@@ -85,6 +93,7 @@ struct Params {
     LayerP layer[kMaxLayers];
     int L;
     int nin, nw, in_stride, w_stride;    // ring depths and slot strides (bytes)
+    int pool_off;                        // fused pool: byte offset of the epilogue staging tile in dynamic smem
     int nacc, acc_stride, tmem_cols;
     int *status;
     int defer;                           // bdl_plan_opts.memo_defer: 1 = hand over only ready tasks (revisit the others)
@@ -170,6 +179,14 @@ __device__ __forceinline__ long long pix(const TView &v, int n, int d, int y, in
     return phys * v.brick_elems + (long long)in * v.Cp;
 }
 
+// First conv-output row / column of tile (ty, tx) (pooled layers: under its first pool window; may be < 0).
+__host__ __device__ __forceinline__ int tile_y0(const LayerP &L, int ty) {
+    return L.pool ? ty * L.Tpb * L.ps[0] - L.ppd[0] : ty * L.Tb;
+}
+__host__ __device__ __forceinline__ int tile_x0(const LayerP &L, int tx) {
+    return L.pool ? tx * L.Tpw * L.ps[1] - L.ppd[1] : tx * L.Tw;
+}
+
 // Dependencies of task t of layer C: the tiles of its input producer P covering its input window (every channel
 // chunk of P), and the tiles of its residual producer R covering its output tile (the same channel chunk).
 struct DepRange { int n, d0, nd, b0, nb, x0, nx, c0, nnc; };
@@ -184,12 +201,13 @@ __host__ __device__ __forceinline__ DepRange dep_range_src(const LayerP &C, cons
     hi = min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.k[0] - 1);
     r.d0 = lo;
     r.nd = max(0, hi - lo + 1);
-    lo = max(0, c.ty * C.Tb * C.s[1] - C.pd[1]);
-    hi = min(C.in_ext[1] - 1, (c.ty * C.Tb + C.Tb - 1) * C.s[1] - C.pd[1] + C.k[1] - 1);
+    const int y0 = tile_y0(C, c.ty), x0 = tile_x0(C, c.tx);
+    lo = max(0, y0 * C.s[1] - C.pd[1]);
+    hi = min(C.in_ext[1] - 1, (y0 + C.Tb - 1) * C.s[1] - C.pd[1] + C.k[1] - 1);
     r.b0 = lo / P.Tb;
     r.nb = hi >= lo ? hi / P.Tb - r.b0 + 1 : 0;
-    lo = max(0, c.tx * C.Tw * C.s[2] - C.pd[2]);
-    hi = min(C.in_ext[2] - 1, (c.tx * C.Tw + C.Tw - 1) * C.s[2] - C.pd[2] + C.k[2] - 1);
+    lo = max(0, x0 * C.s[2] - C.pd[2]);
+    hi = min(C.in_ext[2] - 1, (x0 + C.Tw - 1) * C.s[2] - C.pd[2] + C.k[2] - 1);
     r.x0 = lo / P.Tw;
     r.nx = hi >= lo ? hi / P.Tw - r.x0 + 1 : 0;
     return r;
@@ -260,6 +278,19 @@ __host__ __device__ inline void region_of(const LayerP *ly, int L, const int PB[
     }
     for (int j = L - 1; j > l; j--) {
         const LayerP &J = ly[j];
+        if (J.pool) {   // pooled output region -> the conv output region under its windows (clipped to the map)
+            for (int d = 1; d < 3; d++) {
+                const int h = hi[d] < J.pout[d] ? hi[d] : J.pout[d];
+                if (h <= lo[d]) {
+                    lo[d] = hi[d] = 0;
+                    continue;
+                }
+                const int nlo = lo[d] * J.ps[d - 1] - J.ppd[d - 1], nhi = (h - 1) * J.ps[d - 1] - J.ppd[d - 1] + J.pk[d - 1];
+                lo[d] = nlo > 0 ? nlo : 0;
+                hi[d] = nhi < J.out_ext[d] ? nhi : J.out_ext[d];
+                if (hi[d] < lo[d]) hi[d] = lo[d];
+            }
+        }
         for (int d = 0; d < 3; d++) {
             const int h = hi[d] < J.out_ext[d] ? hi[d] : J.out_ext[d];
             if (h <= lo[d]) {
@@ -280,13 +311,15 @@ __host__ __device__ inline int region_x0(const LayerP &L, int lo2) {
 __host__ __device__ inline int region_subtiles(const LayerP &L, const int lo[3], const int hi[3]) {
     const int a = hi[0] - lo[0], b = hi[1] - lo[1], c = hi[2] - region_x0(L, lo[2]);
     if (a <= 0 || b <= 0 || c <= 0) return 0;
-    return a * ((b + L.Tb - 1) / L.Tb) * ((c + L.Tw - 1) / L.Tw) * L.nnc;
+    const int tb = L.pool ? L.Tpb : L.Tb, tw = L.pool ? L.Tpw : L.Tw;   // pooled: tiles of the pooled region
+    return a * ((b + tb - 1) / tb) * ((c + tw - 1) / tw) * L.nnc;
 }
 
 // One unit of work of the pipeline: an output tile of layer l (memoized/unmerged: a tile of the bricked
 // grid; padded: a tile of a block's region), with where its input comes from and its output goes.
 struct Tile {
     int n, d, y0, x0, nc;
+    int py0, px0;              // pooled layers: first pool-output row / column of the tile
     int hi[3];                 // exclusive bounds of the positions this tile writes
     int src_scr, dst_scr;      // padded: input / output in the CTA's scratch
     int slo[3], shi[3];        // source region (scratch) bounds
@@ -298,7 +331,8 @@ __device__ __forceinline__ Tile make_tile(const Params &p, int l, long long t) {
     Tile T;
     if (!p.padded) {
         const TaskC c = decode(L, t);
-        T.n = c.n; T.d = c.d; T.y0 = c.ty * L.Tb; T.x0 = c.tx * L.Tw; T.nc = c.nc;
+        T.n = c.n; T.d = c.d; T.y0 = tile_y0(L, c.ty); T.x0 = tile_x0(L, c.tx); T.nc = c.nc;
+        T.py0 = c.ty * L.Tpb; T.px0 = c.tx * L.Tpw;
         T.hi[0] = L.grid[0]; T.hi[1] = L.grid[1]; T.hi[2] = L.grid[2];
         T.src_scr = T.dst_scr = 0;
         T.slot = 0;
@@ -317,11 +351,18 @@ __device__ __forceinline__ Tile make_tile(const Params &p, int l, long long t) {
     int lo[3], hi[3];
     region_of(p.layer, p.L, p.PB, blk, l, lo, hi);
     const int xs = region_x0(L, lo[2]);
-    const int nty = (hi[1] - lo[1] + L.Tb - 1) / L.Tb, ntx = (hi[2] - xs + L.Tw - 1) / L.Tw;
+    const int tb = L.pool ? L.Tpb : L.Tb, tw = L.pool ? L.Tpw : L.Tw;
+    const int nty = (hi[1] - lo[1] + tb - 1) / tb, ntx = (hi[2] - xs + tw - 1) / tw;
     const int kx = k % ntx; k /= ntx;
     const int ky = k % nty;
     const int kd = k / nty;
     T.d = lo[0] + kd; T.y0 = lo[1] + ky * L.Tb; T.x0 = xs + kx * L.Tw;
+    if (L.pool) {   // (lo, hi) is a pooled region
+        T.py0 = lo[1] + ky * L.Tpb;
+        T.px0 = xs + kx * L.Tpw;
+        T.y0 = T.py0 * L.ps[0] - L.ppd[0];
+        T.x0 = T.px0 * L.ps[1] - L.ppd[1];
+    }
     for (int d = 0; d < 3; d++) { T.hi[d] = hi[d]; T.dlo[d] = lo[d]; }
     T.dst_scr = l < p.L - 1;
     T.src_scr = l > 0;
@@ -972,7 +1013,89 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(L.res.ptr);
             const int d = T.d;
             __nv_bfloat16 *scr = T.dst_scr ? reinterpret_cast<__nv_bfloat16 *>(scr_slot(p, T.slot) + L.scr_off) : nullptr;
-            for (int it = rank; it < items; it += 4) {
+            if (L.pool) {
+                // fused max-pool (the subgraph's last layer, L620-626): per channel batch, every epilogue warp turns its
+                // TMEM rows into bf16 conv outputs (bias -> ReLU -> RNE, the conv layer's own epilogue) in a shared
+                // staging tile; then the 512 threads take the max over each pool window of the tile's conv positions
+                // that lie inside the conv output (out-of-range taps ignored) and store the pooled
+                // 16-B channel vectors.  The conv output itself is never written to global memory.
+                uint4 *stg = reinterpret_cast<uint4 *>(smem + p.pool_off);
+                const int nck = CB / 8;
+                // channel batches staged together: the 4 warp ranks share ntl x gcb (tile, batch) items, so every
+                // epilogue warp reads TMEM even when a task has a single M tile; staging <= ntl*128 x 128 ch
+                const int gcb = min(ncb, max(1, 4 / L.ntl));
+                const int nchk = gcb * nck;   // 16-B chunks per staged position (a power of two)
+                for (int cb0 = 0; cb0 < ncb; cb0 += gcb) {
+                    const int ng = min(gcb, ncb - cb0);
+                    for (int it = rank; it < L.ntl * ng; it += 4) {
+                        const int tl = it / ng, cbl = it - tl * ng;
+                        const int ch0 = T.nc * L.Nc + (cb0 + cbl) * CB;
+                        const int m = tl * 128 + quad * 32 + lane;
+                        uint32_t r[2][16];
+                        const uint32_t taddr =
+                            tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) + tl * L.Nc + (cb0 + cbl) * CB;
+                        ptx::tmem_ld16(taddr, r[0]);
+                        if (CB == 32) ptx::tmem_ld16(taddr + 16, r[1]);
+                        ptx::tmem_ld_wait();
+                        ptx::reg_fence16(r[0]);
+                        ptx::reg_fence16(r[1]);
+#pragma unroll
+                        for (int k = 0; k < 4; k++) {
+                            if (k >= nck) break;
+                            float v[8];
+                            const float4 b0 = __ldg(reinterpret_cast<const float4 *>(L.bias + ch0 + k * 8));
+                            const float4 b1 = __ldg(reinterpret_cast<const float4 *>(L.bias + ch0 + k * 8 + 4));
+                            const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+                            for (int e = 0; e < 8; e++) {
+                                v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]) + bb[e];
+                                if (L.relu) v[e] = fmaxf(v[e], 0.f);
+                            }
+                            stg[m * nchk + ((cbl * nck + k) ^ (m & (nchk - 1)))] =
+                                make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
+                        }
+                    }
+                    asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");
+                    const int nc_g = ng * nck;
+                    const int nout = L.Tpb * L.Tpw * nc_g;
+                    for (int q = ew * 32 + lane; q < nout; q += 32 * kEpiW) {
+                        const int ck = q % nc_g, o = q / nc_g;
+                        const int ox = o % L.Tpw, oy = o / L.Tpw;
+                        const int py = T.py0 + oy, px = T.px0 + ox;
+                        if (d >= T.hi[0] || py >= T.hi[1] || px >= T.hi[2]) continue;
+                        if (p.padded && (py < T.dlo[1] || px < T.dlo[2])) continue;
+                        uint4 *dst = reinterpret_cast<uint4 *>(outp + pix_pow2(L.out, L.lB, T.n, d, py, px) + T.nc * L.Nc +
+                                                               cb0 * CB) + ck;
+                        if (d >= L.pout[0] || py >= L.pout[1] || px >= L.pout[2]) {   // masked position of the bricked grid
+                            *dst = make_uint4(0, 0, 0, 0);
+                            continue;
+                        }
+                        __nv_bfloat162 mx[4];
+                        bool any = false;
+                        for (int rr = 0; rr < L.pk[0]; rr++) {
+                            const int i = oy * L.ps[0] + rr, y = T.y0 + i;
+                            if (y < 0 || y >= L.out_ext[1]) continue;
+                            for (int cc = 0; cc < L.pk[1]; cc++) {
+                                const int j = ox * L.ps[1] + cc, x = T.x0 + j;
+                                if (x < 0 || x >= L.out_ext[2]) continue;
+                                const int m = i * L.Wp + j;
+                                const uint4 u = stg[m * nchk + (ck ^ (m & (nchk - 1)))];
+                                const __nv_bfloat162 *h = reinterpret_cast<const __nv_bfloat162 *>(&u);
+                                if (!any) {
+                                    mx[0] = h[0]; mx[1] = h[1]; mx[2] = h[2]; mx[3] = h[3];
+                                    any = true;
+                                } else {
+                                    mx[0] = __hmax2(mx[0], h[0]); mx[1] = __hmax2(mx[1], h[1]);
+                                    mx[2] = __hmax2(mx[2], h[2]); mx[3] = __hmax2(mx[3], h[3]);
+                                }
+                            }
+                        }
+                        *dst = *reinterpret_cast<const uint4 *>(mx);
+                    }
+                    asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");   // staging reused by the next group
+                }
+            }
+            for (int it = rank; it < (L.pool ? 0 : items); it += 4) {
                 const int tl = it / ncb, cb = it - tl * ncb;
                 const int m = tl * 128 + quad * 32 + lane;
                 const int i = m / L.Wp, j = m - i * L.Wp;
@@ -1147,16 +1270,31 @@ static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out,
     return true;
 }
 
+// Fused pool: epilogue staging tile, every M row of the conv tile x the channel batches staged together, bf16.
+static int gen_pool_stage_bytes(const gen::LayerP &G) {
+    const int CB = G.Nc >= 32 ? 32 : 16, ncb = G.Nc / CB;
+    const int gcb = std::min(ncb, std::max(1, 4 / G.ntl));   // channel batches staged together (epilogue)
+    return G.ntl * 128 * gcb * CB * 2;
+}
+
 // Tile geometry: output tiles of Tb rows x Tw columns (Tw a multiple of walign) covering cover_h x
 // cover_w positions of one plane; the best useful fraction of MMA rows that fits the shared memory.
-static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign) {
+// Fused-pool layers (G.pool): the loops run over pooled tiles Tpb x Tpw covering cover_h x cover_w pool outputs, and
+// the conv tile is the region under their windows, Tb = (Tpb-1)*ps + pk (likewise Tw).
+constexpr int kGenPoolStageMax = 32 * 1024;   // fused pool: largest epilogue staging tile
+
+static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign, int in_budget = kGenInBudget) {
     double best = -1e30;
     bool found = false;
     gen::LayerP cand = G;
-    for (int Tb = std::min(cover_h, 32); Tb >= 1; Tb--) {
-        for (int Tw = (cover_w + walign - 1) / walign * walign; Tw >= walign; Tw -= walign) {
+    for (int Ub = std::min(cover_h, 32); Ub >= 1; Ub--) {
+        for (int Uw = (cover_w + walign - 1) / walign * walign; Uw >= walign; Uw -= walign) {
+            const int Tb = G.pool ? (Ub - 1) * G.ps[0] + G.pk[0] : Ub, Tw = G.pool ? (Uw - 1) * G.ps[1] + G.pk[1] : Uw;
+            if (Tb > 64 || Tw > 256) continue;
             cand.Tb = Tb;
             cand.Tw = Tw;
+            cand.Tpb = G.pool ? Ub : 0;
+            cand.Tpw = G.pool ? Uw : 0;
             cand.in_rows = (Tb - 1) * G.s[1] + G.k[1];
             cand.in_cols = (Tw - 1) * G.s[2] + G.k[2];
             cand.Wp = (cand.in_cols + G.s[2] - 1) / G.s[2];
@@ -1177,8 +1315,9 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
                                : G.amode == gen::AM_SW64  ? rows * 64
                                : (G.amode == gen::AM_PLANES ? G.kc * rows * 16 : rows * 16);
             cand.stage_bytes = (cand.stage_bytes + 1023) / 1024 * 1024;
-            if (cand.stage_bytes * 2 > kGenInBudget) continue;
-            const int nty = (cover_h + Tb - 1) / Tb, ntx = (cover_w + Tw - 1) / Tw;
+            if (cand.stage_bytes * 2 > in_budget) continue;   // two input stages at least
+            if (G.pool && gen_pool_stage_bytes(cand) > kGenPoolStageMax) continue;
+            const int nty = (cover_h + Ub - 1) / Ub, ntx = (cover_w + Uw - 1) / Uw;
             // time model per plane: tasks x (MMAs per task + a fixed per-task cost), times a penalty for loaded
             // halo pixels.  The fixed cost (claim, dependency acquire, barriers, epilogue hand-off, publication)
             // was measured on B200 at ~3.7 us per task with the MMAs, loads and stores disabled (cfg5,
@@ -1187,7 +1326,7 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
             const double halo = (double)cand.in_rows * cand.in_cols / ((double)Tb * Tw * G.s[1] * G.s[2]);
             const double mmas = (double)cand.ntl * G.nks * G.nkb;
             const double cost = (double)nty * ntx * (mmas + kGenTaskOverheadMmas) * (1.0 + 0.1 * (halo - 1.0));
-            const double score = -cost + 1e-6 * Tb * Tw;
+            const double score = -cost + 1e-6 * Ub * Uw;
             if (score > best) {
                 best = score;
                 G = cand;
@@ -1246,10 +1385,31 @@ static unsigned long long *gen_prof_buffer(cudaStream_t s) {
 struct GenGeom {
     gen::LayerP layer[kMaxLayers];
     int L;
-    int nin, in_stride, nw, w_stride, acc_stride, nacc, tmem_cols, smem;
+    int nin, in_stride, nw, w_stride, acc_stride, nacc, tmem_cols, smem, pool_bytes;
     int PB[3], npb[3];
     long long scr_slot;
 };
+
+// Can the subgraph's trailing max-pool be fused into its last conv's epilogue?  2-D pool reading the last conv,
+// no residual on that conv, and the conv's output is not needed by a later subgraph (then it is never materialized).
+// Measured on B200 (VGG-16 N=128): fused pools win on convs of <= 128 channels in memoized / unmerged
+// execution (stage 2: 1.27 -> 1.09 ms, stage 1 memoized 2.35 -> 2.26 ms) and lose on 256 / 512 channels (1.55 -> 1.75,
+// 0.82 -> 0.93 ms) and in padded mode (2.53 -> 2.72 ms): those keep the separate vectorized pool kernel.
+bool gen_pool_fused(const bdl_plan *p, const Subgraph &sg, int nconv, bool padded) {
+    const int mode = p->opts.fuse_pool;   // 0 measured rule, 1 always, 2 never
+    if (mode == 2 || nconv < 1 || nconv != sg.last - sg.first) return false;
+    if (mode != 1 && (padded || p->layers[sg.first + nconv - 1].L.cout > 128)) return false;
+    const bdl_layer &pl = p->layers[sg.last].L;
+    const int ci = sg.first + nconv - 1;
+    if (pl.kind != BDL_OP_MAXPOOL || pl.input != ci) return false;
+    if (pl.k[0] != 1 || pl.stride[0] != 1 || pl.pad[0] != 0) return false;
+    for (int d = 1; d < 3; d++)
+        if (pl.k[d] > 8 || pl.stride[d] < 1 || pl.stride[d] > pl.k[d] || pl.pad[d] >= pl.k[d]) return false;
+    if (p->layers[ci].L.residual != BDL_NO_RESIDUAL) return false;
+    for (const Tensor &t : p->tensors)
+        if (t.producer == ci) return false;   // a live-out: later subgraphs read the conv output
+    return true;
+}
 
 static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool padded, GenGeom &g) {
     memset(&g, 0, sizeof(g));
@@ -1264,6 +1424,27 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
         g.layer[j].srcl = j < (int)sg.src_local.size() ? sg.src_local[j] : j - 1;
         g.layer[j].resl = j < (int)sg.res_local.size() ? sg.res_local[j] : -1;
         if (g.layer[j].resl >= 0 && g.layer[g.layer[j].resl].Nc != g.layer[j].Nc) return false;
+    }
+    const bool fused = gen_pool_fused(p, sg, nconv, padded && nconv > 1);
+    // the pool's staging tile takes one weight stage's room (2 weight stages instead of 3), not input-ring room: smaller
+    // input stages cost more, smaller tiles (measured on B200, VGG stage 1: 2.9 -> 3.7 ms when the ring shrank)
+    const int in_budget = kGenInBudget;
+    if (fused) {   // the pool's output is the last conv's task grid
+        gen::LayerP &G = g.layer[nconv - 1];
+        const Layer &pl = p->layers[sg.last];
+        bdl_layout lp;
+        bdl_layout_init(&lp, nsp, pl.out_ext[0], pl.L.cout, pl.out_ext[1], pl.out_ext[2], pl.out_ext[3], p->in_layout.Bn,
+                        p->in_layout.Bd, p->in_layout.Bh, p->in_layout.Bw, BDL_BF16);
+        G.pool = 1;
+        for (int d = 0; d < 2; d++) {
+            G.pk[d] = pl.L.k[d + 1];
+            G.ps[d] = pl.L.stride[d + 1];
+            G.ppd[d] = pl.L.pad[d + 1];
+        }
+        for (int d = 0; d < 3; d++) G.pout[d] = pl.out_ext[d + 1];
+        G.grid[0] = (int)(lp.nb[1] * lp.Bd);
+        G.grid[1] = (int)(lp.nb[2] * lp.Bh);
+        G.grid[2] = (int)(lp.nb[3] * lp.Bw);
     }
     if (padded && nconv > 1) {
         if (!sg.chain) return false;   // padded mode: chains only (partition)
@@ -1307,10 +1488,11 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
             const int Bw = p->in_layout.Bw;
             const bool xal = j == 0 && gen_pad_tma_ok(G, nsp, Bw);
             G.xal = xal ? 1 : 0;
-            if (!gen_layer_tiles(G, G.pR[1], xal ? G.pR[2] + Bw - 1 : G.pR[2], xal ? Bw : 1)) return false;
+            if (!gen_layer_tiles(G, G.pR[1], xal ? G.pR[2] + Bw - 1 : G.pR[2], xal ? Bw : 1, in_budget)) return false;
             // padded sub-task ids pack (sub-tile << 8 | channel chunk): 16 + 8 bits
             const int xs = xal ? G.pR[2] + Bw - 1 : G.pR[2];
-            const long long nsub = (long long)G.pR[0] * ((G.pR[1] + G.Tb - 1) / G.Tb) * ((xs + G.Tw - 1) / G.Tw);
+            const int tb = G.pool ? G.Tpb : G.Tb, tw = G.pool ? G.Tpw : G.Tw;
+            const long long nsub = (long long)G.pR[0] * ((G.pR[1] + tb - 1) / tb) * ((xs + tw - 1) / tw);
             if (nsub >= (1LL << 16) || G.nnc >= (1 << 8)) return false;
             if (j < nconv - 1) {
                 G.scr_off = g.scr_slot;
@@ -1320,30 +1502,37 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
     } else {
         for (int j = 0; j < nconv; j++) {
             gen::LayerP &G = g.layer[j];
-            if (!gen_layer_tiles(G, G.grid[1], G.grid[2], p->in_layout.Bw)) return false;
+            // pooled tiles: brick-aligned conv columns (TMA rows) when the windows tile the map (k = s, no padding)
+            int walign = p->in_layout.Bw;
+            if (G.pool) walign = (G.pk[1] == G.ps[1] && G.ppd[1] == 0 && p->in_layout.Bw % G.ps[1] == 0) ? p->in_layout.Bw / G.ps[1] : 1;
+            if (!gen_layer_tiles(G, G.grid[1], G.grid[2], walign, in_budget)) return false;
             G.ntd = G.grid[0];
-            G.nty = (G.grid[1] + G.Tb - 1) / G.Tb;
-            G.ntx = (G.grid[2] + G.Tw - 1) / G.Tw;
+            const int tb = G.pool ? G.Tpb : G.Tb, tw = G.pool ? G.Tpw : G.Tw;   // pooled: tiles of pool outputs
+            G.nty = (G.grid[1] + tb - 1) / tb;
+            G.ntx = (G.grid[2] + tw - 1) / tw;
             G.ntasks = (long long)p->layers[sg.first + j].out_ext[0] * G.ntd * G.nty * G.ntx * G.nnc;
             if (G.ntasks >= (1LL << gen::kTaskBits)) return false;   // order entries: (layer << 26) | task
         }
     }
     int in_stride = 0, w_stride = 0, acc = 0;
+    g.pool_bytes = 0;
     for (int j = 0; j < nconv; j++) {
         const gen::LayerP &G = g.layer[j];
         in_stride = std::max(in_stride, G.stage_bytes);
         w_stride = std::max(w_stride, G.kpw * 2 * G.Nc * 16);
         acc = std::max(acc, G.ntl * G.Nc);
+        if (G.pool) g.pool_bytes = (gen_pool_stage_bytes(G) + 1023) / 1024 * 1024;
     }
     g.in_stride = in_stride;
     g.w_stride = (w_stride + 1023) / 1024 * 1024;
     g.nin = std::min(gen::kMaxIn, kGenInBudget / in_stride);
-    g.nw = kGenW;
+    g.nw = g.pool_bytes ? kGenW - 1 : kGenW;
+    if (g.pool_bytes > kGenWStage) return false;
     g.acc_stride = acc;
     g.nacc = 2 * acc <= 512 ? 2 : 1;
     g.tmem_cols = 32;
     while (g.tmem_cols < g.nacc * acc) g.tmem_cols *= 2;
-    g.smem = g.nin * in_stride + g.nw * g.w_stride + 1024;
+    g.smem = g.nin * in_stride + g.nw * g.w_stride + g.pool_bytes + 1024;
     return g.nin >= 2 && g.smem <= 227 * 1024 - (int)sizeof(gen::Shared) - 1024;
 }
 
@@ -1483,8 +1672,8 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
             if (D.ns == 0) {   // reads an external tensor: how far down its input frame the window reaches
                 const gen::TaskC c = gen::decode(C, t);
                 const int z = std::min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.k[0] - 1);
-                const int y = std::min(C.in_ext[1] - 1, (c.ty * C.Tb + C.Tb - 1) * C.s[1] - C.pd[1] + C.k[1] - 1);
-                const int x = std::min(C.in_ext[2] - 1, (c.tx * C.Tw + C.Tw - 1) * C.s[2] - C.pd[2] + C.k[2] - 1);
+                const int y = std::min(C.in_ext[1] - 1, (gen::tile_y0(C, c.ty) + C.Tb - 1) * C.s[1] - C.pd[1] + C.k[1] - 1);
+                const int x = std::min(C.in_ext[2] - 1, (gen::tile_x0(C, c.tx) + C.Tw - 1) * C.s[2] - C.pd[2] + C.k[2] - 1);
                 k = std::max(k, ((double)std::max(z, 0) * C.in_ext[1] + std::max(y, 0)) * C.in_ext[2] + std::max(x, 0)) /
                     frame;
             }
@@ -1529,8 +1718,9 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
                                const std::vector<TView> &res, unsigned char *wsp, cudaStream_t s, int *launches) {
     const int L = gen_conv_layers(p, sg);
     if (L <= 0) return fail(BDL_EUNSUPPORTED, "generic tcgen05 kernel: subgraph not supported");
-    const bool pool_tail = L < sg.last - sg.first + 1;
     const bool padded = sg.mode == BDL_MODE_PADDED && L > 1;
+    const bool pool_fused = gen_pool_fused(p, sg, L, padded);
+    const bool pool_tail = L < sg.last - sg.first + 1 && !pool_fused;
     GenGeom g;
     gen_geometry(p, sg, L, padded, g);
     gen::Params P;
@@ -1567,8 +1757,11 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
         G.out = outs[j];
         G.tma = 0;
         G.pxo = 0;
+        // pooled tiles start at tx * Tpw * ps - pad: TMA rows need that brick-aligned and non-negative
+        const bool pool_al = !G.pool || (G.ppd[0] == 0 && G.ppd[1] == 0 && (G.Tpw * G.ps[1]) % p->in_layout.Bw == 0);
         // (padded mode: only the first layer, whose tiles are brick-aligned (xal); later layers read CTA scratch)
-        if ((!padded || G.xal) && G.amode == gen::AM_SW128 && G.s[1] == 1 && G.s[2] == 1 && G.k[0] == 1 && nsp == 2 &&
+        if (!pool_al) {
+        } else if ((!padded || G.xal) && G.amode == gen::AM_SW128 && G.s[1] == 1 && G.s[2] == 1 && G.k[0] == 1 && nsp == 2 &&
             !G.src.bmap && G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
             gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw))
             G.tma = 1;
@@ -1595,6 +1788,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
         G.task_base = sg.task_base[j];
     }
     P.nin = g.nin;
+    P.pool_off = g.nin * g.in_stride + g.nw * g.w_stride;
     P.in_stride = g.in_stride;
     P.nw = g.nw;
     P.w_stride = g.w_stride;
@@ -1655,7 +1849,8 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
 
 int gen_launches(const bdl_plan *p, const Subgraph &sg) {
     const int L = gen_conv_layers(p, sg);
-    const bool pool_tail = L < sg.last - sg.first + 1;
+    const bool pool_tail = L < sg.last - sg.first + 1 &&
+                           !gen_pool_fused(p, sg, L, sg.mode == BDL_MODE_PADDED && L > 1);
     const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;
     return (unmerged ? L : 1) + (pool_tail ? 1 : 0);
 }

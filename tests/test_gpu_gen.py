@@ -54,7 +54,14 @@ GRAPHS = {
     "wide_out_nc8": ([W.conv(512, 2048, 1)], 3, 512, 1, 7, 7, (1, 1, 8, 8)),
     "planes_16_32": ([W.conv(16, 32, 3), W.conv(32, 32, 3)], 2, 16, 1, 20, 20, (1, 1, 8, 8)),
     "planes_3d": ([W.conv(32, 32, 3, nsp=3), W.conv(32, 32, 3, nsp=3)], 1, 32, 10, 12, 9, (1, 4, 4, 4)),
+    # max-pool fused into the last conv's epilogue: VGG 2x2/2, ResNet stem 3x3/2 pad 1 (overlapping
+    # windows: conv tiles recompute one shared row/column), ragged floor-mode extents, one conv + pool
     "pool_tail": ([W.conv(64, 64, 3), W.conv(64, 64, 3), W.pool(64, 2, 2, 0)], 2, 64, 1, 20, 20, (1, 1, 8, 8)),
+    "pool_fused_2x2_ragged": ([W.conv(32, 64, 3), W.conv(64, 128, 3), W.pool(128, 2, 2, 0)], 2, 32, 1, 21, 19,
+                              (1, 1, 8, 8)),
+    "pool_fused_stem_3x3s2p1": ([W.conv(3, 64, 7, 2, 3), W.pool(64, 3, 2, 1)], 2, 3, 1, 38, 42, (1, 1, 8, 8)),
+    "pool_fused_chain_3x3s2p1": ([W.conv(64, 64, 1), W.conv(64, 64, 3), W.pool(64, 3, 2, 1)], 2, 64, 1, 27, 30,
+                                 (1, 1, 8, 8)),
     # 3x3x3 x 64 channels = 108 k-steps per layer (the Fig 10/11 microbenchmark layers)
     "sw128_3d_c64": ([W.conv(64, 64, 3, nsp=3), W.conv(64, 64, 3, nsp=3)], 1, 64, 10, 12, 9, (1, 4, 4, 4)),
     "sw128_3d_c64_valid": ([W.conv(64, 64, 3, 1, 0, nsp=3), W.conv(64, 64, 3, 1, 0, nsp=3)], 1, 64, 13, 12, 14,
@@ -66,13 +73,14 @@ GRAPHS = {
 }
 
 
+@pytest.mark.parametrize("fuse", [0, 1])
 @pytest.mark.parametrize("name", sorted(GRAPHS))
-def test_gen_vs_oracle(name):
+def test_gen_vs_oracle(name, fuse):
     layers, N, C, D, H, Wd, brick = GRAPHS[name]
     nsp = 3 if brick[1] > 1 else 2
     wl = W.make_graph_workload(layers, N, C, D, H, Wd, nsp, brick, "bf16", seed=11)
     ref = oracle.run_graph(wl["layers"], wl["x"].numpy(), wl["weights"], wl["biases"], dtype="bf16")
-    plan = engine.plan_from_workload(wl, force_mode=2)
+    plan = engine.plan_from_workload(wl, force_mode=2, fuse_pool=fuse)
     sgs = plan.subgraphs()
     assert any(s["kernel"] == "tcgen05 generic" for s in sgs), sgs
     outs = {}
@@ -85,7 +93,8 @@ def test_gen_vs_oracle(name):
     plan.set_mode("memoized")
     plan.forward(wl["x"])
     for i, s in enumerate(sgs):
-        if s["kernel"] == "tcgen05 generic" and s["last"] > s["first"]:
+        nconv = sum(l["kind"] == "conv" for l in wl["layers"][s["first"]:s["last"] + 1])
+        if s["kernel"] == "tcgen05 generic" and nconv > 1:
             c = plan.counters(i)
             assert c["computed"] == c["cas_ok"] and c["computed"] > 0, c
 
@@ -185,3 +194,22 @@ def test_cuda_graph_replay(which):
             y = plan.unbrickify(yb)
             torch.cuda.synchronize()
             assert torch.equal(y, ref), (which, rep)
+
+
+@pytest.mark.parametrize("brick", [4, 8, 16])
+def test_gen_padded_fused_pool_blocks(brick):
+    """Padded mode with the pool fused into the last conv: each block's pooled region maps back through the pool
+    window (Fig 4 with the pool stride as padding factor, L456-458) and the chain; several block edges."""
+    layers = [W.conv(64, 64, 3), W.conv(64, 64, 3), W.pool(64, 3, 2, 1)]
+    wl = W.make_graph_workload(layers, 2, 64, 1, 30, 27, 2, (1, 1, 8, 8), "bf16", seed=23)
+    ref = oracle.run_graph(wl["layers"], wl["x"].numpy(), wl["weights"], wl["biases"], dtype="bf16")
+    plan = engine.plan_from_workload(wl, force_mode=1, force_brick=brick, fuse_pool=1)
+    assert plan.subgraphs()[0]["last"] == 2 and plan.launches_per_run == 1   # one launch: the pool is fused
+    yp = plan.forward(wl["x"]).float().cpu().numpy()
+    assert rel_err(yp, ref) <= TOL
+    plan.set_mode("memoized")
+    np.testing.assert_array_equal(plan.forward(wl["x"]).float().cpu().numpy(), yp)
+    # the separate pool kernel (fuse_pool=2) gives the same bits
+    p2 = engine.plan_from_workload(wl, force_mode=1, force_brick=brick, fuse_pool=2)
+    assert p2.launches_per_run == 2
+    np.testing.assert_array_equal(p2.forward(wl["x"]).float().cpu().numpy(), yp)
