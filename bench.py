@@ -140,8 +140,7 @@ def measure_config(cfg, dev, K, flush, peaks, mode=None, cudnn=True):
         flush()
         a.record()
         plan.brickify(x, out=xb)
-        plan.run(xb, yb)
-        plan.unbrickify(yb, out=y)
+        plan.run_dense(xb, out=y)
         b.record()
     torch.cuda.synchronize()
     step_ms = statistics.mean(a.elapsed_time(b) for a, b in ev)
@@ -328,15 +327,14 @@ def main():
 
     def step():
         plan.brickify(x_dense, out=xb)
-        plan.run(xb, yb)
-        plan.unbrickify(yb, out=y_dense)
+        plan.run_dense(xb, out=y_dense)
 
     for _ in range(max(3, args.warmup)):
         step()
     torch.cuda.synchronize()
 
     K = args.steps
-    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(K)]
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(K)]
     sv = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(K)]
     with ClockSampler(local) as clk:
         # keep the GPU loaded (untimed) while the clock sampler starts, so that its samples cover the
@@ -356,8 +354,7 @@ def main():
             flush_l2()                         # L2 flush, outside the timed events
             sv[k][0].record(stream)
             plan.brickify(x_dense, out=xb)
-            plan.run(xb, yb)
-            plan.unbrickify(yb, out=y_dense)
+            plan.run_dense(xb, out=y_dense)   # merged subgraphs, unbrickify fused into the last epilogue
             sv[k][1].record(stream)
         torch.cuda.synchronize()
         if world > 1:
@@ -370,10 +367,12 @@ def main():
             e[0].record(stream)
             plan.brickify(x_dense, out=xb)
             e[1].record(stream)
-            plan.run(xb, yb)
+            plan.run_dense(xb, out=y_dense)    # the merged subgraph launch(es) of the step: roofline kernel time
             e[2].record(stream)
-            plan.unbrickify(yb, out=y_dense)
+            plan.run(xb, yb)                   # (breakdown only) bricked-output run + separate unbrickify
             e[3].record(stream)
+            plan.unbrickify(yb, out=y_dense)
+            e[4].record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -403,8 +402,7 @@ def main():
         a.record(stream)
         x_dev2.copy_(x_host, non_blocking=True)
         plan.brickify(x_dev2, out=xb)
-        plan.run(xb, yb)
-        plan.unbrickify(yb, out=y_dense)
+        plan.run_dense(xb, out=y_dense)
         y_host.copy_(y_dense, non_blocking=True)
         b.record(stream)
         b.synchronize()
@@ -447,10 +445,10 @@ def main():
                 "traffic": traffic if len(sg) == 1 else None, "traffic_source": traffic_src, "peak_source": peak_src,
                 "kernel": f"{kname} ({'/'.join(sorted({g['mode'] for g in sg}))})",
                 "algorithmic_flops_per_launch": flops, "kernel_ms_mean": kernel_ms, "hbm_frac_of_step_bytes": None}
-    # step bytes: brickify (read+write) + subgraphs (in, out) + unbrickify (read+write)
+    # step bytes
     in_b = x_dense.numel() * x_dense.element_size()
     out_b = y_dense.numel() * y_dense.element_size()
-    step_bytes = 3 * in_b + 3 * out_b
+    step_bytes = 3 * in_b + out_b   # brickify (read + write), merged (read bricks, write the dense output)
     roofline["hbm_frac_of_step_bytes"] = step_bytes / (statistics.mean(step_ms) / 1e3) / 1e9 / float(peaks["hbm_gbs"])
 
     # ---- layer-by-layer cuDNN reference (context): torch conv2d, channels_last bf16
@@ -478,7 +476,7 @@ def main():
                 extra[name] = {"error": f"{type(e).__name__}: {str(e)[:300]}"}
 
     if rank == 0:
-        launches = K * (2 + plan.launches_per_run)
+        launches = K * (1 + plan.launches_per_run)   # brickify + the merged launches (unbrickify fused)
         line = {
             "metric": "images/sec merged conv chain per B200", "value": value, "unit": "images/s",
             "n_gpus": world, "steps": K, "warmup": max(3, args.warmup), "ms_per_step": total_ms / K,
@@ -486,7 +484,7 @@ def main():
             "data": "synthetic (seeded N(0,1) inputs, He-normal weights; workloads.py)",
             "config": {"workload": workload_desc(wl), "images_per_gpu": wl["N"], "global_batch": wl["N"] * world,
                        "mode": sg[0]["mode"], "mode_model": sg[0]["mode_model"], "delta": round(sg[0]["delta"], 4),
-                       "kernel": sg[0]["kernel"], "subgraphs": len(sg), "step": "brickify + merged subgraph + unbrickify",
+                       "kernel": sg[0]["kernel"], "subgraphs": len(sg), "step": "brickify + merged subgraph with unbrickify fused into its last epilogue (bdl_run_dense)",
                        "l2": "flushed between timed steps (256 MiB write + 256 MiB read, outside the events)",
                        "timing": "value/ms_per_step: K steps with events only around each step; breakdown_ms and "
                                  "roofline: a second K-step pass with events between the kernels",
@@ -503,9 +501,10 @@ def main():
             "roofline": roofline,
             "cpu_baseline": cpu,
             "breakdown_ms": {"brickify": statistics.mean(e[0].elapsed_time(e[1]) for e in ev),
-                             "merged_subgraph": kernel_ms,
-                             "unbrickify": statistics.mean(e[2].elapsed_time(e[3]) for e in ev),
-                             "step_with_events_between_kernels": statistics.mean(e[0].elapsed_time(e[3]) for e in ev)},
+                             "merged_subgraph_dense_out": kernel_ms,
+                             "merged_subgraph_bricked_out": statistics.mean(e[2].elapsed_time(e[3]) for e in ev),
+                             "separate_unbrickify": statistics.mean(e[3].elapsed_time(e[4]) for e in ev),
+                             "step_with_events_between_kernels": statistics.mean(e[0].elapsed_time(e[2]) for e in ev)},
             "cudnn_layer_by_layer": cudnn,
             "other_configs": extra,
         }
@@ -536,7 +535,7 @@ def e2e_pipelined(plan, wl, x_dense, y_dense, xb, yb, K, dev):
     b.record(pipe.s_h2d)
     b.synchronize()
     ms = a.elapsed_time(b)
-    plan.unbrickify(plan.run(plan.brickify(x_dense, out=xb), yb), out=y_dense)
+    plan.run_dense(plan.brickify(x_dense, out=xb), out=y_dense)
     torch.cuda.synchronize(dev)
     if not torch.equal(pipe.y_host[(K - 1) % pipe.slots], y_dense.cpu()):
         raise RuntimeError("pipelined e2e output differs from the device-timed path")
@@ -572,7 +571,7 @@ def bench_spatial(args, world, rank, local, dev):
         step()
     torch.cuda.synchronize()
     K = args.steps
-    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(K)]
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(K)]
     with ClockSampler(local) as clk:
         t_end = time.time() + 0.5
         while time.time() < t_end:

@@ -192,6 +192,13 @@ bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void
 bdl_status bdl_run(bdl_plan *p, const void *in_bricked, void *out_bricked, void *workspace,
                    void *stream);
 
+/* Merged execution of the whole graph with the output written as dense NC(D)HW (out_dense: DEVICE,
+ * N x C x D x H x W of the graph output, dtype of the graph).  Same work as bdl_run + bdl_unbrickify: the last
+ * subgraph's epilogue writes the dense layout directly when its kernel supports it (the tcgen05 band kernel in
+ * memoized / unmerged mode: unbrickify fused into the last layer's stores, L742-743), otherwise its bricked output
+ * is staged in the workspace and one unbrickify launch follows. */
+bdl_status bdl_run_dense(bdl_plan *p, const void *in_bricked, void *out_dense, void *workspace, void *stream);
+
 /* Number of kernels bdl_run enqueues (for launch accounting). */
 int32_t bdl_plan_launches_per_run(const bdl_plan *p);
 

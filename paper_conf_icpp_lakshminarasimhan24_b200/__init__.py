@@ -66,6 +66,7 @@ _SIGS = {
     "bdl_plan_prepare": (_i32, [_vp, _vp, _vp]),
     "bdl_run_subgraph": (_i32, [_vp, _i32, _vp, _vp, _vp, _vp]),
     "bdl_run": (_i32, [_vp, _vp, _vp, _vp, _vp]),
+    "bdl_run_dense": (_i32, [_vp, _vp, _vp, _vp, _vp]),
     "bdl_plan_launches_per_run": (_i32, [_vp]),
     "bdl_plan_counters": (_i32, [_vp, _i32, _vp, _vp, _P(ctypes.c_uint64)]),
     "bdl_plan_destroy": (None, [_vp]),

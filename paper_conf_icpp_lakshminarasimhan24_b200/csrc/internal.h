@@ -100,6 +100,7 @@ struct bdl_plan {
     bdl_layout in_layout, out_layout;
     bdl_plan_opts opts;
     int64_t ws_bytes = 0;
+    int64_t final_off = 0;      // workspace: bricked graph output for bdl_run_dense's unbrickify fallback
     int num_sms = 148;
     int64_t l2_bytes = 0;
     bool prepared = false;

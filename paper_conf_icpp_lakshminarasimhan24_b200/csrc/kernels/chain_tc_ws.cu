@@ -71,6 +71,8 @@ struct Params {
     CUtensorMap tm_out[kMaxLayers];   // 5-D row maps of each layer's output (TMA epilogue stores)
     CUtensorMap tm_res;               // 5-D row map of the residual tensor
     int row_tma;                      // 1: tm_row usable (bricks of a row are consecutive in memory)
+    __nv_bfloat16 *dense;             // non-null: the LAST layer writes dense NCHW [N][C][H][W] here instead of bricks
+                                      // (unbrickify fused into the epilogue, bdl_run_dense)
     int L, C;
     int H, W;
     int Tb, Tw, Wt;
@@ -679,7 +681,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                 // wait until the epilogue warps have written this task's results
                 asm volatile("bar.sync 2, %0;" ::"n"(32 * (kEpiWarps + 1)) : "memory");
                 prev_sync = gtime();
-                if (lane == 0 && RL::TMA) {
+                if (lane == 0 && RL::TMA && !(p.dense && l == p.L - 1)) {   // (dense output: the epilogue wrote it)
                     for (int i = 0; i < p.Tb && y0 + i < Hg; i++) {
                         const int y = y0 + i;
                         for (int kb = 0; kb < C / 64; kb++)
@@ -719,6 +721,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                 }
                 __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(ly.out.ptr);
                 const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(p.res.ptr);
+                const bool dn = p.dense != nullptr && l == p.L - 1;
                 const int Wg = ly.out.nb[3] << p.lBw;  // bricked grid extents
                 const float *bl = bias_s + l * C;
                 for (int tile = tile0; tile < ((p.dbg & 2) ? 0 : p.ntl); tile += 4) {
@@ -781,7 +784,16 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                                 }
                                 o = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
                             }
-                            if constexpr (RL::TMA) {
+                            if (dn) {
+                                // dense NCHW output: lanes hold consecutive pixels of a row, so each channel's store
+                                // of the warp is one contiguous segment
+                                if (kind == 2) {
+                                    const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&o);
+                                    __nv_bfloat16 *q = p.dense + (((long long)n * C + k * 8) * p.H + y) * p.W + x;
+#pragma unroll
+                                    for (int e = 0; e < 8; e++) q[(long long)e * p.H * p.W] = h[e];
+                                }
+                            } else if constexpr (RL::TMA) {
                                 if (kind) *sp = o;
                             } else {
                                 if (kind) dst[k] = o;
@@ -963,12 +975,12 @@ static bool encode_row_map(CUtensorMap *tm, const TView &v, int nseg) {
 }
 
 bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out, const TView *res,
-                              unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged) {
+                              unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged, void *dense) {
     WsGeom g;
-    if (!ws_geometry(p, sg, g))  // wide channel counts: the synchronous band kernel
-        return launch_tc_subgraph(p, sg, in, out, res, wsp, s, launches);
+    if (!ws_geometry(p, sg, g)) return fail(BDL_EUNSUPPORTED, "tcgen05 ws kernel: tile does not fit on chip");
     ws::Params P;
     memset(&P, 0, sizeof(P));
+    P.dense = (__nv_bfloat16 *)dense;
     const Layer &f = p->layers[sg.first];
     const int L = sg.last - sg.first + 1;
     P.L = L;
@@ -1008,8 +1020,8 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
         P.task_base[j] = sg.task_base[j];
     }
     if (P.C % 64 == 0) {
-        if (in.bmap || out.bmap || (res && res->bmap))  // the TMA epilogue needs consecutive bricks per row
-            return launch_tc_subgraph(p, sg, in, out, res, wsp, s, launches);
+        if (in.bmap || out.bmap || (res && res->bmap))  // the TMA epilogue needs consecutive bricks per row (planner)
+            return fail(BDL_EUNSUPPORTED, "tcgen05 ws kernel: a BrickMap needs the generic kernel");
         P.row_tma = 1;
         for (int j = 0; j < L; j++)
             if (!encode_row_map(&P.tm_out[j], P.layer[j].out, g.Tw >> P.lBw))
@@ -1042,7 +1054,7 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
                 tcap = cap;
             }
             cudaMemsetAsync(tbuf, 0, (size_t)cap * 12 * 8, s);
-            cudaMemsetAsync(wsp + sg.counter_off + 5 * 8, 0, 8, s);
+            cudaMemsetAsync(wsp + sg.counter_off + 7 * 8, 0, 8, s);   // trace index
             P.trace = tbuf;
             P.trace_cap = cap;
             ws_trace_buf = tbuf;

@@ -155,6 +155,7 @@ using namespace bdl;
 static bool tc_eligible(const bdl_plan *p, const Subgraph &sg) {
     if (p->in_layout.dtype != BDL_BF16) return false;
     if (p->in_layout.Bn != 1 || !sg.chain) return false;
+    if (p->in_layout.brickmap) return false;   // the band kernels' TMA rows need the identity BrickMap
     const Layer &f = p->layers[sg.first];
     int C = f.L.cin;
     if (!(C == 16 || C == 32 || C == 64 || C == 128)) return false;
@@ -509,6 +510,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             sg.order_off = sg.norder ? take(sg.norder * 4) : -1;
         }
     }
+    p->final_off = take(p->out_layout.total_bytes);   // bdl_run_dense: bricked output when the last kernel cannot write dense
     p->ws_bytes = align_up(off, 256);
     *out = p;
     return BDL_OK;

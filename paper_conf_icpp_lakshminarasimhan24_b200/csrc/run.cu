@@ -18,7 +18,8 @@ bdl_status launch_pack_tc(const bdl_layer &l, void *w_out, cudaStream_t s);
 bdl_status launch_tc_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out,
                               const TView *res, unsigned char *ws, cudaStream_t s, int *launches);
 bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out, const TView *res,
-                              unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged);
+                              unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged, void *dense);
+bdl_status launch_unbrickify(const bdl_layout *l, const void *src, void *dst, cudaStream_t s);
 int tc_launches(const bdl_plan *p, const Subgraph &sg);
 bdl_status launch_pack_gen(const bdl_plan *p, const Subgraph &sg, int j, void *w_out, cudaStream_t s);
 bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TView> &srcv, const TView &out,
@@ -70,8 +71,13 @@ bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream) {
     return BDL_OK;
 }
 
-bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void *out_bricked, void *workspace,
-                            void *stream) {
+}  // extern "C"
+
+// Run subgraph i; dense != NULL (last subgraph only): write the graph output as dense NC(D)HW there when the
+// subgraph's kernel can (*dense_done = 1), else into out_bricked as usual (*dense_done = 0).
+static bdl_status run_subgraph_impl(bdl_plan *p, int32_t i, const void *in_bricked, void *out_bricked, void *workspace,
+                                    void *stream, void *dense, int *dense_done) {
+    if (dense_done) *dense_done = 0;
     if (!p || i < 0 || i >= (int)p->sgs.size()) return fail(BDL_EINVAL, "bdl_run_subgraph: bad plan or index");
     if (!p->prepared || p->prepared_ws != workspace)
         return fail(BDL_EINVAL, "bdl_run_subgraph: call bdl_plan_prepare with this workspace first");
@@ -104,10 +110,35 @@ bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void
     if (kern == KERNEL_TC_BAND) {
         const bool single = sg.first == sg.last;
         if (sg.mode == BDL_MODE_PADDED && !single) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
-        return launch_ws_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches,
-                                  sg.mode == BDL_MODE_UNMERGED || single);
+        if (dense && dense_done) *dense_done = 1;
+        return launch_ws_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches, sg.mode == BDL_MODE_UNMERGED || single,
+                                  dense);
     }
     return launch_brick_subgraph(p, sg, vin, vout, res, ws, s, &launches);
+}
+
+extern "C" {
+
+bdl_status bdl_run_subgraph(bdl_plan *p, int32_t i, const void *in_bricked, void *out_bricked, void *workspace,
+                            void *stream) {
+    return run_subgraph_impl(p, i, in_bricked, out_bricked, workspace, stream, nullptr, nullptr);
+}
+
+bdl_status bdl_run_dense(bdl_plan *p, const void *in_bricked, void *out_dense, void *workspace, void *stream) {
+    if (!p || !out_dense) return fail(BDL_EINVAL, "bdl_run_dense: NULL argument");
+    if (!p->prepared || p->prepared_ws != workspace)
+        return fail(BDL_EINVAL, "bdl_run_dense: call bdl_plan_prepare with this workspace first");
+    unsigned char *ws = (unsigned char *)workspace;
+    void *final_b = ws + p->final_off;   // the bricked graph output, when the last kernel cannot write dense
+    const int n = (int)p->sgs.size();
+    for (int i = 0; i < n; i++) {
+        int done = 0;
+        bdl_status st = run_subgraph_impl(p, i, in_bricked, final_b, workspace, stream, i == n - 1 ? out_dense : nullptr,
+                                          &done);
+        if (st != BDL_OK) return st;
+        if (i == n - 1 && !done) return bdl_unbrickify(&p->out_layout, final_b, out_dense, stream);
+    }
+    return BDL_OK;
 }
 
 bdl_status bdl_run(bdl_plan *p, const void *in_bricked, void *out_bricked, void *workspace, void *stream) {

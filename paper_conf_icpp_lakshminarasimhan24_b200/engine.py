@@ -168,6 +168,16 @@ class Plan:
                                      ctypes.c_void_p(bricked_out.data_ptr()), ctypes.c_void_p(self.ws_ptr),
                                      _stream_handle(stream)))
 
+    def run_dense(self, bricked_in, out=None, stream=None):
+        """Merged execution writing the dense NC(D)HW output (bdl_run_dense: unbrickify fused into the last
+        subgraph's epilogue where its kernel supports it)."""
+        lo = self.out_layout
+        out = out if out is not None else torch.empty((lo.N, lo.C, lo.D, lo.H, lo.W), dtype=self.tdtype,
+                                                      device=self.device)
+        check(lib().bdl_run_dense(self.h, ctypes.c_void_p(bricked_in.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                  ctypes.c_void_p(self.ws_ptr), _stream_handle(stream)))
+        return out
+
     def forward(self, x, stream=None):
         """Dense NC(D)HW -> dense output: brickify, every merged subgraph, unbrickify."""
         return self.unbrickify(self.run(self.brickify(x, stream=stream), stream=stream), stream=stream)
@@ -178,8 +188,7 @@ class Plan:
             self._fw_xb = self.alloc_bricked(self.in_layout)
             self._fw_yb = self.alloc_bricked(self.out_layout)
         self.brickify(x, out=self._fw_xb, stream=stream)
-        self.run(self._fw_xb, self._fw_yb, stream=stream)
-        return self.unbrickify(self._fw_yb, out=out, stream=stream)
+        return self.run_dense(self._fw_xb, out=out, stream=stream)
 
     def counters(self, i=0, stream=None):
         arr = (ctypes.c_uint64 * 4)()
@@ -256,8 +265,7 @@ class HostPipeline:
                 self.s_cmp.wait_event(d2h_done[sl])            # D2H of request k - S has read y_dev[sl]
             self.plan.brickify(self.x_dev[sl], out=self.xb, stream=self.s_cmp)
             x_free[sl].record(self.s_cmp)
-            self.plan.run(self.xb, self.yb, stream=self.s_cmp)
-            self.plan.unbrickify(self.yb, out=self.y_dev[sl], stream=self.s_cmp)
+            self.plan.run_dense(self.xb, out=self.y_dev[sl], stream=self.s_cmp)
             cmp_done[sl].record(self.s_cmp)
             with torch.cuda.stream(self.s_d2h):
                 self.s_d2h.wait_event(cmp_done[sl])

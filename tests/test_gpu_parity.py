@@ -262,3 +262,27 @@ def test_full_batch_sampled(cfg):
     for n in (0, N - 1):
         y1 = p1.forward(wl["x"][n:n + 1]).float().cpu().numpy()
         np.testing.assert_array_equal(y[n:n + 1], y1)
+
+
+@pytest.mark.parametrize("case", ["cfg2_memo", "cfg2_unmerged", "cfg2_padded", "cfg2_c32", "cfg4_small", "cfg1_f32"])
+def test_run_dense_equals_run_then_unbrickify(case):
+    """bdl_run_dense (unbrickify fused into the last subgraph's epilogue where its kernel supports it, else staged +
+    one unbrickify launch) gives exactly the bytes of bdl_run + bdl_unbrickify (the layout conversion is exact,
+    L742-743), and repeated runs stay equal (run state on the device)."""
+    if case.startswith("cfg2"):
+        kw = dict(N=3, H=24, W=40) if case != "cfg2_c32" else dict(N=2, C=32, H=20, W=24)
+        wl = workloads.make_workload("cfg2", **kw)
+        mode = {"cfg2_memo": "memoized", "cfg2_unmerged": "unmerged", "cfg2_padded": "padded"}.get(case, "memoized")
+    elif case == "cfg4_small":
+        wl, mode = workloads.make_workload("cfg4", N=2, H=64, W=64), None
+    else:
+        wl, mode = workloads.make_workload("cfg1", N=2, H=24, W=16), "memoized"
+    plan = engine.plan_from_workload(wl)
+    if mode:
+        plan.set_mode(mode)
+    xb = plan.brickify(wl["x"])
+    ref = plan.unbrickify(plan.run(xb))
+    for _ in range(3):
+        got = plan.run_dense(xb)
+        assert torch.equal(got, ref), case
+    assert rel_err(got.float().cpu().numpy(), oracle_out(wl)) <= TOL[wl["dtype"]]
