@@ -60,6 +60,20 @@ def _compile(src: str, verbose: bool) -> str:
     return obj
 
 
+MB_SRC = os.path.join(CSRC, "microbench", "atomics.cu")
+MB_LIB = os.path.join(PKG, "libbdl_microbench.so")
+
+
+def build_microbench(force: bool = False) -> str:
+    """Memo-atomics microbenchmark library (measurement infrastructure, tools/microbench.py)."""
+    if force or not os.path.exists(MB_LIB) or os.path.getmtime(MB_LIB) < os.path.getmtime(MB_SRC):
+        cmd = [NVCC, *FLAGS, "-shared", MB_SRC, "-o", MB_LIB, "-lcudart"]
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError(f"nvcc failed for microbench:\n{r.stderr}")
+    return MB_LIB
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(BUILD, exist_ok=True)
     if force:
@@ -72,6 +86,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr}")
+    build_microbench(force)
     return LIB
 
 
