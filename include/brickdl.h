@@ -91,6 +91,10 @@ typedef struct bdl_layer {
     const void *w;               /* DEVICE weights [cout][kd][kh][kw][cin] in the graph dtype; read only
                                     by bdl_plan_prepare (may be freed afterwards).  NULL for maxpool. */
     const float *bias;           /* DEVICE [cout] fp32 or NULL; read only by bdl_plan_prepare */
+    int32_t dil[3];              /* dilation (d, h, w); <= 0 reads as 1.  Input extent of a window d(k-1)+1 (SURVEY Q19,
+                                    the mergeable set of L378-385).  Tensor-core kernels: stride 1 when dilated. */
+    int32_t groups;              /* <= 1: dense conv; g > 1: grouped / depthwise (g = cin) conv, weights
+                                    [cout][kd][kh][kw][cin/g]; runs on the CUDA-core brick kernels (not a dense contraction) */
 } bdl_layer;
 
 /* Static-analysis knobs (§3.3); bdl_plan_opts_default gives the paper's values. */

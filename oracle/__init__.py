@@ -88,8 +88,17 @@ def round_bf16(x):
     return a
 
 
-def conv(x, w, bias=None, stride=(1, 1, 1), pad=(0, 0, 0), dil=(1, 1, 1)):
-    """Direct convolution (cross-correlation), fp64.  x [N,Ci,D,H,W] (or 4-D), w [Co,Ci,kd,kh,kw]."""
+def conv(x, w, bias=None, stride=(1, 1, 1), pad=(0, 0, 0), dil=(1, 1, 1), groups=1):
+    """Direct convolution (cross-correlation), fp64.  x [N,Ci,D,H,W] (or 4-D), w [Co,Ci/groups,kd,kh,kw].
+    groups > 1 (grouped / depthwise conv): by definition, output channels [g*Co/G, (g+1)*Co/G) are the conv of
+    input channels [g*Ci/G, (g+1)*Ci/G) alone -- G independent oracle_conv calls on the channel slices."""
+    if groups > 1:
+        xa, wa = np.asarray(x, dtype=np.float64), np.asarray(w, dtype=np.float64)
+        ci, co = xa.shape[1] // groups, wa.shape[0] // groups
+        ys = [conv(xa[:, g * ci:(g + 1) * ci], wa[g * co:(g + 1) * co],
+                   None if bias is None else np.asarray(bias, np.float64)[g * co:(g + 1) * co], stride, pad, dil)
+              for g in range(groups)]
+        return np.ascontiguousarray(np.concatenate(ys, axis=1))
     four = np.asarray(x).ndim == 4
     x = _as5(x)
     w = np.asarray(w, dtype=np.float64)
@@ -193,7 +202,7 @@ def run_graph(layers, x, weights, biases, dtype="bf16", keep_all=False):
         src = x if l["input"] == -1 else outs[l["input"]]
         if l["kind"] == "conv":
             y = conv(src, np.asarray(w, dtype=np.float64), None if b is None else np.asarray(b, np.float64),
-                     stride=l["stride"], pad=l["pad"])
+                     stride=l["stride"], pad=l["pad"], dil=l.get("dil", (1, 1, 1)), groups=l.get("groups", 1))
         else:
             y = maxpool(src, l["k"], l["stride"], l["pad"])
         res = None

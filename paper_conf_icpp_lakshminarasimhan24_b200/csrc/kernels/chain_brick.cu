@@ -61,25 +61,27 @@ __device__ __forceinline__ float eval_elem(const GLayer &ly, const BrickSrc<T> &
                                            int n, int d, int h, int w, int co) {
     const bool pool = ly.kind == BDL_OP_MAXPOOL;
     float acc = pool ? -INFINITY : (ly.bias ? ly.bias[co] : 0.f);
+    // grouped conv (groups = cin: depthwise): output channel co reads the cin/groups input channels of its group
+    const int cin_g = ly.cin / ly.groups, c0 = pool ? 0 : (co / (ly.cout / ly.groups)) * cin_g;
     int tap = 0;
     for (int td = 0; td < ly.k[1]; td++)
         for (int th = 0; th < ly.k[2]; th++)
             for (int tw = 0; tw < ly.k[3]; tw++, tap++) {
-                int id = d * ly.s[1] - ly.p[1] + td;
-                int ih = h * ly.s[2] - ly.p[2] + th;
-                int iw = w * ly.s[3] - ly.p[3] + tw;
+                int id = d * ly.s[1] - ly.p[1] + td * ly.dl[1];
+                int ih = h * ly.s[2] - ly.p[2] + th * ly.dl[2];
+                int iw = w * ly.s[3] - ly.p[3] + tw * ly.dl[3];
                 if (!inside4(ly.in_ext, n, id, ih, iw)) continue;
                 if (pool) {
                     float v = FromRegion ? rs.p[rs.idx(n, id, ih, iw) + co] : to_f(bs.base(n, id, ih, iw)[co]);
                     acc = fmaxf(acc, v);
                 } else {
-                    const float *wp = ly.w + (long long)tap * ly.cin * ly.cout + co;
+                    const float *wp = ly.w + (long long)tap * cin_g * ly.cout + co;
                     if (FromRegion) {
-                        const float *xp = rs.p + rs.idx(n, id, ih, iw);
-                        for (int ci = 0; ci < ly.cin; ci++) acc = fmaf(wp[(long long)ci * ly.cout], xp[ci], acc);
+                        const float *xp = rs.p + rs.idx(n, id, ih, iw) + c0;
+                        for (int ci = 0; ci < cin_g; ci++) acc = fmaf(wp[(long long)ci * ly.cout], xp[ci], acc);
                     } else {
-                        const T *xp = bs.base(n, id, ih, iw);
-                        for (int ci = 0; ci < ly.cin; ci++) acc = fmaf(wp[(long long)ci * ly.cout], to_f(xp[ci]), acc);
+                        const T *xp = bs.base(n, id, ih, iw) + c0;
+                        for (int ci = 0; ci < cin_g; ci++) acc = fmaf(wp[(long long)ci * ly.cout], to_f(xp[ci]), acc);
                     }
                 }
             }
@@ -157,7 +159,7 @@ __global__ void __launch_bounds__(256) padded_chain_kernel(GChain g) {
                 const GLayer &ly = g.layer[j];
                 for (int i = 0; i < 4; i++) {
                     int nlo = lo[i] * ly.s[i] - ly.p[i];
-                    int next = (ext[i] - 1) * ly.s[i] + ly.k[i];
+                    int next = (ext[i] - 1) * ly.s[i] + ly.dl[i] * (ly.k[i] - 1) + 1;
                     lo[i] = nlo;
                     ext[i] = next;
                 }
@@ -202,7 +204,7 @@ __device__ __forceinline__ DepBox dep_box(const GChain &g, int l, long long b) {
     DepBox box;
     for (int i = 0; i < 4; i++) {
         int a = lo[i] * ly.s[i] - ly.p[i];
-        int e = (lo[i] + ext[i] - 1) * ly.s[i] - ly.p[i] + ly.k[i];  // exclusive
+        int e = (lo[i] + ext[i] - 1) * ly.s[i] - ly.p[i] + ly.dl[i] * (ly.k[i] - 1) + 1;  // exclusive
         a = max(a, 0);
         e = min(e, ly.in_ext[i]);
         box.lo[i] = a / src.B[i];
@@ -439,12 +441,13 @@ __global__ void pack_weights_f32_kernel(const T *__restrict__ w, float *__restri
 // ---------------------------------------------------------------------------------------------- host
 bdl_status launch_pack_f32(const bdl_layer &l, int dtype, float *w_out, float *b_out, cudaStream_t s) {
     int taps = l.k[0] * l.k[1] * l.k[2];
-    long long total = (long long)l.cout * taps * l.cin;
+    const int cin_g = l.cin / (l.groups > 1 ? l.groups : 1);   // grouped weights [cout][taps][cin/groups]
+    long long total = (long long)l.cout * taps * cin_g;
     int grid = (int)std::min<long long>((total + 255) / 256, 4096);
     if (dtype == BDL_F32)
-        pack_weights_f32_kernel<float><<<grid, 256, 0, s>>>((const float *)l.w, w_out, l.cout, taps, l.cin, l.bias, b_out);
+        pack_weights_f32_kernel<float><<<grid, 256, 0, s>>>((const float *)l.w, w_out, l.cout, taps, cin_g, l.bias, b_out);
     else
-        pack_weights_f32_kernel<__nv_bfloat16><<<grid, 256, 0, s>>>((const __nv_bfloat16 *)l.w, w_out, l.cout, taps, l.cin, l.bias, b_out);
+        pack_weights_f32_kernel<__nv_bfloat16><<<grid, 256, 0, s>>>((const __nv_bfloat16 *)l.w, w_out, l.cout, taps, cin_g, l.bias, b_out);
     BDL_CUDA_CHECK_LAUNCH("pack_weights");
     return BDL_OK;
 }
@@ -464,8 +467,11 @@ bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &i
         G.kind = ly.L.kind;
         G.cin = ly.L.cin;
         G.cout = ly.L.cout;
-        G.k[0] = 1; G.s[0] = 1; G.p[0] = 0;
-        for (int d = 0; d < 3; d++) { G.k[d + 1] = ly.L.k[d]; G.s[d + 1] = ly.L.stride[d]; G.p[d + 1] = ly.L.pad[d]; }
+        G.k[0] = 1; G.s[0] = 1; G.p[0] = 0; G.dl[0] = 1;
+        for (int d = 0; d < 3; d++) {
+            G.k[d + 1] = ly.L.k[d]; G.s[d + 1] = ly.L.stride[d]; G.p[d + 1] = ly.L.pad[d]; G.dl[d + 1] = ly.L.dil[d];
+        }
+        G.groups = ly.L.groups;
         for (int d = 0; d < 4; d++) { G.in_ext[d] = ly.in_ext[d]; G.out_ext[d] = ly.out_ext[d]; }
         G.relu = ly.L.relu;
         G.w = ly.L.kind == BDL_OP_CONV ? (const float *)(ws + ly.w_off) : nullptr;

@@ -67,6 +67,7 @@ struct LayerP {
     int relu, has_res;
     int cin, cout;
     int k[3], s[3], pd[3];    // (d, h, w)
+    int dl[3], ke[3];         // dilation; window input extent ke = dl*(k-1) + 1 (dilated convs: SURVEY Q19)
     int in_ext[3], out_ext[3];
     int grid[3];              // output bricked-grid extents (D, H, W)
     int Tb, Tw, Wp;
@@ -198,16 +199,16 @@ __host__ __device__ __forceinline__ DepRange dep_range_src(const LayerP &C, cons
     r.nnc = P.nnc;
     int lo, hi;
     lo = max(0, c.d * C.s[0] - C.pd[0]);
-    hi = min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.k[0] - 1);
+    hi = min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.ke[0] - 1);
     r.d0 = lo;
     r.nd = max(0, hi - lo + 1);
     const int y0 = tile_y0(C, c.ty), x0 = tile_x0(C, c.tx);
     lo = max(0, y0 * C.s[1] - C.pd[1]);
-    hi = min(C.in_ext[1] - 1, (y0 + C.Tb - 1) * C.s[1] - C.pd[1] + C.k[1] - 1);
+    hi = min(C.in_ext[1] - 1, (y0 + C.Tb - 1) * C.s[1] - C.pd[1] + C.ke[1] - 1);
     r.b0 = lo / P.Tb;
     r.nb = hi >= lo ? hi / P.Tb - r.b0 + 1 : 0;
     lo = max(0, x0 * C.s[2] - C.pd[2]);
-    hi = min(C.in_ext[2] - 1, (x0 + C.Tw - 1) * C.s[2] - C.pd[2] + C.k[2] - 1);
+    hi = min(C.in_ext[2] - 1, (x0 + C.Tw - 1) * C.s[2] - C.pd[2] + C.ke[2] - 1);
     r.x0 = lo / P.Tw;
     r.nx = hi >= lo ? hi / P.Tw - r.x0 + 1 : 0;
     return r;
@@ -297,7 +298,7 @@ __host__ __device__ inline void region_of(const LayerP *ly, int L, const int PB[
                 lo[d] = hi[d] = 0;
                 continue;
             }
-            const int nlo = lo[d] * J.s[d] - J.pd[d], nhi = (h - 1) * J.s[d] - J.pd[d] + J.k[d];
+            const int nlo = lo[d] * J.s[d] - J.pd[d], nhi = (h - 1) * J.s[d] - J.pd[d] + J.ke[d];
             lo[d] = nlo > 0 ? nlo : 0;
             hi[d] = nhi < J.in_ext[d] ? nhi : J.in_ext[d];
             if (hi[d] < lo[d]) hi[d] = lo[d];
@@ -616,7 +617,7 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
     }
     const int lane = tid & 31, w = tid >> 5;
     const int lkc = L.lkc, kc = 1 << lkc;
-    const int nrow = L.k[0] * L.in_rows;
+    const int nrow = L.ke[0] * L.in_rows;
     const int z0 = T.d * L.s[0] - L.pd[0];
     const int y0 = T.y0 * L.s[1] - L.pd[1];
     const int x0 = T.x0 * L.s[2] - L.pd[2];
@@ -778,7 +779,10 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             t1 = 2 * u + 1 < L.k[2] ? tap + 1 : -1;
         }
         auto tap_px = [&](int tp) {
-            const int s = tp % L.k[2], r = (tp / L.k[2]) % L.k[1], a = tp / (L.k[2] * L.k[1]);
+            // tap (a, r, s) reads input offset (a*dl0, r*dl1, s*dl2) of the output position: its polyphase block and
+            // row / column inside the block
+            const int s = (tp % L.k[2]) * L.dl[2], r = ((tp / L.k[2]) % L.k[1]) * L.dl[1],
+                      a = (tp / (L.k[2] * L.k[1])) * L.dl[0];
             return a * L.plane_px + ((r % L.s[1]) * L.s[2] + (s % L.s[2])) * L.blk_px + (r / L.s[1]) * L.Wp + s / L.s[2];
         };
         uint32_t aoff, lbo;
@@ -1228,11 +1232,15 @@ static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out,
     if (l.kind != BDL_OP_CONV) return false;
     G.amode = gen_amode(l.cin);
     if (G.amode < 0 || l.cout % 16 != 0) return false;
+    if (l.groups > 1) return false;   // grouped / depthwise: not a dense contraction (CUDA-core kernels)
     for (int d = 0; d < 3; d++) {
         G.k[d] = l.k[d];
         G.s[d] = l.stride[d];
         G.pd[d] = l.pad[d];
+        G.dl[d] = l.dil[d] > 1 ? l.dil[d] : 1;
+        G.ke[d] = G.dl[d] * (G.k[d] - 1) + 1;
         if (G.k[d] > 7 || (G.s[d] != 1 && G.s[d] != 2)) return false;
+        if (G.dl[d] > 1 && G.s[d] != 1) return false;   // dilated layers: stride 1
         G.in_ext[d] = ly.in_ext[d + 1];
         G.out_ext[d] = ly.out_ext[d + 1];
     }
@@ -1295,8 +1303,8 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
             cand.Tw = Tw;
             cand.Tpb = G.pool ? Ub : 0;
             cand.Tpw = G.pool ? Uw : 0;
-            cand.in_rows = (Tb - 1) * G.s[1] + G.k[1];
-            cand.in_cols = (Tw - 1) * G.s[2] + G.k[2];
+            cand.in_rows = (Tb - 1) * G.s[1] + G.ke[1];
+            cand.in_cols = (Tw - 1) * G.s[2] + G.ke[2];
             cand.Wp = (cand.in_cols + G.s[2] - 1) / G.s[2];
             cand.rb = (cand.in_rows + G.s[1] - 1) / G.s[1];
             cand.blk_px = cand.rb * cand.Wp;
@@ -1304,9 +1312,9 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
             const int M = Tb * cand.Wp;
             cand.ntl = (M + 127) / 128;
             if (cand.ntl * G.Nc > 256) continue;       // double-buffered accumulators
-            const int max_tap = (G.k[0] - 1) * cand.plane_px + (cand.nblk - 1) * cand.blk_px +
-                                ((G.k[1] - 1) / G.s[1]) * cand.Wp + (G.k[2] - 1) / G.s[2];
-            int rows = std::max(G.k[0] * cand.plane_px, max_tap + cand.ntl * 128);
+            const int max_tap = (G.ke[0] - 1) * cand.plane_px + (cand.nblk - 1) * cand.blk_px +
+                                ((G.ke[1] - 1) / G.s[1]) * cand.Wp + (G.ke[2] - 1) / G.s[2];
+            int rows = std::max(G.ke[0] * cand.plane_px, max_tap + cand.ntl * 128);
             rows = (rows + 7) / 8 * 8;
             if (G.amode == gen::AM_PLANES) rows += 1;   // odd plane stride: conflict-free loader stores
             if (G.amode == gen::AM_SW64) rows = (rows + 1 + 7) / 8 * 8;   // room for the alignment offset pxo
@@ -1671,9 +1679,9 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
             }
             if (D.ns == 0) {   // reads an external tensor: how far down its input frame the window reaches
                 const gen::TaskC c = gen::decode(C, t);
-                const int z = std::min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.k[0] - 1);
-                const int y = std::min(C.in_ext[1] - 1, (gen::tile_y0(C, c.ty) + C.Tb - 1) * C.s[1] - C.pd[1] + C.k[1] - 1);
-                const int x = std::min(C.in_ext[2] - 1, (gen::tile_x0(C, c.tx) + C.Tw - 1) * C.s[2] - C.pd[2] + C.k[2] - 1);
+                const int z = std::min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.ke[0] - 1);
+                const int y = std::min(C.in_ext[1] - 1, (gen::tile_y0(C, c.ty) + C.Tb - 1) * C.s[1] - C.pd[1] + C.ke[1] - 1);
+                const int x = std::min(C.in_ext[2] - 1, (gen::tile_x0(C, c.tx) + C.Tw - 1) * C.s[2] - C.pd[2] + C.ke[2] - 1);
                 k = std::max(k, ((double)std::max(z, 0) * C.in_ext[1] + std::max(y, 0)) * C.in_ext[2] + std::max(x, 0)) /
                     frame;
             }

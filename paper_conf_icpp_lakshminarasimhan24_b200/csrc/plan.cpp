@@ -14,7 +14,9 @@
 namespace bdl {
 
 // Output extent of a layer along one dim: floor((I + 2p - (k-1) - 1)/s) + 1.
-static int out_extent(int I, int k, int s, int p) { return (I + 2 * p - (k - 1) - 1) / s + 1; }
+static int out_extent(int I, int k, int s, int p, int d) { return (I + 2 * p - d * (k - 1) - 1) / s + 1; }
+// Input extent of one window, d(k-1) + 1.  Layers are normalized at partition time (dil >= 1).
+static int keff(const bdl_layer &l, int dim) { return (l.dil[dim] > 1 ? l.dil[dim] : 1) * (l.k[dim] - 1) + 1; }
 
 static int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 
@@ -38,7 +40,7 @@ static void regions_dag(const std::vector<Layer> &ly, int first, int last, int d
     for (int j = L - 1; j >= 0; j--) {
         if (olo[j] >= ohi[j]) continue;   // output not needed inside the subgraph (a live-out only)
         const bdl_layer &l = ly[first + j].L;
-        int k = dim == 0 ? 1 : l.k[dim - 1], s = dim == 0 ? 1 : l.stride[dim - 1], p = dim == 0 ? 0 : l.pad[dim - 1];
+        int k = dim == 0 ? 1 : keff(l, dim - 1), s = dim == 0 ? 1 : l.stride[dim - 1], p = dim == 0 ? 0 : l.pad[dim - 1];
         int64_t lo, hi;
         if (halo) {
             lo = olo[j] * s - p;               // input extent I = s(O-1) + k (Q19)
@@ -162,7 +164,8 @@ static bool tc_eligible(const bdl_plan *p, const Subgraph &sg) {
     int nsp = p->in_layout.nsp;
     for (int j = sg.first; j <= sg.last; j++) {
         const bdl_layer &l = p->layers[j].L;
-        if (l.kind != BDL_OP_CONV || l.cin != C || l.cout != C) return false;
+        if (l.kind != BDL_OP_CONV || l.cin != C || l.cout != C || l.groups != 1) return false;
+        if (l.dil[0] != 1 || l.dil[1] != 1 || l.dil[2] != 1) return false;
         for (int d = 0; d < 3; d++) {
             bool spatial = (nsp == 3) || d > 0;
             int k = spatial ? 3 : 1, pp = spatial ? 1 : 0;
@@ -211,7 +214,17 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
     for (int i = 0; i < nlayers; i++) {
         Layer &L = p->layers[i];
         L.L = layers[i];
-        const bdl_layer &l = layers[i];
+        for (int d = 0; d < 3; d++) L.L.dil[d] = std::max(1, L.L.dil[d]);
+        L.L.groups = std::max(1, L.L.groups);
+        const bdl_layer &l = L.L;
+        if (l.groups > 1 && (l.kind != BDL_OP_CONV || l.cin % l.groups || l.cout % l.groups)) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": groups must divide cin and cout (convs only)");
+        }
+        if (l.kind == BDL_OP_MAXPOOL && (l.dil[0] != 1 || l.dil[1] != 1 || l.dil[2] != 1)) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EUNSUPPORTED, "layer " + std::to_string(i) + ": dilated pooling");
+        }
         if (l.kind != BDL_OP_CONV && l.kind != BDL_OP_MAXPOOL) {
             bdl_plan_destroy(p);
             return fail(BDL_EUNSUPPORTED, "layer " + std::to_string(i) + ": unknown op kind");
@@ -220,7 +233,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             bdl_plan_destroy(p);
             return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": input must be an earlier layer or -1");
         }
-        int cin_expected = l.input == -1 ? (int)in->C : layers[l.input].cout;
+        int cin_expected = l.input == -1 ? (int)in->C : p->layers[l.input].L.cout;
         if (l.cin != cin_expected || l.cout <= 0 || (l.kind == BDL_OP_MAXPOOL && l.cout != l.cin)) {
             bdl_plan_destroy(p);
             return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": channel count mismatch");
@@ -239,7 +252,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
                 bdl_plan_destroy(p);
                 return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": bad kernel/stride/pad");
             }
-            L.out_ext[d + 1] = out_extent(L.in_ext[d + 1], l.k[d], l.stride[d], l.pad[d]);
+            L.out_ext[d + 1] = out_extent(L.in_ext[d + 1], l.k[d], l.stride[d], l.pad[d], l.dil[d]);
             if (L.out_ext[d + 1] <= 0) {
                 bdl_plan_destroy(p);
                 return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": empty output");
@@ -265,7 +278,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
     auto fits_brick = [&](int j) {
         const bdl_layer &l = p->layers[j].L;
         for (int d = 0; d < 3; d++)
-            if (l.k[d] > Bx[d + 1] || l.pad[d] > Bx[d + 1]) return false;
+            if (keff(l, d) > Bx[d + 1] || l.pad[d] > Bx[d + 1]) return false;
         return true;
     };
     auto consumed_after = [&](int m, int end) {
@@ -288,6 +301,11 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             branch = branch || (j > first && p->layers[j].L.input != j - 1) || (r != BDL_NO_RESIDUAL && r >= first) ||
                      (j < end && consumed_after(j, end));
             if (!(j == end && is_pool(p->layers[j]))) all_gen = all_gen && gen_layer_supported(p, j);
+            // bf16: grouped (depthwise) convs run on the CUDA-core kernels, dense ones on the tensor cores: the two
+            // do not share a subgraph (the whole subgraph runs on one kernel)
+            if (in->dtype == BDL_BF16 && j > first && p->layers[j].L.kind == BDL_OP_CONV &&
+                p->layers[j - 1].L.kind == BDL_OP_CONV && (p->layers[j].L.groups > 1) != (p->layers[j - 1].L.groups > 1))
+                return false;
         }
         if (branch && !(dag_ok && all_gen)) return false;
         // footprint (L605-614): concurrently resident bricks x padded regions + weights.  The persistent kernels hold
@@ -307,7 +325,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
         fp = (int64_t)nconc * vol_sum * in->elem_bytes;
         for (int j = first; j <= end; j++) {
             const bdl_layer &l = p->layers[j].L;
-            fp += (int64_t)l.cout * l.cin * l.k[0] * l.k[1] * l.k[2] * in->elem_bytes;
+            fp += (int64_t)l.cout * (l.cin / l.groups) * l.k[0] * l.k[1] * l.k[2] * in->elem_bytes;
         }
         return fp <= budget;
     };
@@ -445,7 +463,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
     for (auto &L : p->layers) {
         if (L.L.kind != BDL_OP_CONV) continue;
         int64_t taps = (int64_t)L.L.k[0] * L.L.k[1] * L.L.k[2];
-        L.w_off = take(taps * L.L.cin * L.L.cout * 4);
+        L.w_off = take(taps * (L.L.cin / L.L.groups) * L.L.cout * 4);
         L.b_off = take((int64_t)L.L.cout * 4);
     }
     for (auto &sg : p->sgs)

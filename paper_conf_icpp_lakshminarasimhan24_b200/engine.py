@@ -64,6 +64,8 @@ class Plan:
             a.cin, a.cout = l["cin"], l["cout"]
             for d in range(3):
                 a.k[d], a.stride[d], a.pad[d] = l["k"][d], l["stride"][d], l["pad"][d]
+                a.dil[d] = l.get("dil", (1, 1, 1))[d]
+            a.groups = l.get("groups", 1)
             a.relu = int(l["relu"])
             a.input = l["input"]
             a.residual = BDL_NO_RESIDUAL if l["residual"] is None else l["residual"]

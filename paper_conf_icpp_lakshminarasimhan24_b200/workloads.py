@@ -43,15 +43,15 @@ CONFIGS = {
 _CFG_NUM = {"cfg1": 1, "cfg2": 2, "cfg3": 3, "cfg4": 4, "cfg5": 5}
 
 
-def _conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2):
+def _conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2, dil=1, groups=1):
     if p is None:
-        p = (k - 1) // 2
+        p = dil * (k - 1) // 2
     if nsp == 3:
-        kk, ss, pp = (k, k, k), (s, s, s), (p, p, p)
+        kk, ss, pp, dd = (k, k, k), (s, s, s), (p, p, p), (dil, dil, dil)
     else:
-        kk, ss, pp = (1, k, k), (1, s, s), (0, p, p)
+        kk, ss, pp, dd = (1, k, k), (1, s, s), (0, p, p), (1, dil, dil)
     return dict(kind="conv", cin=cin, cout=cout, k=kk, stride=ss, pad=pp, relu=relu,
-                input=inp, residual=res, wscale=wscale)
+                input=inp, residual=res, wscale=wscale, dil=dd, groups=groups)
 
 
 def _pool(c, k, s, p):
@@ -106,10 +106,10 @@ def make_layers(cfg: str, C: int | None = None, nlayers: int | None = None):
 
 
 def layer_out_shape(layer, D, H, W):
-    """Output spatial extent of one layer: floor((I + 2p - (k-1) - 1)/s) + 1 per dim."""
+    """Output spatial extent of one layer: floor((I + 2p - d(k-1) - 1)/s) + 1 per dim."""
     out = []
-    for I, k, s, p in zip((D, H, W), layer["k"], layer["stride"], layer["pad"]):
-        out.append((I + 2 * p - (k - 1) - 1) // s + 1)
+    for I, k, s, p, d in zip((D, H, W), layer["k"], layer["stride"], layer["pad"], layer.get("dil", (1, 1, 1))):
+        out.append((I + 2 * p - d * (k - 1) - 1) // s + 1)
     return tuple(out)
 
 
@@ -134,9 +134,10 @@ def make_workload(cfg: str, N=None, C=None, D=None, H=None, W=None, nlayers=None
     return wl
 
 
-def conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2):
-    """Layer dict of a conv (public form of the graph builder used by the configurations)."""
-    return _conv(cin, cout, k, s, p, relu, inp, res, wscale, nsp)
+def conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2, dil=1, groups=1):
+    """Layer dict of a conv (public form of the graph builder used by the configurations).  dil: dilation;
+    groups: grouped conv (groups = cin: depthwise), weights [cout, cin/groups, k...]."""
+    return _conv(cin, cout, k, s, p, relu, inp, res, wscale, nsp, dil, groups)
 
 
 def pool(c, k, s, p):
@@ -164,8 +165,9 @@ def make_graph_workload(layers, N, C, D, H, W, nsp, brick, dtype, seed=0, input_
             biases.append(None)
             continue
         kd, kh, kw = l["k"]
-        fan_in = l["cin"] * kd * kh * kw
-        w = torch.randn(l["cout"], l["cin"], kd, kh, kw, generator=gw, dtype=torch.float32)
+        cin_g = l["cin"] // l.get("groups", 1)
+        fan_in = cin_g * kd * kh * kw
+        w = torch.randn(l["cout"], cin_g, kd, kh, kw, generator=gw, dtype=torch.float32)
         w = w * (math.sqrt(2.0 / fan_in) * l["wscale"])
         if bf16:
             w = w.to(torch.bfloat16).to(torch.float32)

@@ -62,6 +62,11 @@ GRAPHS = {
     "pool_fused_stem_3x3s2p1": ([W.conv(3, 64, 7, 2, 3), W.pool(64, 3, 2, 1)], 2, 3, 1, 38, 42, (1, 1, 8, 8)),
     "pool_fused_chain_3x3s2p1": ([W.conv(64, 64, 1), W.conv(64, 64, 3), W.pool(64, 3, 2, 1)], 2, 64, 1, 27, 30,
                                  (1, 1, 8, 8)),
+    # dilated convs (DRN / DeepCAM style, L378-385): taps d apart, halo d(k-1)/2 per layer
+    "dilated_chain_d2": ([W.conv(64, 64, 3, dil=2), W.conv(64, 64, 3, dil=2)], 2, 64, 1, 26, 21, (1, 1, 8, 8)),
+    "dilated_mixed_d1_d3": ([W.conv(32, 64, 3), W.conv(64, 64, 3, dil=3), W.conv(64, 64, 1)], 1, 32, 1, 30, 27,
+                            (1, 1, 8, 8)),
+    "dilated_3d_d2": ([W.conv(32, 32, 3, nsp=3, dil=2), W.conv(32, 32, 3, nsp=3)], 1, 32, 12, 13, 10, (1, 4, 4, 4)),
     # 3x3x3 x 64 channels = 108 k-steps per layer (the Fig 10/11 microbenchmark layers)
     "sw128_3d_c64": ([W.conv(64, 64, 3, nsp=3), W.conv(64, 64, 3, nsp=3)], 1, 64, 10, 12, 9, (1, 4, 4, 4)),
     "sw128_3d_c64_valid": ([W.conv(64, 64, 3, 1, 0, nsp=3), W.conv(64, 64, 3, 1, 0, nsp=3)], 1, 64, 13, 12, 14,
@@ -213,3 +218,27 @@ def test_gen_padded_fused_pool_blocks(brick):
     p2 = engine.plan_from_workload(wl, force_mode=1, force_brick=brick, fuse_pool=2)
     assert p2.launches_per_run == 2
     np.testing.assert_array_equal(p2.forward(wl["x"]).float().cpu().numpy(), yp)
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_grouped_and_depthwise(dtype):
+    """Grouped and depthwise convs (MobileNet-style separable block: depthwise 3x3 -> pointwise 1x1; L378-385) run on
+    the CUDA-core brick kernels (not a dense contraction); bf16 graphs cut the subgraph between the depthwise and the
+    dense layers so the pointwise convs stay on the tensor cores.  Every mode against the oracle."""
+    layers = [W.conv(32, 32, 3, groups=32), W.conv(32, 64, 1), W.conv(64, 64, 3, groups=8),
+              W.conv(64, 64, 3, groups=64, dil=2), W.conv(64, 32, 1, res=None)]
+    wl = W.make_graph_workload(layers, 2, 32, 1, 19, 22, 2, (1, 1, 8, 8), dtype, seed=29)
+    ref = oracle.run_graph(wl["layers"], wl["x"].numpy(), wl["weights"], wl["biases"], dtype=dtype)
+    plan = engine.plan_from_workload(wl, force_mode=2)
+    sgs = plan.subgraphs()
+    if dtype == "bf16":
+        kinds = {(s["first"], s["last"]): s["kernel"] for s in sgs}
+        assert any(k == "tcgen05 generic" for k in kinds.values()), kinds      # the pointwise convs
+        assert any(k == "cuda-core brick" for k in kinds.values()), kinds      # the depthwise / grouped convs
+    outs = {}
+    for mode in ("memoized", "padded", "unmerged"):
+        plan.set_mode(mode)
+        outs[mode] = plan.forward(wl["x"]).float().cpu().numpy()
+        assert rel_err(outs[mode], ref) <= (TOL if dtype == "bf16" else 1e-5), (mode, rel_err(outs[mode], ref))
+    np.testing.assert_array_equal(outs["memoized"], outs["unmerged"])
+    np.testing.assert_array_equal(outs["memoized"], outs["padded"])

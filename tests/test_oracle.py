@@ -349,3 +349,38 @@ def test_p6_dag_resnet50_prefix_vs_torch():
     with pytest.raises(AssertionError):
         yb = oracle.run_graph(bad, wl["x"].numpy(), wl["weights"], wl["biases"], dtype="f64")
         np.testing.assert_allclose(yb[:, :, 0], ref.numpy(), rtol=1e-12, atol=1e-12)
+
+
+# ---------------------------------------------------------------- dilated and grouped convolution (N2)
+@pytest.mark.parametrize("dil,groups,s,p", [(2, 1, 1, 2), (3, 1, 1, 0), (1, 4, 1, 1), (2, 4, 2, 2), (1, 8, 1, 1)])
+def test_p6_torch_conv2d_dilated_grouped(dil, groups, s, p):
+    """Dilated / grouped / depthwise convs (the mergeable set beyond dense convs, L378-385) against torch fp64."""
+    x = rng.standard_normal((2, 8, 13, 11))
+    w = rng.standard_normal((8, 8 // groups, 3, 3))
+    b = rng.standard_normal(8)
+    y = oracle.conv(x, w, bias=b, stride=(s, s), pad=(p, p), dil=(dil, dil), groups=groups)
+    ref = torch.nn.functional.conv2d(torch.from_numpy(x), torch.from_numpy(w), torch.from_numpy(b), stride=s,
+                                     padding=p, dilation=dil, groups=groups).numpy()
+    np.testing.assert_allclose(y, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_p1_delta_input_dilated():
+    """Delta input: a dilated kernel's taps land d apart: y[oh, ow] = w[r, s] where oh - p + d*r = h0."""
+    x = np.zeros((1, 1, 9, 9))
+    x[0, 0, 4, 4] = 1.0
+    w = rng.standard_normal((1, 1, 3, 3))
+    y = oracle.conv(x, w, pad=(2, 2), dil=(2, 2))
+    expect = np.zeros_like(y)
+    for r in range(3):
+        for c in range(3):
+            expect[0, 0, 4 + 2 - 2 * r, 4 + 2 - 2 * c] = w[0, 0, r, c]
+    np.testing.assert_array_equal(y, expect)
+
+
+def test_depthwise_is_per_channel():
+    """groups = C: each output channel is the 1-channel conv of its own input channel (brute force per channel)."""
+    x = rng.standard_normal((1, 3, 7, 6))
+    w = rng.standard_normal((3, 1, 3, 3))
+    y = oracle.conv(x, w, pad=(1, 1), groups=3)
+    for c in range(3):
+        np.testing.assert_array_equal(y[:, c:c + 1], oracle.conv(x[:, c:c + 1], w[c:c + 1], pad=(1, 1)))
