@@ -32,7 +32,25 @@ __global__ void __launch_bounds__(128, 1) mma_loop(int iters, unsigned long long
     if (wid == 0) {
         const uint32_t tb = __shfl_sync(0xffffffff, tbase, 0);
         const uint32_t abase = smem_u32(A) >> 4, bbase = smem_u32(B) >> 4;
-        if (MODE == 7 || MODE == 8) {
+        if (MODE == 9 || MODE == 10) {
+            // generic-kernel cfg5 shape on the 64-B swizzled layout (AM_SW64): pixel rows of 64 B, Wp = 18, plane 288
+            // rows, 27 taps x 2 k-steps, ntl = 2 (mode 9) or 1 (mode 10)
+            const uint64_t a0 = umma_desc_sw64(0, 512), b0 = umma_desc_noswz(0, N * 16, 128);
+            const int ntl = MODE == 9 ? 2 : 1;
+            for (int it = 0; it < iters; it++) {
+                for (int tap = 0; tap < 27; tap++) {
+                    const uint32_t px = (tap / 9) * 288 + ((tap / 3) % 3) * 18 + tap % 3;
+#pragma unroll
+                    for (int kk = 0; kk < 2; kk++) {
+                        uint64_t bd = b0 | ((bbase + (tap * 2 + kk) * (N * 2)) & 0x3FFF);
+                        for (int tl = 0; tl < ntl; tl++) {
+                            uint64_t ad = a0 | ((abase + (px + tl * 128) * 4 + kk * 2) & 0x3FFF);
+                            mma_bf16_elect(tb + (it & 1) * 128 + tl * N, ad, bd, ID, 1);
+                        }
+                    }
+                }
+            }
+        } else if (MODE == 7 || MODE == 8) {
             // generic-kernel cfg5 shape: chunk planes of 497 (7) or 496 (8) rows, 27 taps x 2 k-steps, ntl = 1
             const uint32_t rowsP = MODE == 7 ? 497 : 496;
             const uint32_t LBO7 = rowsP * 16;
@@ -143,7 +161,7 @@ template <int N, int MODE> void run(int sms, const uint8_t *gw) {
     cudaEventRecord(b); cudaEventSynchronize(b);
     float ms; cudaEventElapsedTime(&ms, a, b);
     unsigned long long h[256]; cudaMemcpy(h, d, sms * 8, cudaMemcpyDeviceToHost);
-    double n_mma = (double)iters * (MODE >= 7 ? 54 : MODE >= 4 ? 12 : 16);
+    double n_mma = (double)iters * (MODE == 9 ? 108 : MODE >= 7 ? 54 : MODE >= 4 ? 12 : 16);
     double flops = n_mma * 2.0 * 128 * N * 16 * sms;
     printf("mode=%d N=%3d  cycles/MMA=%.1f (ideal %d)  chip %.1f TFLOP/s  (%s)\n", MODE, N, h[0] / n_mma, 128 * N / 256,
            flops / (ms * 1e-3) / 1e12, cudaGetErrorString(cudaGetLastError()));
@@ -159,5 +177,6 @@ int main() {
     run<64, 4>(1, gw); run<64, 5>(1, gw); run<64, 6>(1, gw);
     run<192, 0>(sms, gw); run<192, 4>(sms, gw); run<128, 4>(sms, gw); run<256, 4>(sms, gw);
     run<32, 7>(sms, gw); run<32, 8>(sms, gw); run<32, 0>(sms, gw);
+    run<32, 9>(sms, gw); run<32, 10>(sms, gw); run<64, 9>(sms, gw);
     return 0;
 }
