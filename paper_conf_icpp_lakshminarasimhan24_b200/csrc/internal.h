@@ -44,6 +44,7 @@ struct Layer {
     bdl_layer L;               // as given
     int in_ext[4], out_ext[4]; // (n, d, h, w)
     int64_t w_off = -1, b_off = -1;  // workspace offsets of packed weights / bias
+    int64_t gen_w_off = -1;          // generic-kernel packed weights of a band-kernel subgraph (its padded mode)
     int64_t tc_w_off = -1;           // tcgen05 packed weights (band kernels: [tap][cin/8][cout][8];
                                      // generic kernel: [nc][kb][kstep][2][Nc][8])
 };
@@ -63,6 +64,7 @@ struct Subgraph {
     double delta, delta_first;
     int kernel;                 // KernelKind the subgraph is able to run on
     int gen_layers = 0;         // generic tcgen05 kernel: leading conv layers it runs (a pool tail follows)
+    bool gen_padded = false;    // band-kernel subgraph whose padded mode runs on the generic kernel
     int64_t gen_scr_off = -1;   // generic tcgen05 kernel, padded mode: per-CTA region scratch
     int in_tensor;              // index into Plan::tensors (the first layer's input)
     int out_tensor;

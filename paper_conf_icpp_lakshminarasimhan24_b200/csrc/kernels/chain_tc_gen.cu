@@ -1791,7 +1791,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
         if (sg.res_tensor[j] >= 0) G.res = res[j];
         else if (G.resl >= 0) G.res = outs[G.resl];
         G.relu = ly.L.relu;
-        G.w = (const __nv_bfloat16 *)(wsp + ly.tc_w_off);
+        G.w = (const __nv_bfloat16 *)(wsp + (ly.gen_w_off >= 0 ? ly.gen_w_off : ly.tc_w_off));
         G.bias = (const float *)(wsp + ly.b_off);
         G.task_base = sg.task_base[j];
     }

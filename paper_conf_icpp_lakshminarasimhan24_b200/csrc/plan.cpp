@@ -447,6 +447,11 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
     for (auto &sg : p->sgs) {
         sg.kernel = tc_eligible(p, sg) ? KERNEL_TC_BAND : KERNEL_BRICK;
         if (sg.kernel == KERNEL_BRICK && (sg.gen_layers = gen_conv_layers(p, sg)) > 0) sg.kernel = KERNEL_TC_GEN;
+        // band-kernel chains run PADDED mode on the generic kernel (warp-specialized, measured faster on B200 than
+        // the synchronous band padded kernel: cfg2 0.195 -> see DESIGN.md §8); same per-element K order, so the
+        // modes stay bit-equal
+        if (sg.kernel == KERNEL_TC_BAND && sg.last > sg.first && (sg.gen_layers = gen_conv_layers(p, sg)) > 0)
+            sg.gen_padded = true;
         if (!sg.chain && sg.kernel != KERNEL_TC_GEN) {
             bdl_plan_destroy(p);
             return fail(BDL_EUNSUPPORTED, "partition: a branched subgraph cannot run on the generic kernel");
@@ -475,6 +480,9 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             }
         else if (sg.kernel == KERNEL_TC_GEN)
             for (int j = 0; j < sg.gen_layers; j++) p->layers[sg.first + j].tc_w_off = take(gen_packed_bytes(p, sg, j));
+    for (auto &sg : p->sgs)
+        if (sg.gen_padded)
+            for (int j = 0; j < sg.gen_layers; j++) p->layers[sg.first + j].gen_w_off = take(gen_packed_bytes(p, sg, j));
     for (size_t t = 1; t < p->tensors.size(); t++)
         if (p->tensors[t].ws_off == 0) p->tensors[t].ws_off = take(p->tensors[t].layout.total_bytes);
     for (auto &sg : p->sgs) {
@@ -521,6 +529,9 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             sg.order_host = ws_task_order(p, sg);
             sg.norder = (int64_t)sg.order_host.size();
             sg.order_off = sg.norder ? take(sg.norder * 4) : -1;
+        }
+        if (sg.gen_padded) {
+            if (int64_t sb = gen_scratch_bytes(p, sg)) sg.gen_scr_off = take(sb);
         } else if (sg.kernel == KERNEL_TC_GEN) {
             if (int64_t sb = gen_scratch_bytes(p, sg)) sg.gen_scr_off = take(sb);
             sg.order_host = gen_task_order(p, sg);

@@ -52,6 +52,10 @@ bdl_status bdl_plan_prepare(bdl_plan *p, void *workspace, void *stream) {
     for (auto &sg : p->sgs) {
         for (int j = sg.first; j <= sg.last; j++) {
             const Layer &L = p->layers[j];
+            if (L.gen_w_off >= 0) {
+                bdl_status st = launch_pack_gen(p, sg, j - sg.first, ws + L.gen_w_off, s);
+                if (st != BDL_OK) return st;
+            }
             if (L.tc_w_off < 0) continue;
             bdl_status st = sg.kernel == KERNEL_TC_GEN ? launch_pack_gen(p, sg, j - sg.first, ws + L.tc_w_off, s)
                                                        : launch_pack_tc(L.L, ws + L.tc_w_off, s);
@@ -109,6 +113,11 @@ static bdl_status run_subgraph_impl(bdl_plan *p, int32_t i, const void *in_brick
     }
     if (kern == KERNEL_TC_BAND) {
         const bool single = sg.first == sg.last;
+        if (sg.mode == BDL_MODE_PADDED && !single && sg.gen_padded) {
+            std::vector<TView> srcv(sg.last - sg.first + 1);
+            srcv[0] = vin;
+            return launch_gen_subgraph(p, sg, srcv, vout, res, ws, s, &launches);
+        }
         if (sg.mode == BDL_MODE_PADDED && !single) return launch_tc_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches);
         if (dense && dense_done) *dense_done = 1;
         return launch_ws_subgraph(p, sg, vin, vout, tc_res, ws, s, &launches, sg.mode == BDL_MODE_UNMERGED || single,
