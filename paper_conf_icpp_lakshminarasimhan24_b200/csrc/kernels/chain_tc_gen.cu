@@ -953,6 +953,17 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             const uint32_t d_base = tmem_base + a * p.acc_stride;
             const uint32_t lbo_b = (uint32_t)L.Nc * 16;
             const uint32_t ks_u = (uint32_t)L.Nc * 2;   // 16-B units per k-step of B
+            // issue constants hoisted out of the k-step loop; descriptors advance by 64-bit adds (start-address fields
+            // stay below 2^14 16-B units: shared memory < 256 KB)
+            const int ntl = L.ntl;
+            const uint32_t idesc = L.idesc, dstep = (uint32_t)L.Nc;
+            const uint64_t astep = 128ull * (uint64_t)L.row_u;
+            const bool noswz = L.amode != AM_SW128 && L.amode != AM_SW64;
+            const uint64_t ad_t = L.amode == AM_SW128 ? ptx::umma_desc_sw128(0, 1024)
+                                  : L.amode == AM_SW64 ? ptx::umma_desc_sw64(0, 512)
+                                                       : ptx::umma_desc_noswz(0, 0, 128);
+            const uint64_t bd_t = ptx::umma_desc_noswz(0, lbo_b, 128);
+            const uint32_t *ksl = sh.ks[l];
             for (int kb = 0; kb < L.nkb; kb++, gin++) {
                 const int s = gin % p.nin;
                 pwait(p, &sh.in_full[s], (gin / p.nin) & 1, win);
@@ -967,19 +978,24 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     ptx::tc_fence_after();
                     const uint32_t b_base = ptx::smem_u32(w_ring + (size_t)st * p.w_stride) >> 4;
                     const int q0 = j * L.kpw, q1 = (p.dbg & 1) ? q0 + 1 : min(L.nks, q0 + L.kpw);
-                    for (int q = q0; q < q1; q++) {
-                        const uint32_t ev = sh.ks[l][q];
-                        const uint2 e = make_uint2(ev & 0xFFFF, ev >> 16);
-                        const uint64_t bd = ptx::umma_desc_noswz(0, lbo_b, 128) |
-                                            (uint64_t)((b_base + (q - q0) * ks_u) & 0x3FFF);
-                        uint64_t ad0;
-                        if (L.amode == AM_SW128) ad0 = ptx::umma_desc_sw128(0, 1024);
-                        else if (L.amode == AM_SW64) ad0 = ptx::umma_desc_sw64(0, 512);
-                        else ad0 = ptx::umma_desc_noswz(0, e.y * 16, 128);
-                        for (int tl = 0; tl < L.ntl; tl++) {
-                            const uint64_t ad = ad0 | (uint64_t)((a_base + e.x + tl * 128 * L.row_u) & 0x3FFF);
-                            ptx::mma_bf16_elect(d_base + tl * L.Nc, ad, bd, L.idesc, (kb | q) != 0);
+                    const uint64_t a_d0 = ad_t + a_base;
+                    uint64_t bd = bd_t + b_base;
+                    auto issue = [&](uint64_t ad, uint32_t acc) {
+                        ptx::mma_bf16_elect_nc(d_base, ad, bd, idesc, acc);
+                        if (ntl > 1) ptx::mma_bf16_elect_nc(d_base + dstep, ad + astep, bd, idesc, acc);
+                        if (ntl > 2) ptx::mma_bf16_elect_nc(d_base + 2 * dstep, ad + 2 * astep, bd, idesc, acc);
+                        if (ntl > 3)
+                            for (int tl = 3; tl < ntl; tl++)
+                                ptx::mma_bf16_elect_nc(d_base + tl * dstep, ad + tl * astep, bd, idesc, acc);
+                    };
+                    if (noswz) {
+                        for (int q = q0; q < q1; q++, bd += ks_u) {
+                            const uint32_t ev = ksl[q];
+                            issue((ad_t | ((uint64_t)(ev >> 16) << 16)) + a_base + (ev & 0xFFFF), (kb | q) != 0);
                         }
+                    } else {
+#pragma unroll 4
+                        for (int q = q0; q < q1; q++, bd += ks_u) issue(a_d0 + (ksl[q] & 0xFFFFu), (kb | q) != 0);
                     }
                     ptx::mma_commit_elect(&sh.wempty[st]);
                 }

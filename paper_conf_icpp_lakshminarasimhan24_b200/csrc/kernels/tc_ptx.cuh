@@ -132,6 +132,18 @@ __device__ __forceinline__ void mma_bf16_elect(uint32_t d_tmem, uint64_t a_desc,
         "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
         : "memory");
 }
+// mma_bf16_elect without the memory clobber: operand readiness is ordered by the mbarrier waits and tcgen05 fences
+// issued before the k-step loop, so the compiler may hoist the next k-step's table load and descriptor arithmetic
+// above this issue (the issue chain, not the tensor pipe, bounded small-N layers).
+__device__ __forceinline__ void mma_bf16_elect_nc(uint32_t d_tmem, uint64_t a_desc, uint64_t b_desc, uint32_t idesc,
+                                                  uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p, q;\n\t.reg .b32 e;\n\t"
+        "elect.sync e|p, 0xffffffff;\n\t"
+        "setp.ne.b32 q, %4, 0;\n\t"
+        "@p tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, q;\n\t}" ::"r"(d_tmem),
+        "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate));
+}
 __device__ __forceinline__ void mma_commit_elect(uint64_t *bar) {
     asm volatile(
         "{\n\t.reg .pred p;\n\t.reg .b32 e;\n\t"
