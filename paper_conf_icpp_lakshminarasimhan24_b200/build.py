@@ -33,7 +33,7 @@ FLAGS = [
     "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=default",
     "--expt-relaxed-constexpr",
     "-I", os.path.join(ROOT, "include"),
-]
+] + os.environ.get("BDL_EXTRA_NVCC_FLAGS", "").split()   # e.g. -DBDL_DEBUG for the timing knobs (A/B runs only)
 
 
 def _headers():

@@ -151,13 +151,16 @@ __device__ __forceinline__ int *status_word(const Params &p, int l, long long t)
 }
 
 struct TaskC { int n, d, ty, tx, nc; };
-__host__ __device__ __forceinline__ TaskC decode(const LayerP &L, long long t) {
+// (task ids fit 32 bits, kTaskBits: 32-bit unsigned divisions, several times cheaper than 64-bit ones on the
+// per-task path of the scheduler, loaders and epilogue)
+__host__ __device__ __forceinline__ TaskC decode(const LayerP &L, long long t64) {
     TaskC c;
-    c.nc = (int)(t % L.nnc); t /= L.nnc;
-    c.tx = (int)(t % L.ntx); t /= L.ntx;
-    c.ty = (int)(t % L.nty); t /= L.nty;
-    c.d = (int)(t % L.ntd);
-    c.n = (int)(t / L.ntd);
+    unsigned t = (unsigned)t64, q;
+    q = t / (unsigned)L.nnc; c.nc = (int)(t - q * (unsigned)L.nnc); t = q;
+    q = t / (unsigned)L.ntx; c.tx = (int)(t - q * (unsigned)L.ntx); t = q;
+    q = t / (unsigned)L.nty; c.ty = (int)(t - q * (unsigned)L.nty); t = q;
+    q = t / (unsigned)L.ntd; c.d = (int)(t - q * (unsigned)L.ntd);
+    c.n = (int)q;
     return c;
 }
 
@@ -232,11 +235,12 @@ __host__ __device__ __forceinline__ DepRange dep_range_res(const LayerP &C, cons
 }
 __host__ __device__ __forceinline__ int dep_count(const DepRange &r) { return r.nd * r.nb * r.nx * r.nnc; }
 __host__ __device__ __forceinline__ long long dep_task(const LayerP &P, const DepRange &r, int i) {
-    const int c = r.c0 + i % r.nnc; i /= r.nnc;
-    const int x = r.x0 + i % r.nx; i /= r.nx;
-    const int b = r.b0 + i % r.nb; i /= r.nb;
-    const int d = r.d0 + i;
-    return ((((long long)r.n * P.ntd + d) * P.nty + b) * P.ntx + x) * P.nnc + c;
+    unsigned u = (unsigned)i, q;
+    q = u / (unsigned)r.nnc; const int c = r.c0 + (int)(u - q * (unsigned)r.nnc); u = q;
+    q = u / (unsigned)r.nx; const int x = r.x0 + (int)(u - q * (unsigned)r.nx); u = q;
+    q = u / (unsigned)r.nb; const int b = r.b0 + (int)(u - q * (unsigned)r.nb);
+    const int d = r.d0 + (int)q;
+    return (long long)(((((unsigned)r.n * P.ntd + d) * P.nty + b) * P.ntx + x) * P.nnc + c);
 }
 // All dependencies of (l, t) as one index space: [0, ns) on the input producer, [ns, ns + nr) on the residual's.
 struct Deps {
@@ -343,12 +347,12 @@ __device__ __forceinline__ Tile make_tile(const Params &p, int l, long long t) {
     T.slot = (int)(t & 1);
     T.nc = (int)((t >> 1) & 0xFF);
     int k = (int)((t >> 9) & 0xFFFF);
-    long long P = t >> 25;
+    unsigned P = (unsigned)(t >> 25), q;
     int blk[3];
-    blk[2] = (int)(P % p.npb[2]); P /= p.npb[2];
-    blk[1] = (int)(P % p.npb[1]); P /= p.npb[1];
-    blk[0] = (int)(P % p.npb[0]);
-    T.n = (int)(P / p.npb[0]);
+    q = P / (unsigned)p.npb[2]; blk[2] = (int)(P - q * (unsigned)p.npb[2]); P = q;
+    q = P / (unsigned)p.npb[1]; blk[1] = (int)(P - q * (unsigned)p.npb[1]); P = q;
+    q = P / (unsigned)p.npb[0]; blk[0] = (int)(P - q * (unsigned)p.npb[0]);
+    T.n = (int)q;
     int lo[3], hi[3];
     region_of(p.layer, p.L, p.PB, blk, l, lo, hi);
     const int xs = region_x0(L, lo[2]);
@@ -914,7 +918,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             t = __shfl_sync(0xffffffff, t, 0);
             if (l < 0) break;
             const LayerP &L = p.layer[l];
-            const int nc = p.padded ? (int)((t >> 1) & 0xFF) : (int)(t % L.nnc);
+            const int nc = p.padded ? (int)((t >> 1) & 0xFF) : (int)((unsigned)t % (unsigned)L.nnc);
             const size_t ks_bytes = (size_t)2 * L.Nc * 16;
             const uint8_t *wl = reinterpret_cast<const uint8_t *>(L.w) + (size_t)nc * L.nkb * L.nks * ks_bytes;
             for (int kb = 0; kb < L.nkb; kb++) {
