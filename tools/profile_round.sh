@@ -1,38 +1,34 @@
 #!/bin/bash
-# Round profiling (under gpurun): GPU tests, bench lines of every config, launch list (cold, serialized),
-# one full ncu capture of each hot kernel, compute-sanitizer over the generic kernel.
-# Usage: bash tools/profile_round.sh r01c
-R=${1:-r01}
+# Round profiling (under gpurun): GPU tests, the bench line (all configurations), launch list of the bench command (cold,
+# serialized), one full ncu capture of each hot kernel, ncu DRAM bytes merged vs layer-by-layer, compute-sanitizer.
+# Usage: bash tools/profile_round.sh r02b
+R=${1:-r02}
 cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
-timeout 900 python -m pytest tests -m gpu -q 2>&1 | tail -3 | tee gpurun_out/${R}_pytest_gpu.txt
-timeout 400 python bench.py > gpurun_out/${R}_bench.json 2> gpurun_out/${R}_bench.err; echo bench=$?
-for c in cfg1 cfg3 cfg4 cfg5; do
-  timeout 400 python bench.py --config $c --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/${R}_bench_$c.json 2> gpurun_out/${R}_bench_$c.err
-  echo "$c rc=$?"
-done
+timeout 1200 python -m pytest tests -m gpu -q 2>&1 | tail -3 | tee gpurun_out/${R}_pytest_gpu.txt
+timeout 900 python bench.py > gpurun_out/${R}_bench.json 2> gpurun_out/${R}_bench.err; echo bench=$?
 timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --csv \
-    --log-file gpurun_out/${R}_launches.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-cudnn > /dev/null 2>&1
+    --log-file gpurun_out/${R}_launches.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-cudnn --no-extra > /dev/null 2>&1
 echo launches=$?
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:memo_ws -s 3 -c 1 \
-    -o gpurun_out/${R}_memo_ws python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn > /dev/null 2>&1
+    -o gpurun_out/${R}_memo_ws python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn --no-extra > /dev/null 2>&1
 echo memo=$?
 timeout 600 ncu --set full --clock-control none -k regex:brickify -s 2 -c 2 \
-    -o gpurun_out/${R}_brickify python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn > /dev/null 2>&1
+    -o gpurun_out/${R}_brickify python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn --no-extra > /dev/null 2>&1
 echo brickify=$?
 timeout 600 ncu --set full --clock-control none --import-source on -k gen_kernel -s 2 -c 1 \
-    -o gpurun_out/${R}_gen_cfg5 python bench.py --config cfg5 --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn > /dev/null 2>&1
+    -o gpurun_out/${R}_gen_cfg5 python tools/run_subgraph.py cfg5 0 > /dev/null 2>&1
 echo gen_cfg5=$?
-timeout 600 ncu --set full --clock-control none -k gen_kernel -s 40 -c 1 \
-    -o gpurun_out/${R}_gen_cfg4 python bench.py --config cfg4 --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn > /dev/null 2>&1
+timeout 600 ncu --set full --clock-control none -k gen_kernel -s 10 -c 1 \
+    -o gpurun_out/${R}_gen_cfg4 python tools/run_subgraph.py cfg4 1 > /dev/null 2>&1
 echo gen_cfg4=$?
 for c in cfg3 cfg4 cfg5; do
   timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv \
       --log-file gpurun_out/${R}_launches_$c.csv python bench.py --config $c --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn > /dev/null 2>&1
   echo launches_$c=$?
 done
-CASES='tests/test_gpu_gen.py -k "sw128_chain_grow or planes_3d or s2_1x1_proj or bottleneck_res"'
+CASES='tests/test_gpu_gen.py -k "sw128_chain_grow or planes_3d or s2_1x1_proj or dag_bottlenecks_s1 or pool_fused_stem or dilated_chain_d2"'
 for tool in memcheck synccheck racecheck; do
-  eval timeout 900 compute-sanitizer --tool $tool --print-limit 20 --target-processes all \
+  eval timeout 1200 compute-sanitizer --tool $tool --print-limit 20 --target-processes all \
       python -m pytest $CASES -q -p no:cacheprovider > gpurun_out/${R}_sanitize_gen_$tool.log 2>&1
   echo "sanitize $tool rc=$?"; grep -E "ERROR SUMMARY|passed|failed|RACECHECK SUMMARY" gpurun_out/${R}_sanitize_gen_$tool.log | tail -3
 done
