@@ -541,6 +541,7 @@ __device__ void scheduler(const Params &p, Shared &sh) {
         ok = __shfl_sync(0xffffffff, ok, 0);
         if (!ok) continue;   // already claimed (by a dependent's walk back)
         oks++;
+        __syncwarp();   // every lane is done reading the previous bundle's stack (racecheck)
         if (lane == 0) {
             sh.stk_l[0] = l0;
             sh.stk_t[0] = t0;

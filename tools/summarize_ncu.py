@@ -44,7 +44,8 @@ if os.path.exists(lc):
         tot.setdefault(key, []).append(v)
     summary["launch_list"] = {k: {"count": len(v), "mean_ns": sum(v) / len(v)} for k, v in tot.items()}
     step = [v for k, v in launches if "brickify" in k or "memo_ws" in k]
-    ours = {k: sum(v) for k, v in tot.items() if "bdl::" in k and "pack" not in k}
+    ours = {k: sum(v) for k, v in tot.items()
+            if any(t in k for t in ("bdl::", "memo_ws", "gen_kernel", "brickify", "pool_vec")) and "pack" not in k}
     s = sum(ours.values())
     summary["launch_share_of_step"] = {k: v / s for k, v in ours.items()}
     with open(f"profiles/{R}_launches.csv", "w") as f:
