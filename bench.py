@@ -41,6 +41,8 @@ def parse():
     ap.add_argument("--no-extra", action="store_true",
                     help="skip the other configurations (cfg3/cfg4/cfg5 and cfg2 padded) measured in the default run")
     ap.add_argument("--micro", type=int, default=2, help="strong scaling: micro-batches per rank for the gather overlap")
+    ap.add_argument("--strong", action="store_true",
+                    help="strong scaling with the overlapped output gather (default for cfg4 when WORLD_SIZE > 1)")
     ap.add_argument("--spatial", action="store_true",
                     help="3-D configs: shard ONE volume into depth slabs with a brick-plane halo exchange "
                          "(default for 3-D configs when WORLD_SIZE > 1)")
@@ -302,7 +304,7 @@ def main():
 
     if workloads.CONFIGS[args.config]["nsp"] == 3 and (world > 1 or args.spatial):
         return bench_spatial(args, world, rank, local, dev)
-    if args.config == "cfg4" and world > 1:
+    if args.strong or (args.config == "cfg4" and world > 1):
         return bench_strong(args, world, rank, local, dev)
     wl = workloads.make_workload(args.config, input_seed_offset=rank)
     plan = engine.plan_from_workload(wl, device=dev)
@@ -642,6 +644,10 @@ def bench_strong(args, world, rank, local, dev):
     import torch.distributed as dist
 
     from paper_conf_icpp_lakshminarasimhan24_b200 import engine, parallel, workloads
+    if not dist.is_initialized():   # --strong at N = 1 without torchrun: a one-rank NCCL group (the same code path)
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        dist.init_process_group("nccl", rank=0, world_size=1, device_id=dev)
     full = workloads.make_workload(args.config)
     n_total = full["N"]
     mb, ranges = parallel.micro_batches(n_total, world, args.micro)

@@ -81,18 +81,19 @@ class BatchRunner:
             if not gather:
                 continue
             dst = self.y_all[i * W * mb:(i + 1) * W * mb]
+            coll = W > 1 or (dist.is_available() and dist.is_initialized())   # (world 1 under torchrun: NCCL too)
             if self.cuda:
                 ev = torch.cuda.Event()
                 ev.record()
                 self.comm.wait_event(ev)
                 with torch.cuda.stream(self.comm):
-                    if W > 1:
+                    if coll:
                         dist.all_gather_into_tensor(dst, yi, group=self.group)
                     else:
                         dst.copy_(yi)
                 yi.record_stream(self.comm)
             else:
-                if W > 1:
+                if coll:
                     done.append(dist.all_gather_into_tensor(dst, yi, group=self.group, async_op=True))
                 else:
                     dst.copy_(yi)

@@ -54,3 +54,19 @@ def test_spatial_sharding_full_size_8_slabs():
     got, runners = _sharded(wl, 8, mode)
     assert runners[3].geo.ext_D == 16 + 8 and runners[0].geo.ext_D == 16 + 4
     np.testing.assert_array_equal(got, ref)
+
+
+def test_batch_runner_gather_on_gpu():
+    """Strong-scaling runner on one GPU (world 1, NCCL when a group exists, else a copy): micro-batched merged
+    execution + the gather path reproduce the one-shot plan output bit for bit, in global image order."""
+    wl = workloads.make_workload("cfg4", N=4, H=64, W=64)
+    plan1 = engine.plan_from_workload(wl)
+    ref = plan1.forward(wl["x"])
+    mb_wl = workloads.make_workload("cfg4", N=2, H=64, W=64)
+    plan = engine.plan_from_workload(mb_wl)
+    lo = plan.out_layout
+    run = parallel.BatchRunner(4, (lo.C, lo.D, lo.H, lo.W), 0, 1, micro=2, plan=plan, device="cuda")
+    x_local = wl["x"][run.global_images()].cuda().to(plan.tdtype)
+    y = run.forward(x_local)
+    torch.cuda.synchronize()
+    assert torch.equal(y, ref)
