@@ -68,6 +68,9 @@ struct LayerP {
     int cin, cout;
     int k[3], s[3], pd[3];    // (d, h, w)
     int dl[3], ke[3];         // dilation; window input extent ke = dl*(k-1) + 1 (dilated convs: SURVEY Q19)
+    int stk, Td;              // depth stacking (3-D, k0 = 3): a task computes Td output planes and one MMA of N = up to
+                              // 3 Nc feeds up to three of them from one input plane (stk = 0: Td = 1)
+    uint32_t idesc_s[3];      // stacked MMAs: instruction descriptors for N = Nc, 2 Nc, 3 Nc
     int in_ext[3], out_ext[3];
     int grid[3];              // output bricked-grid extents (D, H, W)
     int Tb, Tw, Wp;
@@ -150,6 +153,18 @@ __device__ __forceinline__ int *status_word(const Params &p, int l, long long t)
     return p.status + p.layer[l].task_base + t;
 }
 
+// K-step q of a layer whose A layout is not tap-paired: the depth tap is the FASTEST index, q = (rs * kpt + kk) * k0 + a
+// (rs = r * k2 + s, kk = 16-channel slice of the K-block).  Every output element then accumulates, per (r, s, kk),
+// the depth taps a = 0, 1, 2 in order -- the order the depth-stacked MMAs of 3-D layers produce (one MMA feeds three
+// output planes from one input plane), so stacked and unstacked execution of a layer give the same bits.
+__host__ __device__ __forceinline__ void kstep_tap(int q, int k0, int k1, int k2, int kpt, int &tap, int &kk) {
+    const int a = q % k0;
+    q /= k0;
+    kk = q % kpt;
+    const int rs = q / kpt;
+    tap = (a * k1 + rs / k2) * k2 + rs % k2;
+}
+
 struct TaskC { int n, d, ty, tx, nc; };
 // (task ids fit 32 bits, kTaskBits: 32-bit unsigned divisions, several times cheaper than 64-bit ones on the
 // per-task path of the scheduler, loaders and epilogue)
@@ -201,10 +216,11 @@ __host__ __device__ __forceinline__ DepRange dep_range_src(const LayerP &C, cons
     r.c0 = 0;
     r.nnc = P.nnc;
     int lo, hi;
-    lo = max(0, c.d * C.s[0] - C.pd[0]);
-    hi = min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.ke[0] - 1);
-    r.d0 = lo;
-    r.nd = max(0, hi - lo + 1);
+    // (tasks of depth-stacked layers cover Td planes: C's planes [c.d*Td, +Td), P's blocks of P.Td planes)
+    lo = max(0, c.d * C.Td * C.s[0] - C.pd[0]);
+    hi = min(C.in_ext[0] - 1, (c.d * C.Td + C.Td - 1) * C.s[0] - C.pd[0] + C.ke[0] - 1);
+    r.d0 = lo / P.Td;
+    r.nd = hi >= lo ? hi / P.Td - r.d0 + 1 : 0;
     const int y0 = tile_y0(C, c.ty), x0 = tile_x0(C, c.tx);
     lo = max(0, y0 * C.s[1] - C.pd[1]);
     hi = min(C.in_ext[1] - 1, (y0 + C.Tb - 1) * C.s[1] - C.pd[1] + C.ke[1] - 1);
@@ -222,8 +238,11 @@ __host__ __device__ __forceinline__ DepRange dep_range_res(const LayerP &C, cons
     r.n = c.n;
     r.c0 = c.nc;     // same cout, same Nc: the same channel chunk
     r.nnc = 1;
-    r.d0 = c.d;
-    r.nd = c.d < C.out_ext[0] ? 1 : 0;
+    {
+        const int dlo = c.d * C.Td, dhi = min(C.out_ext[0], dlo + C.Td) - 1;
+        r.d0 = dlo / R.Td;
+        r.nd = dhi >= dlo ? dhi / R.Td - r.d0 + 1 : 0;
+    }
     int lo = c.ty * C.Tb, hi = min(C.out_ext[1], lo + C.Tb) - 1;
     r.b0 = lo / R.Tb;
     r.nb = hi >= lo ? hi / R.Tb - r.b0 + 1 : 0;
@@ -336,7 +355,7 @@ __device__ __forceinline__ Tile make_tile(const Params &p, int l, long long t) {
     Tile T;
     if (!p.padded) {
         const TaskC c = decode(L, t);
-        T.n = c.n; T.d = c.d; T.y0 = tile_y0(L, c.ty); T.x0 = tile_x0(L, c.tx); T.nc = c.nc;
+        T.n = c.n; T.d = c.d * L.Td; T.y0 = tile_y0(L, c.ty); T.x0 = tile_x0(L, c.tx); T.nc = c.nc;
         T.py0 = c.ty * L.Tpb; T.px0 = c.tx * L.Tpw;
         T.hi[0] = L.grid[0]; T.hi[1] = L.grid[1]; T.hi[2] = L.grid[2];
         T.src_scr = T.dst_scr = 0;
@@ -622,7 +641,7 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
     }
     const int lane = tid & 31, w = tid >> 5;
     const int lkc = L.lkc, kc = 1 << lkc;
-    const int nrow = L.ke[0] * L.in_rows;
+    const int nrow = (L.ke[0] + L.Td - 1) * L.in_rows;   // input planes x rows (Td output planes per task)
     const int z0 = T.d * L.s[0] - L.pd[0];
     const int y0 = T.y0 * L.s[1] - L.pd[1];
     const int x0 = T.x0 * L.s[2] - L.pd[2];
@@ -759,6 +778,20 @@ __device__ __forceinline__ uint32_t pack2(float a, float b) {
     return *reinterpret_cast<uint32_t *>(&v);
 }
 
+// One stacked k-step (not the first: every MMA accumulates), input planes and M tiles unrolled: per input plane i the
+// D column, B row offset and instruction descriptor are loop-invariant (precomputed by the caller), so the issue chain
+// is two 64-bit adds per MMA.
+template <int TD, int NTL>
+__device__ __forceinline__ void issue_stacked_q(uint64_t adq, uint64_t bd, uint32_t d_base, const uint32_t *col,
+                                                const uint64_t *bo, const uint32_t *idn, uint64_t pstep, uint64_t astep,
+                                                uint32_t tstep) {
+#pragma unroll
+    for (int i = 0; i < TD + 2; i++)
+#pragma unroll
+        for (int tl = 0; tl < NTL; tl++)
+            ptx::mma_bf16_elect_nc(d_base + tl * tstep + col[i], adq + i * pstep + tl * astep, bd + bo[i], idn[i], 1u);
+}
+
 // ---------------------------------------------------------------------------------------------- kernel
 __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant__ Params p) {
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -772,11 +805,13 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
     for (int i = threadIdx.x; i < p.L * kMaxKs; i += kThreads) {
         const int l = i / kMaxKs, q = i % kMaxKs;
         const LayerP &L = p.layer[l];
-        if (q >= L.nks) continue;
+        if (q >= (L.stk ? L.nks / L.k[0] : L.nks)) continue;
         int tap, kk = 0, t1 = -1;
-        if (L.amode == AM_SW128) { tap = q / 4; kk = q % 4; }
-        else if (L.amode == AM_SW64) { tap = q / 2; kk = q % 2; }
-        else if (L.amode == AM_PLANES) { const int kpt = (L.cin + 15) / 16; tap = q / kpt; kk = q % kpt; }
+        // stacked 3-D layers: the table holds the k0 = 1 view (r, s, kk); the depth tap picks the input plane at issue
+        const int k0t = L.stk ? 1 : L.k[0];
+        if (L.amode == AM_SW128) kstep_tap(q, k0t, L.k[1], L.k[2], 4, tap, kk);
+        else if (L.amode == AM_SW64) kstep_tap(q, k0t, L.k[1], L.k[2], 2, tap, kk);
+        else if (L.amode == AM_PLANES) kstep_tap(q, k0t, L.k[1], L.k[2], (L.cin + 15) / 16, tap, kk);
         else {   // pair taps (a, r, 2u) and (a, r, 2u+1)
             const int np = (L.k[2] + 1) / 2;
             const int u = q % np, ar = q / np;
@@ -920,17 +955,18 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             if (l < 0) break;
             const LayerP &L = p.layer[l];
             const int nc = p.padded ? (int)((t >> 1) & 0xFF) : (int)((unsigned)t % (unsigned)L.nnc);
-            const size_t ks_bytes = (size_t)2 * L.Nc * 16;
-            const uint8_t *wl = reinterpret_cast<const uint8_t *>(L.w) + (size_t)nc * L.nkb * L.nks * ks_bytes;
+            const size_t ks_bytes = (size_t)2 * (L.stk ? 3 : 1) * L.Nc * 16;   // stacked: three depth taps per k-step
+            const int nqs = L.stk ? L.nks / 3 : L.nks;
+            const uint8_t *wl = reinterpret_cast<const uint8_t *>(L.w) + (size_t)nc * L.nkb * nqs * ks_bytes;
             for (int kb = 0; kb < L.nkb; kb++) {
                 for (int j = 0; j < L.nws; j++, gw++) {
                     const int st = gw % p.nw;
-                    const int q0 = j * L.kpw, nq = min(L.kpw, L.nks - q0);
+                    const int q0 = j * L.kpw, nq = min(L.kpw, nqs - q0);
                     const uint32_t bytes = (uint32_t)(nq * ks_bytes);
                     if (gw >= (uint32_t)p.nw) pwait(p, &sh.wempty[st], ((gw / p.nw) - 1) & 1, ww);
                     if (ptx::elect_one()) {
                         ptx::mbar_arrive_expect_tx(&sh.wfull[st], bytes);
-                        ptx::bulk_g2s(w_ring + (size_t)st * p.w_stride, wl + ((size_t)kb * L.nks + q0) * ks_bytes, bytes,
+                        ptx::bulk_g2s(w_ring + (size_t)st * p.w_stride, wl + ((size_t)kb * nqs + q0) * ks_bytes, bytes,
                                       &sh.wfull[st]);
                     }
                     __syncwarp();
@@ -956,8 +992,9 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             if (seq >= (uint32_t)p.nacc) pwait(p, &sh.acc_empty[a], ((seq / p.nacc) - 1) & 1, wacc);
             ptx::tc_fence_after();
             const uint32_t d_base = tmem_base + a * p.acc_stride;
-            const uint32_t lbo_b = (uint32_t)L.Nc * 16;
-            const uint32_t ks_u = (uint32_t)L.Nc * 2;   // 16-B units per k-step of B
+            const uint32_t nbr = (uint32_t)(L.stk ? 3 : 1) * L.Nc;   // B rows per k-step (stacked: three depth taps)
+            const uint32_t lbo_b = nbr * 16;
+            const uint32_t ks_u = nbr * 2;   // 16-B units per k-step of B
             // issue constants hoisted out of the k-step loop; descriptors advance by 64-bit adds (start-address fields
             // stay below 2^14 16-B units: shared memory < 256 KB)
             const int ntl = L.ntl;
@@ -982,9 +1019,63 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     pwait(p, &sh.wfull[st], (gw / p.nw) & 1, wwt);
                     ptx::tc_fence_after();
                     const uint32_t b_base = ptx::smem_u32(w_ring + (size_t)st * p.w_stride) >> 4;
-                    const int q0 = j * L.kpw, q1 = (p.dbg & 1) ? q0 + 1 : min(L.nks, q0 + L.kpw);
+                    const int q0 = j * L.kpw, q1 = (p.dbg & 1) ? q0 + 1 : min(L.stk ? L.nks / 3 : L.nks, q0 + L.kpw);
                     const uint64_t a_d0 = ad_t + a_base;
                     uint64_t bd = bd_t + b_base;
+                    if (L.stk) {
+                        // depth-stacked 3-D layer: per k-step (r, s, kk), input plane i feeds output planes o = i - a for the
+                        // depth taps a in [alo, ahi]: ONE MMA with N = (ahi - alo + 1) Nc, B = those taps' weights side
+                        // by side, D = the planes' accumulators, laid out at columns (Td - 1 - o) Nc so they are contiguous
+                        // and ascending.  The first k-step gives each plane's first product (a = 0) its own MMA without
+                        // accumulate.  Per output element the order is (r, s, kk) outer, a inner -- the unstacked order.
+                        const int Td = L.Td, Nc = L.Nc;
+                        const uint64_t pstep = (uint64_t)L.plane_px * (uint64_t)L.row_u;
+                        const uint32_t tstep = (uint32_t)(Td * Nc);
+                        auto issue_n = [&](uint64_t ad, uint64_t bdd, int o_hi, int na, uint32_t acc) {
+                            const uint32_t col = (uint32_t)((Td - 1 - o_hi) * Nc);
+                            const uint32_t idn = L.idesc_s[na - 1];
+                            for (int tl = 0; tl < ntl; tl++)
+                                ptx::mma_bf16_elect_nc(d_base + tl * tstep + col, ad + tl * astep, bdd, idn, acc);
+                        };
+                        // per input plane: D column, B row offset, descriptor (loop-invariant over the k-steps)
+                        uint32_t colv[6], idnv[6];
+                        uint64_t bov[6];
+#pragma unroll
+                        for (int i = 0; i < 6; i++) {
+                            const int alo = max(0, i - Td + 1), ahi = min(2, i);
+                            colv[i] = (uint32_t)((Td - 1 - (i - alo)) * Nc);
+                            bov[i] = (uint64_t)(alo * Nc);
+                            idnv[i] = L.idesc_s[max(0, min(2, ahi - alo))];
+                        }
+                        const bool fast = !noswz && (Td == 1 || Td == 2 || Td == 4) && (ntl == 1 || ntl == 2);
+                        for (int q = q0; q < q1; q++, bd += ks_u) {
+                            const uint32_t ev = ksl[q];
+                            const uint64_t adq = noswz ? (ad_t | ((uint64_t)(ev >> 16) << 16)) + a_base + (ev & 0xFFFF)
+                                                       : a_d0 + (ev & 0xFFFFu);
+                            const bool first = (kb | q) == 0;
+                            if (fast && !first) {
+                                if (Td == 1 && ntl == 1) issue_stacked_q<1, 1>(adq, bd, d_base, colv, bov, idnv, pstep, astep, tstep);
+                                else if (Td == 1) issue_stacked_q<1, 2>(adq, bd, d_base, colv, bov, idnv, pstep, astep, tstep);
+                                else if (Td == 2 && ntl == 1) issue_stacked_q<2, 1>(adq, bd, d_base, colv, bov, idnv, pstep, astep, tstep);
+                                else if (Td == 2) issue_stacked_q<2, 2>(adq, bd, d_base, colv, bov, idnv, pstep, astep, tstep);
+                                else if (ntl == 1) issue_stacked_q<4, 1>(adq, bd, d_base, colv, bov, idnv, pstep, astep, tstep);
+                                else issue_stacked_q<4, 2>(adq, bd, d_base, colv, bov, idnv, pstep, astep, tstep);
+                                continue;
+                            }
+                            for (int i = 0; i < Td + 2; i++) {
+                                const int alo = max(0, i - Td + 1), ahi = min(2, i);
+                                const uint64_t ad = adq + i * pstep;
+                                if (first && alo == 0) {
+                                    issue_n(ad, bd, i, 1, 0u);
+                                    if (ahi >= 1) issue_n(ad, bd + (uint64_t)Nc, i - 1, ahi, 1u);
+                                } else {
+                                    issue_n(ad, bd + (uint64_t)(alo * Nc), i - alo, ahi - alo + 1, 1u);
+                                }
+                            }
+                        }
+                        ptx::mma_commit_elect(&sh.wempty[st]);
+                        continue;
+                    }
                     auto issue = [&](uint64_t ad, uint32_t acc) {
                         ptx::mma_bf16_elect_nc(d_base, ad, bd, idesc, acc);
                         if (ntl > 1) ptx::mma_bf16_elect_nc(d_base + dstep, ad + astep, bd, idesc, acc);
@@ -1033,7 +1124,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             ptx::tc_fence_after();
             const int CB = L.Nc >= 32 ? 32 : 16;
             const int ncb = L.Nc / CB;
-            const int items = L.ntl * ncb;
+            const int items = L.ntl * ncb * L.Td;   // (stacked layers: Td output planes per task)
             __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(L.out.ptr);
             const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(L.res.ptr);
             const int d = T.d;
@@ -1121,16 +1212,19 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 }
             }
             for (int it = rank; it < (L.pool ? 0 : items); it += 4) {
-                const int tl = it / ncb, cb = it - tl * ncb;
+                const int o = it / (L.ntl * ncb), itr = it - o * (L.ntl * ncb);   // output plane of the task
+                const int tl = itr / ncb, cb = itr - tl * ncb;
                 const int m = tl * 128 + quad * 32 + lane;
                 const int i = m / L.Wp, j = m - i * L.Wp;
                 const int y = T.y0 + i, x = T.x0 + j;
+                const int d = T.d + o;
                 int kind = 0;   // 0 skip, 1 zero (masked), 2 value
                 if (i < L.Tb && j < L.Tw && d < T.hi[0] && y < T.hi[1] && x < T.hi[2] && (!p.padded || x >= T.dlo[2]))
                     kind = (d < L.out_ext[0] && y < L.out_ext[1] && x < L.out_ext[2]) ? 2 : 1;
                 const int ch0 = T.nc * L.Nc + cb * CB;
                 uint32_t r[2][16];
-                const uint32_t taddr = tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) + tl * L.Nc + cb * CB;
+                const uint32_t taddr = tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) +
+                                       tl * (L.Td * L.Nc) + (L.Td - 1 - o) * L.Nc + cb * CB;
                 ptx::tmem_ld16(taddr, r[0]);
                 if (CB == 32) ptx::tmem_ld16(taddr + 16, r[1]);
                 ptx::tmem_ld_wait();
@@ -1199,21 +1293,32 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
 }
 
 // weights [cout][kd][kh][kw][cin] bf16 -> [nc][kb][ks][2][Nc][8] per the layer's A mode
+// stk (depth-stacked 3-D layer): per k-step q' = (rs, kk) the B operand is [2][kd * Nc][8]: the kd depth taps' weights
+// side by side along N (tap a at rows [a*Nc, (a+1)*Nc)), so one MMA can feed several output planes.
 __global__ void pack_gen_kernel(const __nv_bfloat16 *__restrict__ w, __nv_bfloat16 *__restrict__ out, int cout, int cin,
-                                int kd, int kh, int kw, int amode, int Nc, int nkb, int nks) {
-    const long long total = (long long)(cout / Nc) * nkb * nks * 2 * Nc * 8;
+                                int kd, int kh, int kw, int amode, int Nc, int nkb, int nks, int stk) {
+    const int NB = stk ? kd * Nc : Nc;           // B rows per k-step
+    const int nq = stk ? nks / kd : nks;         // k-steps in the packed layout
+    const long long total = (long long)(cout / Nc) * nkb * nq * 2 * NB * 8;
     const int taps = kd * kh * kw;
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
         long long r = i;
         const int e = (int)(r % 8); r /= 8;
-        const int col = (int)(r % Nc); r /= Nc;
+        int col = (int)(r % NB); r /= NB;
         const int j = (int)(r % 2); r /= 2;
-        const int q = (int)(r % nks); r /= nks;
+        int q = (int)(r % nq); r /= nq;
         const int kb = (int)(r % nkb);
         const int nc = (int)(r / nkb);
-        int tap, ci;
-        if (amode == AM_SW128) { tap = q / 4; ci = kb * 64 + (q % 4) * 16 + j * 8 + e; }
-        else if (amode == AM_PLANES || amode == AM_SW64) { const int kpt = (cin + 15) / 16; tap = q / kpt; ci = (q % kpt) * 16 + j * 8 + e; }
+        if (stk) {   // (q', a) -> the unstacked k-step q = q' * kd + a
+            q = q * kd + col / Nc;
+            col %= Nc;
+        }
+        int tap, ci, kk;
+        if (amode == AM_SW128) { kstep_tap(q, kd, kh, kw, 4, tap, kk); ci = kb * 64 + kk * 16 + j * 8 + e; }
+        else if (amode == AM_PLANES || amode == AM_SW64) {
+            kstep_tap(q, kd, kh, kw, (cin + 15) / 16, tap, kk);
+            ci = kk * 16 + j * 8 + e;
+        }
         else {
             const int np = (kw + 1) / 2, u = q % np, ar = q / np;
             const int s = 2 * u + j;
@@ -1246,6 +1351,12 @@ constexpr int kGenInBudget = 112 * 1024;   // input-stage ring
 constexpr int kGenWStage = 32 * 1024;      // one weight stage
 constexpr int kGenW = 3;                   // weight stages
 constexpr double kGenTaskOverheadMmas = 96.0;   // fixed per-task cost in units of one 128-row MMA (tile model)
+
+// BDL_GEN_STACK=0: no depth stacking (A/B runs)
+static bool gen_stack_ok() {
+    static const int v = [] { const char *e = getenv("BDL_GEN_STACK"); return e ? atoi(e) : 1; }();
+    return v != 0;
+}
 
 // Static (tile-independent) fields of a layer.  Returns false if the layer cannot run on the kernel.
 static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out, gen::LayerP &G) {
@@ -1295,6 +1406,18 @@ static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out,
     G.kpw = std::max(1, std::min(G.nks, kGenWStage / ks_bytes));
     G.nws = (G.nks + G.kpw - 1) / G.kpw;
     G.idesc = ptx::idesc_bf16_f32(128, G.Nc);
+    // depth stacking (3-D 3x3x3 layers of one K-block and one channel chunk, 3 Nc <= 256): the packed B of a k-step
+    // holds the three depth taps side by side, in every mode (padded runs it with Td = 1)
+    G.stk = 0;
+    G.Td = 1;
+    if (nsp == 3 && G.k[0] == 3 && G.s[0] == 1 && G.dl[0] == 1 && G.nkb == 1 && G.amode != gen::AM_PAIR &&
+        3 * G.Nc <= 256 && G.nnc == 1 && gen_stack_ok()) {
+        G.stk = 1;
+        const int nq = G.nks / 3, ksb = 2 * 3 * G.Nc * 16;
+        G.kpw = std::max(1, std::min(nq, kGenWStage / ksb));
+        G.nws = (nq + G.kpw - 1) / G.kpw;
+        for (int i = 0; i < 3; i++) G.idesc_s[i] = ptx::idesc_bf16_f32(128, (i + 1) * G.Nc);
+    }
     G.nblk = G.s[1] * G.s[2];
     return true;
 }
@@ -1312,10 +1435,12 @@ static int gen_pool_stage_bytes(const gen::LayerP &G) {
 // the conv tile is the region under their windows, Tb = (Tpb-1)*ps + pk (likewise Tw).
 constexpr int kGenPoolStageMax = 32 * 1024;   // fused pool: largest epilogue staging tile
 
-static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign, int in_budget = kGenInBudget) {
+static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign, int in_budget = kGenInBudget,
+                            int max_td = 1) {
     double best = -1e30;
     bool found = false;
     gen::LayerP cand = G;
+    for (int Td = 1; Td <= (G.stk ? max_td : 1); Td *= 2)
     for (int Ub = std::min(cover_h, 32); Ub >= 1; Ub--) {
         for (int Uw = (cover_w + walign - 1) / walign * walign; Uw >= walign; Uw -= walign) {
             const int Tb = G.pool ? (Ub - 1) * G.ps[0] + G.pk[0] : Ub, Tw = G.pool ? (Uw - 1) * G.ps[1] + G.pk[1] : Uw;
@@ -1332,10 +1457,12 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
             cand.plane_px = cand.nblk * cand.blk_px;
             const int M = Tb * cand.Wp;
             cand.ntl = (M + 127) / 128;
-            if (cand.ntl * G.Nc > 256) continue;       // double-buffered accumulators
-            const int max_tap = (G.ke[0] - 1) * cand.plane_px + (cand.nblk - 1) * cand.blk_px +
+            cand.Td = Td;
+            if (cand.ntl * Td * G.Nc > 256) continue;   // double-buffered accumulators (Td planes per task)
+            const int npl = G.ke[0] + Td - 1;            // input planes of a task's stage
+            const int max_tap = (npl - 1) * cand.plane_px + (cand.nblk - 1) * cand.blk_px +
                                 ((G.ke[1] - 1) / G.s[1]) * cand.Wp + (G.ke[2] - 1) / G.s[2];
-            int rows = std::max(G.ke[0] * cand.plane_px, max_tap + cand.ntl * 128);
+            int rows = std::max(npl * cand.plane_px, max_tap + cand.ntl * 128);
             rows = (rows + 7) / 8 * 8;
             if (G.amode == gen::AM_PLANES) rows += 1;   // odd plane stride: conflict-free loader stores
             if (G.amode == gen::AM_SW64) rows = (rows + 1 + 7) / 8 * 8;   // room for the alignment offset pxo
@@ -1353,9 +1480,20 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
             // BDL_GEN_DBG=7), i.e. on the order of a hundred 128-row MMAs, so small tiles lose even when their
             // MMA rows are better used.
             const double halo = (double)cand.in_rows * cand.in_cols / ((double)Tb * Tw * G.s[1] * G.s[2]);
-            const double mmas = (double)cand.ntl * G.nks * G.nkb;
-            const double cost = (double)nty * ntx * (mmas + kGenTaskOverheadMmas) * (1.0 + 0.1 * (halo - 1.0));
-            const double score = -cost + 1e-6 * Ub * Uw;
+            double mmas = (double)cand.ntl * G.nks * G.nkb;
+            if (G.stk) {
+                // stacked: per k-step one MMA per input plane, of N = (number of output planes it feeds) x Nc, costed by
+                // its shared-memory operand bytes relative to an N = Nc MMA (A 4 KB + B 32 B per N row)
+                double w = 0;
+                for (int i = 0; i < npl; i++) {
+                    const int na = std::min(2, i) - std::max(0, i - Td + 1) + 1;
+                    w += (4096.0 + na * G.Nc * 32.0) / (4096.0 + G.Nc * 32.0);
+                }
+                mmas = (double)cand.ntl * (G.nks / 3) * w;
+            }
+            // per output plane: tasks / Td
+            const double cost = (double)nty * ntx / Td * (mmas + kGenTaskOverheadMmas) * (1.0 + 0.1 * (halo - 1.0));
+            const double score = -cost + 1e-6 * Ub * Uw * Td;
             if (score > best) {
                 best = score;
                 G = cand;
@@ -1457,7 +1595,14 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
     const bool fused = gen_pool_fused(p, sg, nconv, padded && nconv > 1);
     // the pool's staging tile takes one weight stage's room (2 weight stages instead of 3), not input-ring room: smaller
     // input stages cost more, smaller tiles (measured on B200, VGG stage 1: 2.9 -> 3.7 ms when the ring shrank)
-    const int in_budget = kGenInBudget;
+    // depth-stacked subgraphs (memoized geometry): Td planes per task need deeper input stages; the weight ring gives up
+    // a stage for them (A/B knobs: BDL_GEN_MAXTD, BDL_GEN_STK_NW)
+    static const int max_td_env = [] { const char *e = getenv("BDL_GEN_MAXTD"); return e ? atoi(e) : 4; }();
+    static const int stk_nw_env = [] { const char *e = getenv("BDL_GEN_STK_NW"); return e ? atoi(e) : 2; }();
+    bool any_stk = false;
+    for (int j = 0; j < nconv; j++) any_stk = any_stk || g.layer[j].stk;
+    const bool stk_geo = any_stk && !padded && max_td_env > 1;
+    const int in_budget = stk_geo ? kGenInBudget + (kGenW - stk_nw_env) * kGenWStage : kGenInBudget;
     if (fused) {   // the pool's output is the last conv's task grid
         gen::LayerP &G = g.layer[nconv - 1];
         const Layer &pl = p->layers[sg.last];
@@ -1534,8 +1679,8 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
             // pooled tiles: brick-aligned conv columns (TMA rows) when the windows tile the map (k = s, no padding)
             int walign = p->in_layout.Bw;
             if (G.pool) walign = (G.pk[1] == G.ps[1] && G.ppd[1] == 0 && p->in_layout.Bw % G.ps[1] == 0) ? p->in_layout.Bw / G.ps[1] : 1;
-            if (!gen_layer_tiles(G, G.grid[1], G.grid[2], walign, in_budget)) return false;
-            G.ntd = G.grid[0];
+            if (!gen_layer_tiles(G, G.grid[1], G.grid[2], walign, in_budget, stk_geo ? max_td_env : 1)) return false;
+            G.ntd = (G.grid[0] + G.Td - 1) / G.Td;   // plane blocks of Td output planes
             const int tb = G.pool ? G.Tpb : G.Tb, tw = G.pool ? G.Tpw : G.Tw;   // pooled: tiles of pool outputs
             G.nty = (G.grid[1] + tb - 1) / tb;
             G.ntx = (G.grid[2] + tw - 1) / tw;
@@ -1548,14 +1693,14 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
     for (int j = 0; j < nconv; j++) {
         const gen::LayerP &G = g.layer[j];
         in_stride = std::max(in_stride, G.stage_bytes);
-        w_stride = std::max(w_stride, G.kpw * 2 * G.Nc * 16);
-        acc = std::max(acc, G.ntl * G.Nc);
+        w_stride = std::max(w_stride, G.kpw * 2 * (G.stk ? 3 : 1) * G.Nc * 16);
+        acc = std::max(acc, G.ntl * G.Td * G.Nc);
         if (G.pool) g.pool_bytes = (gen_pool_stage_bytes(G) + 1023) / 1024 * 1024;
     }
     g.in_stride = in_stride;
     g.w_stride = (w_stride + 1023) / 1024 * 1024;
-    g.nin = std::min(gen::kMaxIn, kGenInBudget / in_stride);
-    g.nw = g.pool_bytes ? kGenW - 1 : kGenW;
+    g.nin = std::min(gen::kMaxIn, in_budget / in_stride);
+    g.nw = g.pool_bytes ? kGenW - 1 : stk_geo ? stk_nw_env : kGenW;
     if (g.pool_bytes > kGenWStage) return false;
     g.acc_stride = acc;
     g.nacc = 2 * acc <= 512 ? 2 : 1;
@@ -1700,7 +1845,7 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
             }
             if (D.ns == 0) {   // reads an external tensor: how far down its input frame the window reaches
                 const gen::TaskC c = gen::decode(C, t);
-                const int z = std::min(C.in_ext[0] - 1, c.d * C.s[0] - C.pd[0] + C.ke[0] - 1);
+                const int z = std::min(C.in_ext[0] - 1, (c.d * C.Td + C.Td - 1) * C.s[0] - C.pd[0] + C.ke[0] - 1);
                 const int y = std::min(C.in_ext[1] - 1, (gen::tile_y0(C, c.ty) + C.Tb - 1) * C.s[1] - C.pd[1] + C.ke[1] - 1);
                 const int x = std::min(C.in_ext[2] - 1, (gen::tile_x0(C, c.tx) + C.Tw - 1) * C.s[2] - C.pd[2] + C.ke[2] - 1);
                 k = std::max(k, ((double)std::max(z, 0) * C.in_ext[1] + std::max(y, 0)) * C.in_ext[2] + std::max(x, 0)) /
@@ -1735,7 +1880,7 @@ bdl_status launch_pack_gen(const bdl_plan *p, const Subgraph &sg, int j, void *w
     const long long total = (long long)G.nnc * G.nkb * G.nks * 2 * G.Nc * 8;
     const int grid = (int)std::min<long long>((total + 255) / 256, 4096);
     gen::pack_gen_kernel<<<grid, 256, 0, s>>>((const __nv_bfloat16 *)l.w, (__nv_bfloat16 *)w_out, l.cout, l.cin, l.k[0],
-                                              l.k[1], l.k[2], G.amode, G.Nc, G.nkb, G.nks);
+                                              l.k[1], l.k[2], G.amode, G.Nc, G.nkb, G.nks, G.stk);
     BDL_CUDA_CHECK_LAUNCH("pack_gen");
     return BDL_OK;
 }
