@@ -219,8 +219,13 @@ __host__ __device__ __forceinline__ DepRange dep_range_src(const LayerP &C, cons
     // (tasks of depth-stacked layers cover Td planes: C's planes [c.d*Td, +Td), P's blocks of P.Td planes)
     lo = max(0, c.d * C.Td * C.s[0] - C.pd[0]);
     hi = min(C.in_ext[0] - 1, (c.d * C.Td + C.Td - 1) * C.s[0] - C.pd[0] + C.ke[0] - 1);
-    r.d0 = lo / P.Td;
-    r.nd = hi >= lo ? hi / P.Td - r.d0 + 1 : 0;
+    if (P.Td == 1) {   // (2-D and unstacked layers: no division on the per-task path)
+        r.d0 = lo;
+        r.nd = max(0, hi - lo + 1);
+    } else {
+        r.d0 = lo / P.Td;
+        r.nd = hi >= lo ? hi / P.Td - r.d0 + 1 : 0;
+    }
     const int y0 = tile_y0(C, c.ty), x0 = tile_x0(C, c.tx);
     lo = max(0, y0 * C.s[1] - C.pd[1]);
     hi = min(C.in_ext[1] - 1, (y0 + C.Tb - 1) * C.s[1] - C.pd[1] + C.ke[1] - 1);
@@ -240,8 +245,8 @@ __host__ __device__ __forceinline__ DepRange dep_range_res(const LayerP &C, cons
     r.nnc = 1;
     {
         const int dlo = c.d * C.Td, dhi = min(C.out_ext[0], dlo + C.Td) - 1;
-        r.d0 = dlo / R.Td;
-        r.nd = dhi >= dlo ? dhi / R.Td - r.d0 + 1 : 0;
+        r.d0 = R.Td == 1 ? dlo : dlo / R.Td;
+        r.nd = dhi >= dlo ? (R.Td == 1 ? dhi : dhi / R.Td) - r.d0 + 1 : 0;
     }
     int lo = c.ty * C.Tb, hi = min(C.out_ext[1], lo + C.Tb) - 1;
     r.b0 = lo / R.Tb;
@@ -793,6 +798,9 @@ __device__ __forceinline__ void issue_stacked_q(uint64_t adq, uint64_t bd, uint3
 }
 
 // ---------------------------------------------------------------------------------------------- kernel
+// STK: the subgraph has depth-stacked layers.  Two instantiations, so the stacked issue path is absent from the kernel
+// that 2-D subgraphs run (present, it cost 2-D layers ~15 % through the MMA warp's register allocation; B200 A/B).
+template <bool STK>
 __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant__ Params p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     __shared__ Shared sh;
@@ -1022,7 +1030,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     const int q0 = j * L.kpw, q1 = (p.dbg & 1) ? q0 + 1 : min(L.stk ? L.nks / 3 : L.nks, q0 + L.kpw);
                     const uint64_t a_d0 = ad_t + a_base;
                     uint64_t bd = bd_t + b_base;
-                    if (L.stk) {
+                    if (STK && L.stk) {
                         // depth-stacked 3-D layer: per k-step (r, s, kk), input plane i feeds output planes o = i - a for the
                         // depth taps a in [alo, ahi]: ONE MMA with N = (ahi - alo + 1) Nc, B = those taps' weights side
                         // by side, D = the planes' accumulators, laid out at columns (Td - 1 - o) Nc so they are contiguous
@@ -1124,7 +1132,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             ptx::tc_fence_after();
             const int CB = L.Nc >= 32 ? 32 : 16;
             const int ncb = L.Nc / CB;
-            const int items = L.ntl * ncb * L.Td;   // (stacked layers: Td output planes per task)
+            const int Tdv = STK ? L.Td : 1;          // output planes per task (stacked 3-D layers)
+            const int items = L.ntl * ncb * Tdv;
             __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(L.out.ptr);
             const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(L.res.ptr);
             const int d = T.d;
@@ -1212,7 +1221,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 }
             }
             for (int it = rank; it < (L.pool ? 0 : items); it += 4) {
-                const int o = it / (L.ntl * ncb), itr = it - o * (L.ntl * ncb);   // output plane of the task
+                const int o = STK ? it / (L.ntl * ncb) : 0, itr = it - o * (L.ntl * ncb);   // output plane of the task
                 const int tl = itr / ncb, cb = itr - tl * ncb;
                 const int m = tl * 128 + quad * 32 + lane;
                 const int i = m / L.Wp, j = m - i * L.Wp;
@@ -1224,7 +1233,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 const int ch0 = T.nc * L.Nc + cb * CB;
                 uint32_t r[2][16];
                 const uint32_t taddr = tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) +
-                                       tl * (L.Td * L.Nc) + (L.Td - 1 - o) * L.Nc + cb * CB;
+                                       tl * (Tdv * L.Nc) + (Tdv - 1 - o) * L.Nc + cb * CB;
                 ptx::tmem_ld16(taddr, r[0]);
                 if (CB == 32) ptx::tmem_ld16(taddr + 16, r[1]);
                 ptx::tmem_ld_wait();
@@ -1972,7 +1981,10 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
     P.status = (int *)(wsp + sg.status_off);
     P.defer = p->opts.memo_defer;
     P.counters = (unsigned long long *)(wsp + sg.counter_off);
-    cudaFuncSetAttribute(gen::gen_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
+    bool any_stk = false;
+    for (int j = 0; j < L; j++) any_stk = any_stk || P.layer[j].stk;
+    auto kern = any_stk ? gen::gen_kernel<true> : gen::gen_kernel<false>;
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
     const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;
     if (padded) {
         P.padded = 1;
@@ -1985,14 +1997,14 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
         P.scr_slot = g.scr_slot;
         P.norder = (long long)p->layers[sg.first].in_ext[0] * g.npb[0] * g.npb[1] * g.npb[2];
         const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-        launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+        launch_pdl(kern, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
         *launches += 1;
     } else if (!unmerged) {
         P.only_layer = -1;
         P.order = (const int *)(wsp + sg.order_off);
         P.norder = sg.norder;
         const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-        launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+        launch_pdl(kern, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
         *launches += 1;
     } else {
         P.order = nullptr;
@@ -2000,7 +2012,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
             P.only_layer = j;
             P.norder = P.layer[j].ntasks;
             const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-            launch_pdl(gen::gen_kernel, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+            launch_pdl(kern, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
             *launches += 1;
         }
     }
