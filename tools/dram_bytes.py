@@ -88,6 +88,30 @@ def summarize(path):
     return tot, per, n
 
 
+def per_launch(path):
+    """[(kernel name, DRAM bytes, duration s)] in launch order."""
+    rows = list(csv.reader(open(path)))
+    i = next(k for k, r in enumerate(rows) if r and r[0] == "ID")
+    hdr = rows[i]
+    by = {}
+    for r in rows[i + 1:]:
+        if len(r) != len(hdr):
+            continue
+        d = dict(zip(hdr, r))
+        try:
+            v = float(d["Metric Value"].replace(",", ""))
+        except ValueError:
+            continue
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-9, "us": 1e-6, "ms": 1e-3,
+                 "nsecond": 1e-9, "usecond": 1e-6, "msecond": 1e-3}.get(d["Metric Unit"], 1)
+        e = by.setdefault(int(d["ID"]), {"name": d["Kernel Name"].split("(")[0][:40], "bytes": 0.0, "t": 0.0})
+        if d["Metric Name"].startswith("dram__bytes"):
+            e["bytes"] += v * scale
+        else:
+            e["t"] += v * scale
+    return [by[k] for k in sorted(by)]
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("cmd", choices=["run", "sum"])
@@ -104,6 +128,9 @@ def main():
               f"{(rd + wr) / 1e6:.1f} MB, kernel time (cold, serialized) {tot['gpu__time_duration.sum'] * 1e3:.3f} ms")
         for k, v in sorted(per.items(), key=lambda kv: -(kv[1]["dram__bytes_read.sum"] + kv[1]["dram__bytes_write.sum"]))[:6]:
             print(f"    {k:40s} {(v['dram__bytes_read.sum'] + v['dram__bytes_write.sum']) / 1e6:10.1f} MB")
+        if "merged" in os.path.basename(a.arg):   # one line per launch: brickify, each subgraph (+ pool tail), output
+            for j, e in enumerate(per_launch(a.arg)):
+                print(f"      launch {j:2d} {e['name']:40s} {e['bytes'] / 1e6:10.1f} MB")
 
 
 if __name__ == "__main__":
