@@ -435,16 +435,29 @@ def main():
             traffic = None
     kinds = {g["kernel"] for g in sg}
     if kinds == {"cuda-core brick"}:
-        # plain FMA pipes: 148 SMs x 128 fp32 FMA/clk x 2 flop x max SM clock
-        bound, peak = "alu", 148 * 128 * 2 * 1.965e9 / 1e12
-        peak_src = "derived: 148 SM x 128 FFMA/clk x 2 x 1965 MHz"
+        # plain FMA pipes: measured on this box (8 independent FFMA chains per thread, 4 x 256 threads per SM;
+        # libbdl_microbench.so), the derived figure 148 SM x 128 FFMA/clk x 2 x 1965 MHz as a fallback
+        bound = "alu"
+        try:
+            import ctypes
+            from paper_conf_icpp_lakshminarasimhan24_b200 import build as _b
+            mb = ctypes.CDLL(_b.build_microbench())
+            tf = ctypes.c_double()
+            if mb.bdl_mb_ffma(ctypes.byref(tf)) != 0:
+                raise RuntimeError("ffma microbenchmark failed")
+            peak, peak_src = tf.value, "measured in this run: FFMA microbenchmark (libbdl_microbench.so bdl_mb_ffma)"
+        except Exception as e:
+            peak = 148 * 128 * 2 * 1.965e9 / 1e12
+            peak_src = f"derived (microbenchmark unavailable: {e}): 148 SM x 128 FFMA/clk x 2 x 1965 MHz"
     else:
         bound, peak = "tensor", float(peaks["bf16_tflops"])
         peak_src = f"{peak_src} bf16_tflops (burst, cuBLAS 8192^3)"
     achieved = flops / (kernel_ms / 1e3) / 1e12
     kname = sg[0]["kernel"] if len(sg) == 1 else f"{len(sg)} subgraph launches ({', '.join(sorted(kinds))})"
     roofline = {"bound": bound, "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
-                "traffic": traffic if len(sg) == 1 else None, "traffic_source": traffic_src, "peak_source": peak_src,
+                "traffic": traffic if len(sg) == 1 and kinds == {"tcgen05 band"} else None,
+                "traffic_source": traffic_src if len(sg) == 1 and kinds == {"tcgen05 band"} else None,
+                "peak_source": peak_src,
                 "kernel": f"{kname} ({'/'.join(sorted({g['mode'] for g in sg}))})",
                 "algorithmic_flops_per_launch": flops, "kernel_ms_mean": kernel_ms, "hbm_frac_of_step_bytes": None}
     # step bytes

@@ -86,3 +86,47 @@ extern "C" int bdl_mb_cas(int ctas, int iters, int mode, double *ns_per_op, doub
     cudaFree(fl);
     return e == cudaSuccess ? 0 : 2;
 }
+
+// ---------------------------------------------------------------------------------------------------------------------
+// FFMA throughput of the device (the "alu" roofline peak of the fp32 CUDA-core paths: measured on the
+// box, not derived): every thread runs 8 independent fp32 FMA chains; 4 CTAs of 256 threads per SM.
+namespace {
+__global__ void ffma_kernel(float *out, int iters, float a, float b) {
+    float x0 = threadIdx.x, x1 = x0 + 1, x2 = x0 + 2, x3 = x0 + 3, x4 = x0 + 4, x5 = x0 + 5, x6 = x0 + 6, x7 = x0 + 7;
+    for (int i = 0; i < iters; i++) {
+#pragma unroll
+        for (int k = 0; k < 16; k++) {
+            x0 = fmaf(x0, a, b); x1 = fmaf(x1, a, b); x2 = fmaf(x2, a, b); x3 = fmaf(x3, a, b);
+            x4 = fmaf(x4, a, b); x5 = fmaf(x5, a, b); x6 = fmaf(x6, a, b); x7 = fmaf(x7, a, b);
+        }
+    }
+    const float s = x0 + x1 + x2 + x3 + x4 + x5 + x6 + x7;
+    if (s == 1234.5f) out[blockIdx.x] = s;   // keeps the chains live
+}
+}  // namespace
+
+extern "C" int bdl_mb_ffma(double *tflops) {
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+    float *out = nullptr;
+    cudaMalloc(&out, 4096 * 4);
+    const int grid = sms * 4, block = 256, iters = 4096;
+    ffma_kernel<<<grid, block>>>(out, 16, 0.999f, 0.001f);
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    double best = 0;
+    for (int r = 0; r < 3; r++) {
+        cudaEventRecord(e0);
+        ffma_kernel<<<grid, block>>>(out, iters, 0.999f, 0.001f);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        const double flops = 2.0 * 8 * 16 * (double)iters * grid * block;
+        best = flops / (ms * 1e-3) / 1e12 > best ? flops / (ms * 1e-3) / 1e12 : best;
+    }
+    *tflops = best;
+    cudaFree(out);
+    return cudaGetLastError() == cudaSuccess ? 0 : 2;
+}
