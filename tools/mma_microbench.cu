@@ -29,10 +29,56 @@ __global__ void __launch_bounds__(128, 1) mma_loop(int iters, unsigned long long
     constexpr uint32_t ID = idesc_bf16_f32(128, N);
     unsigned long long t0 = clock64();
     const int wid = __shfl_sync(0xffffffff, (int)threadIdx.x / 32, 0);
+    __shared__ volatile int stop;
+    if (threadIdx.x == 0) stop = 0;
+    __syncthreads();
+    if ((MODE == 12 || MODE == 14) && wid >= 1) {
+        // epilogue-like interference: tcgen05.ld of TMEM columns 384..511 (not used by the MMAs) in a loop
+        const uint32_t tb = __shfl_sync(0xffffffff, tbase, 0);
+        uint32_t r[16], acc = 0;
+        while (!stop) {
+            for (int c = 0; c < 128; c += 16) {
+                tmem_ld16(tb + ((uint32_t)(wid * 32) << 16) + 384 + c, r);
+                tmem_ld_wait();
+                acc += r[0];
+            }
+        }
+        if (acc == 12345) cyc[blockIdx.x + 1000] = acc;
+    } else if ((MODE == 13 || MODE == 14) && wid == 1) {
+        // loader-like interference: bulk copies of 32 KB into shared memory (region 160-192 KB, not read by the MMAs)
+        uint32_t ph = 0;
+        while (!stop) {
+            if (elect_one()) {
+                mbar_arrive_expect_tx(&wfull[0], 32768);
+                bulk_g2s(smem + 160 * 1024, gw, 32768, &wfull[0]);
+            }
+            __syncwarp();
+            mbar_wait(&wfull[0], ph);
+            ph ^= 1;
+        }
+    }
     if (wid == 0) {
         const uint32_t tb = __shfl_sync(0xffffffff, tbase, 0);
         const uint32_t abase = smem_u32(A) >> 4, bbase = smem_u32(B) >> 4;
-        if (MODE == 9 || MODE == 10) {
+        if (MODE >= 11) {
+            // depth-stacked cfg5 pattern: per k-step (18) six input planes, MMAs of N = 32, 64, 96, 96, 64, 32
+            // (Td = 4), SW64 A (plane = 162 rows), B stacked [2][96][8] per k-step
+            const uint64_t a0 = umma_desc_sw64(0, 512), b0 = umma_desc_noswz(0, 96 * 16, 128);
+            const uint32_t nn[6] = {32, 64, 96, 96, 64, 32};
+            const uint32_t bo[6] = {0, 0, 0, 0, 32, 64};
+            const uint32_t col[6] = {96, 64, 32, 0, 0, 0};
+            for (int it = 0; it < iters; it++) {
+                for (int q = 0; q < 18; q++) {
+                    const uint32_t px = ((q / 2) / 3) * 18 + (q / 2) % 3;
+                    const uint64_t bd0 = b0 + bbase + q * (96 * 2);
+#pragma unroll
+                    for (int i = 0; i < 6; i++) {
+                        const uint64_t ad = a0 + abase + (px + i * 162) * 4 + (q % 2) * 2;
+                        mma_bf16_elect(tb + (it & 1) * 128 + col[i], ad, bd0 + bo[i], idesc_bf16_f32(128, nn[i]), 1);
+                    }
+                }
+            }
+        } else if (MODE == 9 || MODE == 10) {
             // generic-kernel cfg5 shape on the 64-B swizzled layout (AM_SW64): pixel rows of 64 B, Wp = 18, plane 288
             // rows, 27 taps x 2 k-steps, ntl = 2 (mode 9) or 1 (mode 10)
             const uint64_t a0 = umma_desc_sw64(0, 512), b0 = umma_desc_noswz(0, N * 16, 128);
@@ -143,7 +189,11 @@ __global__ void __launch_bounds__(128, 1) mma_loop(int iters, unsigned long long
             __syncwarp();
         }
     }
-    mbar_wait(&done, 0);
+    if (wid == 0) {
+        mbar_wait(&done, 0);
+        if (threadIdx.x == 0) stop = 1;
+    }
+    __syncthreads();
     unsigned long long t1 = clock64();
     if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
     tc_fence_before(); __syncthreads();
@@ -161,7 +211,7 @@ template <int N, int MODE> void run(int sms, const uint8_t *gw) {
     cudaEventRecord(b); cudaEventSynchronize(b);
     float ms; cudaEventElapsedTime(&ms, a, b);
     unsigned long long h[256]; cudaMemcpy(h, d, sms * 8, cudaMemcpyDeviceToHost);
-    double n_mma = (double)iters * (MODE == 9 ? 108 : MODE >= 7 ? 54 : MODE >= 4 ? 12 : 16);
+    double n_mma = (double)iters * (MODE >= 11 ? 108 : MODE == 9 ? 108 : MODE >= 7 ? 54 : MODE >= 4 ? 12 : 16);
     double flops = n_mma * 2.0 * 128 * N * 16 * sms;
     printf("mode=%d N=%3d  cycles/MMA=%.1f (ideal %d)  chip %.1f TFLOP/s  (%s)\n", MODE, N, h[0] / n_mma, 128 * N / 256,
            flops / (ms * 1e-3) / 1e12, cudaGetErrorString(cudaGetLastError()));
@@ -177,6 +227,7 @@ int main() {
     run<64, 4>(1, gw); run<64, 5>(1, gw); run<64, 6>(1, gw);
     run<192, 0>(sms, gw); run<192, 4>(sms, gw); run<128, 4>(sms, gw); run<256, 4>(sms, gw);
     run<32, 7>(sms, gw); run<32, 8>(sms, gw); run<32, 0>(sms, gw);
-    run<32, 9>(sms, gw); run<32, 10>(sms, gw); run<64, 9>(sms, gw);
+    run<32, 9>(sms, gw); run<32, 10>(sms, gw); run<32, 11>(sms, gw); run<32, 12>(sms, gw); run<32, 13>(sms, gw);
+    run<32, 14>(sms, gw);
     return 0;
 }
