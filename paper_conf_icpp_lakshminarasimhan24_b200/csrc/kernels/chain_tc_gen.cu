@@ -109,8 +109,9 @@ struct Params {
     // halo-extended region is recomputed by the CTA into its private scratch (two slots, so two blocks
     // interleave and one block's loads overlap the other's MMAs)
     int dbg;                             // debug timing knobs (BDL_GEN_DBG): 1 = one k-step per task, 2 = no input loads,
-                                         // 4 = no epilogue stores (all give wrong results)
-    unsigned long long *prof;            // debug (BDL_GEN_PROF): per CTA 16 x u64 of role wait / busy cycles, or null
+                                         // 4 = no epilogue stores, 8 = no bias reads, 16 = no residual reads (all give
+                                         // wrong results)
+    unsigned long long *prof;            // debug (BDL_GEN_PROF): per CTA 32 x u64 of role wait / busy cycles, or null
     int padded;
     int PB[3], npb[3];
     unsigned char *scratch;
@@ -135,6 +136,15 @@ struct Shared {
     uint32_t ks[kMaxLayers][kMaxKs];     // per k-step: A offset | LBO << 16 (both in 16-B units, < 2^14)
 };
 
+// detailed per-phase timers of the debug profiler (BDL_GEN_PROF): debug builds only (they cost the release kernel
+// registers and issue slots)
+#ifdef BDL_DEBUG
+#define PT(x) x
+#define DBG(p, bit) ((p).dbg & (bit))   // work-skipping timing knobs (wrong results)
+#else
+#define PT(x)
+#define DBG(p, bit) 0
+#endif
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ptx::smem_u32(bar)) : "memory");
 }
@@ -896,7 +906,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         // ------------------------------------------------------------------ loaders
         const int tid = threadIdx.x - 32 * kLoad0;
         uint32_t gin = 0;
-        unsigned long long wq = 0, wdep = 0, wbuf = 0;
+        unsigned long long wq = 0, wdep = 0, wbuf = 0, wiss = 0, wbar = 0;
         const unsigned long long t_start = clock64();
         for (uint32_t seq = 0;; seq++) {
             const int slot = seq % kQ;
@@ -932,7 +942,9 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 for (int o = 16; o; o >>= 1) spins += __shfl_xor_sync(0xffffffff, spins, o);
                 if (lane == 0 && spins) atomicAdd(&p.counters[3], spins);
             }
+            PT(const unsigned long long tlb = p.prof ? clock64() : 0;)
             asm volatile("bar.sync 1, %0;" ::"n"(kLoadT) : "memory");
+            PT(if (p.prof) wbar += clock64() - tlb;)
             if (l >= 0 && p.layer[l].tma) ptx::fence_proxy_async();   // acquired data is read by TMA (async proxy)
             if (tid == 0) {
                 sh.desc_l[seq % kRing] = l;
@@ -946,14 +958,16 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             for (int kb = 0; kb < L.nkb; kb++, gin++) {
                 const int s = gin % p.nin;
                 if (gin >= (uint32_t)p.nin) pwait(p, &sh.in_empty[s], ((gin / p.nin) - 1) & 1, wbuf);
-                if (!(p.dbg & 2)) load_stage(p, L, T, kb, in_ring + (size_t)s * p.in_stride, tid, &sh.in_full[s]);
+                PT(const unsigned long long tl0 = p.prof ? clock64() : 0;)
+                if (!DBG(p, 2)) load_stage(p, L, T, kb, in_ring + (size_t)s * p.in_stride, tid, &sh.in_full[s]);
+                PT(if (p.prof) wiss += clock64() - tl0;)
                 // completion tracked by the barrier (the loader moves on to the next stage / task at once)
                 ptx::cp_async_arrive_noinc(&sh.in_full[s]);
             }
         }
         if (p.prof && tid == 0) {
-            unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
-            r[0] = wq; r[1] = wdep; r[2] = wbuf; r[3] = clock64() - t_start;
+            unsigned long long *r = p.prof + (size_t)blockIdx.x * 32;
+            r[0] = wq; r[1] = wdep; r[2] = wbuf; r[3] = clock64() - t_start; r[20] = wiss; r[21] = wbar;
         }
     } else if (warp == kWProd) {
         // ------------------------------------------------------------------ weight producer
@@ -995,7 +1009,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             }
         }
         if (p.prof && lane == 0) {
-            unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
+            unsigned long long *r = p.prof + (size_t)blockIdx.x * 32;
             r[4] = ww; r[5] = clock64() - t_start;
         }
     } else if (warp == kMma) {
@@ -1040,7 +1054,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     pwait(p, &sh.wfull[st], (gw / p.nw) & 1, wwt);
                     ptx::tc_fence_after();
                     const uint32_t b_base = ptx::smem_u32(w_ring + (size_t)st * p.w_stride) >> 4;
-                    const int q0 = j * L.kpw, q1 = (p.dbg & 1) ? q0 + 1 : min(L.stk ? L.nks / 3 : L.nks, q0 + L.kpw);
+                    const int q0 = j * L.kpw, q1 = DBG(p, 1) ? q0 + 1 : min(L.stk ? L.nks / 3 : L.nks, q0 + L.kpw);
                     const uint64_t a_d0 = ad_t + a_base;
                     uint64_t bd = bd_t + b_base;
                     if (STK && L.stk) {
@@ -1132,13 +1146,13 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             __syncwarp();
         }
         if (p.prof && lane == 0) {
-            unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
+            unsigned long long *r = p.prof + (size_t)blockIdx.x * 32;
             r[6] = wdesc; r[7] = wacc; r[8] = win; r[9] = wwt; r[10] = clock64() - t_start; r[15] = wfence;
         }
     } else {
         // ------------------------------------------------------------------ epilogue
         const int ew = warp - kEpi0;
-        unsigned long long wed = 0, wea = 0, web = 0;
+        unsigned long long wed = 0, wea = 0, web = 0, wtm = 0, wit = 0, wpub = 0, ntask = 0, ncomp = 0;
         const unsigned long long t_start = clock64();
         const int quad = warp % 4;        // TMEM lane quadrant this warp may access
         const int rank = ew / 4;          // 4 warps per quadrant split the (tile, column batch) items
@@ -1157,8 +1171,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             const int ncb = L.Nc / CB;
             const int Tdv = STK ? L.Td : 1;          // output planes per task (stacked 3-D layers)
             const int items = L.ntl * ncb * Tdv;
-            __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(L.out.ptr);
             const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(L.res.ptr);
+            __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(L.out.ptr);
             const int d = T.d;
             __nv_bfloat16 *scr = T.dst_scr ? reinterpret_cast<__nv_bfloat16 *>(scr_slot(p, T.slot) + L.scr_off) : nullptr;
             if (L.pool) {
@@ -1179,6 +1193,9 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                         const int tl = it / ng, cbl = it - tl * ng;
                         const int ch0 = T.nc * L.Nc + (cb0 + cbl) * CB;
                         const int m = tl * 128 + quad * 32 + lane;
+                        // one coalesced bias load per item (lane c holds channel ch0 + c), issued before the TMEM load;
+                        // lanes take their channels' values by shuffle
+                        const float bl = __ldg(L.bias + ch0 + (lane & (CB - 1)));
                         uint32_t r[2][16];
                         const uint32_t taddr =
                             tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) + tl * L.Nc + (cb0 + cbl) * CB;
@@ -1191,12 +1208,9 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                         for (int k = 0; k < 4; k++) {
                             if (k >= nck) break;
                             float v[8];
-                            const float4 b0 = __ldg(reinterpret_cast<const float4 *>(L.bias + ch0 + k * 8));
-                            const float4 b1 = __ldg(reinterpret_cast<const float4 *>(L.bias + ch0 + k * 8 + 4));
-                            const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
                             for (int e = 0; e < 8; e++) {
-                                v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]) + bb[e];
+                                v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]) + __shfl_sync(0xffffffffu, bl, k * 8 + e);
                                 if (L.relu) v[e] = fmaxf(v[e], 0.f);
                             }
                             stg[m * nchk + ((cbl * nck + k) ^ (m & (nchk - 1)))] =
@@ -1243,6 +1257,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");   // staging reused by the next group
                 }
             }
+            PT(const unsigned long long ti0 = p.prof ? clock64() : 0;)
             for (int it = rank; it < (L.pool ? 0 : items); it += 4) {
                 const int o = STK ? it / (L.ntl * ncb) : 0, itr = it - o * (L.ntl * ncb);   // output plane of the task
                 const int tl = itr / ncb, cb = itr - tl * ncb;
@@ -1254,35 +1269,45 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 if (i < L.Tb && j < L.Tw && d < T.hi[0] && y < T.hi[1] && x < T.hi[2] && (!p.padded || x >= T.dlo[2]))
                     kind = (d < L.out_ext[0] && y < L.out_ext[1] && x < L.out_ext[2]) ? 2 : 1;
                 const int ch0 = T.nc * L.Nc + cb * CB;
+                // global reads ahead of their use: one coalesced bias load per item (lane c holds channel ch0 + c,
+                // shuffled out below) and the residual one 16-B chunk ahead (issued before the store of the previous
+                // chunk, which the compiler may not move it past).  Measured on B200 against per-chunk bias loads and
+                // in-order residual loads: cfg4 11.46 -> 11.25 ms, cfg3 7.28 -> 7.16 ms; all four residual chunks up
+                // front (registers), two chunks ahead, or 16-channel items with the next item's reads in flight were slower.
+                const float bl = DBG(p, 8) ? 0.f : __ldg(L.bias + ch0 + (lane & (CB - 1)));
+                const bool has_rs = L.has_res && kind == 2 && !DBG(p, 16);
+                const uint4 *rsp = has_rs ? reinterpret_cast<const uint4 *>(resp + pix_pow2(L.res, L.lB, T.n, d, y, x) + ch0) : nullptr;
+                uint4 rnext = make_uint4(0, 0, 0, 0);
+                if (has_rs) rnext = __ldcg(rsp);
                 uint32_t r[2][16];
                 const uint32_t taddr = tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) +
                                        tl * (Tdv * L.Nc) + (Tdv - 1 - o) * L.Nc + cb * CB;
+                PT(const unsigned long long tt0 = p.prof ? clock64() : 0;)
                 ptx::tmem_ld16(taddr, r[0]);
                 if (CB == 32) ptx::tmem_ld16(taddr + 16, r[1]);
                 ptx::tmem_ld_wait();
                 ptx::reg_fence16(r[0]);
                 ptx::reg_fence16(r[1]);
-                if (!kind) continue;
+                PT(if (p.prof) wtm += clock64() - tt0;)
+                if (!__any_sync(0xffffffffu, kind != 0)) continue;   // (warp-uniform: the bias shuffles need every lane)
                 uint4 *dst = reinterpret_cast<uint4 *>(
                     T.dst_scr ? scr + ((((long long)(d - T.dlo[0]) * L.pR[1] + (y - T.dlo[1])) * L.pR[2] + (x - T.dlo[2])) *
                                            L.cout + ch0)
                               : outp + pix_pow2(L.out, L.lB, T.n, d, y, x) + ch0);
-                if (kind == 1) {
-                    for (int k = 0; k < CB / 8; k++) dst[k] = make_uint4(0, 0, 0, 0);
-                    continue;
-                }
-                const uint4 *rs = L.has_res ? reinterpret_cast<const uint4 *>(resp + pix_pow2(L.res, L.lB, T.n, d, y, x) + ch0) : nullptr;
 #pragma unroll
                 for (int k = 0; k < 4; k++) {
                     if (k >= CB / 8) break;
                     float v[8];
-                    const float4 b0 = __ldg(reinterpret_cast<const float4 *>(L.bias + ch0 + k * 8));
-                    const float4 b1 = __ldg(reinterpret_cast<const float4 *>(L.bias + ch0 + k * 8 + 4));
-                    const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
-                    for (int e = 0; e < 8; e++) v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]) + bb[e];
-                    if (rs) {
-                        const uint4 rr = __ldcg(rs + k);
+                    for (int e = 0; e < 8; e++)
+                        v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]) + __shfl_sync(0xffffffffu, bl, k * 8 + e);
+                    if (kind != 2) {
+                        if (kind == 1) dst[k] = make_uint4(0, 0, 0, 0);
+                        continue;
+                    }
+                    if (has_rs) {
+                        const uint4 rr = rnext;
+                        if (k + 1 < CB / 8) rnext = __ldcg(rsp + k + 1);
                         const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr);
 #pragma unroll
                         for (int e = 0; e < 4; e++) {
@@ -1295,10 +1320,11 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
 #pragma unroll
                         for (int e = 0; e < 8; e++) v[e] = fmaxf(v[e], 0.f);
                     }
-                    if (!(p.dbg & 4))
+                    if (!DBG(p, 4))
                         dst[k] = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
                 }
             }
+            PT(if (p.prof) { wit += clock64() - ti0; ntask++; })
             ptx::tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&sh.acc_empty[a]);
@@ -1307,15 +1333,26 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");
             if (p.prof) web += clock64() - tb0;
             if (ew == 0 && lane == 0) {
-                __threadfence();
-                if (p.padded) atomicMax_block(&sh.done_seq, (int)seq + 1);
-                else if (p.only_layer < 0) st_release(status_word(p, l, t), (int)(EP | 2));
-                atomicAdd(&p.counters[0], 1ULL);
+                PT(const unsigned long long tp0 = p.prof ? clock64() : 0;)
+                if (p.padded) {
+                    // CTA-local hand-off to this CTA's loaders, which read the scratch through L2 (cp.async.cg)
+                    __threadfence();
+                    atomicMax_block(&sh.done_seq, (int)seq + 1);
+                } else if (p.only_layer < 0) {
+                    // the release store is cumulative over the epilogue warps' stores ordered before it by the named
+                    // barrier (the bar.sync + st.release.gpu publication pattern; no separate membar.gl, which cost
+                    // ~1 us per task: measured)
+                    st_release(status_word(p, l, t), (int)(EP | 2));
+                }
+                ncomp++;
+                PT(if (p.prof) wpub += clock64() - tp0;)
             }
         }
+        if (ew == 0 && lane == 0 && ncomp) atomicAdd(&p.counters[0], ncomp);   // tasks computed by this CTA
         if (p.prof && ew == 0 && lane == 0) {
-            unsigned long long *r = p.prof + (size_t)blockIdx.x * 16;
+            unsigned long long *r = p.prof + (size_t)blockIdx.x * 32;
             r[11] = wed; r[12] = wea; r[13] = web; r[14] = clock64() - t_start;
+            r[16] = wtm; r[17] = wit; r[18] = wpub; r[19] = ntask;
         }
     }
     ptx::tc_fence_before();
@@ -1576,8 +1613,8 @@ static unsigned long long *gen_prof_buf = nullptr;
 static unsigned long long *gen_prof_buffer(cudaStream_t s) {
     static const bool on = getenv("BDL_GEN_PROF") != nullptr;
     if (!on) return nullptr;
-    if (!gen_prof_buf) cudaMalloc(&gen_prof_buf, 1024 * 16 * 8);
-    cudaMemsetAsync(gen_prof_buf, 0, 1024 * 16 * 8, s);
+    if (!gen_prof_buf) cudaMalloc(&gen_prof_buf, 1024 * 32 * 8);
+    cudaMemsetAsync(gen_prof_buf, 0, 1024 * 32 * 8, s);
     return gen_prof_buf;
 }
 
@@ -2071,6 +2108,6 @@ extern "C" int bdl_debug_gen_prof(unsigned long long *host, int max_ctas) {
     if (!bdl::gen_prof_buf) return 0;
     const int n = max_ctas < 1024 ? max_ctas : 1024;
     cudaDeviceSynchronize();
-    cudaMemcpy(host, bdl::gen_prof_buf, (size_t)n * 16 * 8, cudaMemcpyDeviceToHost);
+    cudaMemcpy(host, bdl::gen_prof_buf, (size_t)n * 32 * 8, cudaMemcpyDeviceToHost);
     return n;
 }

@@ -1,7 +1,7 @@
 """Per-role wait/busy split of the generic tcgen05 kernel, per subgraph (debug, BDL_GEN_PROF).
     python tools/gen_prof.py cfg4 [subgraph ...]"""
 import ctypes, os, sys
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.environ.get("BDL_ROOT") or os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 os.environ["BDL_GEN_PROF"] = "1"
 import numpy as np, torch
 from paper_conf_icpp_lakshminarasimhan24_b200 import engine, workloads, lib
@@ -20,9 +20,9 @@ for i in ids:
     if sgs[i]["kernel"] != "tcgen05 generic":
         continue
     plan.run_subgraph(i, xb, yb); torch.cuda.synchronize()
-    buf = (ctypes.c_ulonglong * (1024 * 16))()
+    buf = (ctypes.c_ulonglong * (1024 * 32))()
     f(buf, 1024)
-    a = np.frombuffer(buf, dtype=np.uint64).reshape(1024, 16).astype(np.float64)
+    a = np.frombuffer(buf, dtype=np.uint64).reshape(1024, 32).astype(np.float64)
     a = a[a[:, 3] > 0]
     m = a.mean(axis=0)
     ls = wl["layers"][sgs[i]["first"]:sgs[i]["last"] + 1]
@@ -30,3 +30,7 @@ for i in ids:
     print(f"sg {i} {sgs[i]['mode']} {desc}: ctas {len(a)}  total {m[14]/1.9e3:.0f} us")
     print("   " + "  ".join(f"{n} {100*m[k]/max(m[14],1):.0f}%" for k, n in enumerate(names) if k not in (3, 5, 10, 14)))
     print(f"   per-role totals (us): loader {m[3]/1.9e3:.0f} wprod {m[5]/1.9e3:.0f} mma {m[10]/1.9e3:.0f} epi {m[14]/1.9e3:.0f}")
+    nt = max(m[19], 1)
+    print(f"   per task (us, {nt:.0f} tasks/CTA): epi items {m[17]/nt/1.9e3:.2f} (tmem {m[16]/nt/1.9e3:.2f}) "
+          f"publish {m[18]/nt/1.9e3:.2f} bar {m[13]/nt/1.9e3:.2f} acc_wait {m[12]/nt/1.9e3:.2f} | "
+          f"loader issue {m[20]/nt/1.9e3:.2f} bar1 {m[21]/nt/1.9e3:.2f} deps {m[1]/nt/1.9e3:.2f} in_empty {m[2]/nt/1.9e3:.2f}")

@@ -6,7 +6,7 @@ import argparse
 import os
 import sys
 
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.environ.get("BDL_ROOT") or os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 
 from paper_conf_icpp_lakshminarasimhan24_b200 import engine, workloads
