@@ -2023,6 +2023,9 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
                  gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, 2 * G.Tw / p->in_layout.Bw, 2))
             G.tma = 2;
         G.has_res = sg.res_tensor[j] >= 0 || G.resl >= 0;
+        if (getenv("BDL_GEN_GEOM"))
+            fprintf(stderr, "gen sg[%d..%d] layer %d: tma %d amode %d s %d,%d k %d,%d Tb %d Tw %d nkb %d\n", sg.first, sg.last, j,
+                    G.tma, G.amode, G.s[1], G.s[2], G.k[1], G.k[2], G.Tb, G.Tw, G.nkb);
         if (sg.res_tensor[j] >= 0) G.res = res[j];
         else if (G.resl >= 0) G.res = outs[G.resl];
         G.relu = ly.L.relu;
