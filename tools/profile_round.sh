@@ -26,6 +26,11 @@ for c in cfg3 cfg4 cfg5; do
       --log-file gpurun_out/${R}_launches_$c.csv python bench.py --config $c --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn > /dev/null 2>&1
   echo launches_$c=$?
 done
+for c in cfg2 cfg3 cfg4 cfg5; do   # merged-side DRAM bytes of one forward (the layer-by-layer side: tools/dram_bytes.py --impl lbl)
+  timeout 600 ncu --nvtx --nvtx-include "fwd/" --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
+      --csv --log-file gpurun_out/${R}_dram_${c}_merged.csv python tools/dram_bytes.py run --impl merged --config $c > /dev/null 2>&1
+  echo dram_$c=$?
+done
 CASES='tests/test_gpu_gen.py -k "sw128_chain_grow or planes_3d or s2_1x1_proj or dag_bottlenecks_s1 or pool_fused_stem or dilated_chain_d2"'
 for tool in memcheck synccheck racecheck; do
   eval timeout 1200 compute-sanitizer --tool $tool --print-limit 20 --target-processes all \
