@@ -669,7 +669,6 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
         // row 2 * (y0 + i); one TMA box per row picks every other pixel (element stride 2 along x in brick)
         // and lands the Tw pixels contiguously at block row i.
         const int l = (int)(&L - p.layer);
-        bool wrote = false;   // generic-proxy shared-memory writes (zero-filled rows) by this thread
         for (int i = w; i < L.Tb; i += kLW) {
             const int y = y0 + 2 * i;
             uint8_t *dst = buf + (size_t)(i * L.Wp) * 128;
@@ -683,10 +682,9 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
             } else {
                 for (int q = lane; q < L.Tw * 8; q += 32)
                     *reinterpret_cast<uint4 *>(dst + (size_t)(q >> 3) * 128 + ((q & 7) << 4)) = make_uint4(0, 0, 0, 0);
-                wrote = true;
             }
         }
-        if (wrote) ptx::fence_proxy_async_smem();   // zero-filled rows (generic stores) -> tcgen05 operand reads
+        ptx::fence_proxy_async_smem();
         return;
     }
     if (L.tma && !T.src_scr) {
@@ -704,7 +702,6 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
         // 2.45 -> 2.04 ms with per-thread rows, while per-thread rows cost cfg3 / cfg4 1.5-3.5 %.
         const int rstep = sw64 ? kLoadT : kLW, rbeg = sw64 ? tid : w;
         const int hstep = sw64 ? 1 : 32, hbeg = sw64 ? 0 : lane;
-        bool wrote = false;   // generic-proxy shared-memory writes (zero fill, cp.async halos) by this thread
         for (int r2 = rbeg; r2 < nrow; r2 += rstep) {
             const int a = r2 / L.in_rows, yy = r2 - a * L.in_rows;
             const int z = z0 + a, y = y0 + yy;
@@ -722,9 +719,7 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
                 for (int q = hbeg; q < L.Tw * nchr; q += hstep)
                     *reinterpret_cast<uint4 *>(buf + ((size_t)(rowpx + pdw) << lrb) + ((size_t)q << 4)) =
                         make_uint4(0, 0, 0, 0);
-                wrote = true;
             }
-            wrote = wrote || hbeg < nh * nchr;
             const long long rowlog = (((long long)T.n * v.nb[1] + bz) * v.nb[2] + by) * v.nb[3];
             const int rowin = ((z - (bz << lBd)) << lBh) + (y - (by << lBh));
             for (int q = hbeg; q < nh * nchr; q += hstep) {
@@ -743,7 +738,7 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
                 ptx::cp_async16(buf + off, g, ok ? 16u : 0u);
             }
         }
-        if (wrote) ptx::fence_proxy_async_smem();   // zero-filled rows, halo chunks (generic) -> tcgen05 operand reads
+        ptx::fence_proxy_async_smem();   // zero-filled rows (generic stores) -> tcgen05 operand reads
         return;
     }
     for (int r2 = w; r2 < nrow; r2 += kLW) {
@@ -950,9 +945,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             PT(const unsigned long long tlb = p.prof ? clock64() : 0;)
             asm volatile("bar.sync 1, %0;" ::"n"(kLoadT) : "memory");
             PT(if (p.prof) wbar += clock64() - tlb;)
-            // acquired data is read by TMA (async proxy): the threads that issue the TMA loads (lane 0 of each warp; every
-            // thread for one-row-per-thread SW64 stages)
-            if (l >= 0 && p.layer[l].tma && (lane == 0 || p.layer[l].amode == AM_SW64)) ptx::fence_proxy_async();
+            if (l >= 0 && p.layer[l].tma) ptx::fence_proxy_async();   // acquired data is read by TMA (async proxy)
             if (tid == 0) {
                 sh.desc_l[seq % kRing] = l;
                 sh.desc_t[seq % kRing] = t;
