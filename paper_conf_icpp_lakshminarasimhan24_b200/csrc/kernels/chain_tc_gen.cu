@@ -1420,6 +1420,22 @@ constexpr int kGenInBudget = 112 * 1024;   // input-stage ring
 constexpr int kGenWStage = 32 * 1024;      // one weight stage
 constexpr int kGenW = 3;                   // weight stages
 constexpr double kGenTaskOverheadMmas = 96.0;   // fixed per-task cost in units of one 128-row MMA (tile model)
+// Shallow-K subgraphs (FLOP-weighted mean reduction length cin * taps below this) run 2 weight stages and give the
+// third to the input ring: larger input stages, larger tiles, fewer tasks, where the weights streamed per task are
+// small.  Measured on B200 (same box, all plain subgraphs switched): ResNet-50 conv2_x / conv3_x subgraphs (mean K
+// 340-900) 2.20 -> 2.01, 2.96 -> 2.64, 1.72 -> 1.66 ms; deep-K subgraphs lose (VGG-16 conv3-5, K 2000-4600: +4-11 %;
+// ResNet-50 conv5_x +4-8 %).
+constexpr double kGenShallowK = 1024.0;
+// A/B knobs of the tile model (host only): BDL_GEN_OVH overrides the per-task cost; BDL_GEN_NW2 = 0 / 1 forces 3 / 2
+// weight stages for plain (unstacked, pool-free) subgraphs instead of the shallow-K rule
+static double gen_task_overhead() {
+    static const double v = [] { const char *e = getenv("BDL_GEN_OVH"); return e ? atof(e) : kGenTaskOverheadMmas; }();
+    return v;
+}
+static int gen_nw2() {
+    static const int v = [] { const char *e = getenv("BDL_GEN_NW2"); return e ? atoi(e) : -1; }();
+    return v;
+}
 
 // BDL_GEN_STACK=0: no depth stacking (A/B runs)
 static bool gen_stack_ok() {
@@ -1561,7 +1577,7 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
                 mmas = (double)cand.ntl * (G.nks / 3) * w;
             }
             // per output plane: tasks / Td
-            const double cost = (double)nty * ntx / Td * (mmas + kGenTaskOverheadMmas) * (1.0 + 0.1 * (halo - 1.0));
+            const double cost = (double)nty * ntx / Td * (mmas + gen_task_overhead()) * (1.0 + 0.1 * (halo - 1.0));
             const double score = -cost + 1e-6 * Ub * Uw * Td;
             if (score > best) {
                 best = score;
@@ -1671,7 +1687,19 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
     bool any_stk = false;
     for (int j = 0; j < nconv; j++) any_stk = any_stk || g.layer[j].stk;
     const bool stk_geo = any_stk && !padded && max_td_env > 1;
-    const int in_budget = stk_geo ? kGenInBudget + (kGenW - stk_nw_env) * kGenWStage : kGenInBudget;
+    double kf = 0, f = 0;   // FLOP-weighted mean reduction length of the subgraph's convs
+    for (int j = 0; j < nconv; j++) {
+        const Layer &ly = p->layers[sg.first + j];
+        const double K = (double)ly.L.cin / std::max(1, (int)ly.L.groups) * ly.L.k[0] * ly.L.k[1] * ly.L.k[2];
+        const double F = K * ly.L.cout * ly.out_ext[1] * ly.out_ext[2] * ly.out_ext[3];
+        kf += K * F;
+        f += F;
+    }
+    const bool shallow = f > 0 && kf / f < kGenShallowK;
+    const bool nw2 = !stk_geo && !fused && (gen_nw2() < 0 ? shallow : gen_nw2() == 1);
+    const int in_budget = stk_geo ? kGenInBudget + (kGenW - stk_nw_env) * kGenWStage
+                          : nw2   ? kGenInBudget + kGenWStage
+                                  : kGenInBudget;
     if (fused) {   // the pool's output is the last conv's task grid
         gen::LayerP &G = g.layer[nconv - 1];
         const Layer &pl = p->layers[sg.last];
@@ -1769,7 +1797,7 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
     g.in_stride = in_stride;
     g.w_stride = (w_stride + 1023) / 1024 * 1024;
     g.nin = std::min(gen::kMaxIn, in_budget / in_stride);
-    g.nw = g.pool_bytes ? kGenW - 1 : stk_geo ? stk_nw_env : kGenW;
+    g.nw = g.pool_bytes ? kGenW - 1 : stk_geo ? stk_nw_env : nw2 ? kGenW - 1 : kGenW;
     if (g.pool_bytes > kGenWStage) return false;
     g.acc_stride = acc;
     g.nacc = 2 * acc <= 512 ? 2 : 1;
