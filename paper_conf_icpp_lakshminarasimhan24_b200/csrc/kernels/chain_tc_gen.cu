@@ -687,6 +687,50 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
         ptx::fence_proxy_async_smem();
         return;
     }
+    if (L.tma == 3 && !T.src_scr) {
+        // 3x3 stride-2 SW128 layer (padding 1): polyphase block (yr, xr) holds input pixels (2 yq + yr, 2 xq + xr) of the
+        // window starting at (y0, x0) = (2 Y - 1, 2 X - 1).  Per input row, two TMA boxes with element stride 2 along x
+        // fetch the Tw interior even columns 2X, 2X + 2, ... into block (yr, 1) at xq = 0..Tw-1 and the Tw odd columns
+        // 2X + 1, ... into block (yr, 0) at xq = 1..Tw; the two halo pixels 2X - 1 (block (yr, 0), xq 0) and 2X + 2Tw
+        // (block (yr, 1), xq Tw) come by cp.async; rows outside the image are zero-filled.
+        const int l = (int)(&L - p.layer);
+        const int X = T.x0 * 2;   // first interior input column: brick aligned (Tw % Bw == 0)
+        for (int yy = w; yy < L.in_rows; yy += kLW) {
+            const int y = y0 + yy;
+            const int rowpx0 = (yy & 1) * 2 * L.blk_px + (yy >> 1) * L.Wp, rowpx1 = rowpx0 + L.blk_px;
+            const bool rok = y >= 0 && y < L.in_ext[1];
+            const int by = y >> lBh, yin = y - (by << lBh);
+            if (rok) {
+                if (lane == 0) {
+                    ptx::mbar_expect_tx(bar, 2u * (uint32_t)L.Tw * 128u);
+                    ptx::tma_load_5d(buf + (size_t)rowpx1 * 128, &p.tm_row[l], kb * 64, 0, X >> lBw, yin,
+                                     T.n * v.nb[2] + by, bar);
+                    ptx::tma_load_5d(buf + (size_t)(rowpx0 + 1) * 128, &p.tm_row[l], kb * 64, 1, X >> lBw, yin,
+                                     T.n * v.nb[2] + by, bar);
+                }
+            } else {
+                for (int q = lane; q < 2 * L.Tw * 8; q += 32) {
+                    const int px = q < L.Tw * 8 ? rowpx1 + (q >> 3) : rowpx0 + 1 + ((q - L.Tw * 8) >> 3);
+                    *reinterpret_cast<uint4 *>(buf + (size_t)px * 128 + (((q & 7) ^ (px & 7)) << 4)) = make_uint4(0, 0, 0, 0);
+                }
+            }
+            if (lane < 16) {   // halo pixels: 8 16-B chunks each
+                const int side = lane >> 3, ch = lane & 7;
+                const int x = side ? X + 2 * L.Tw : X - 1;
+                const int px = side ? rowpx1 + L.Tw : rowpx0;
+                const bool ok = rok && x >= 0 && x < L.in_ext[2];
+                const void *g = base;
+                if (ok) {
+                    const int bx = x >> lBw;
+                    g = base + ((((long long)T.n * v.nb[1]) * v.nb[2] + by) * v.nb[3] + bx) * v.brick_elems +
+                        (long long)((yin << lBw) + (x - (bx << lBw))) * v.Cp + kb * 64 + ch * 8;
+                }
+                ptx::cp_async16(buf + (size_t)px * 128 + ((ch ^ (px & 7)) << 4), g, ok ? 16u : 0u);
+            }
+        }
+        ptx::fence_proxy_async_smem();   // zero-filled rows (generic stores) -> tcgen05 operand reads
+        return;
+    }
     if (L.tma && !T.src_scr) {
         // stride-1 swizzled rows (SW128: 64-channel K-block rows of 128 B; SW64: 32-channel rows of 64 B): the
         // Tw in-tile columns of an in-image row by one TMA box (completion on `bar` by transaction count), halo
@@ -1436,6 +1480,10 @@ static int gen_nw2() {
     static const int v = [] { const char *e = getenv("BDL_GEN_NW2"); return e ? atoi(e) : -1; }();
     return v;
 }
+static int gen_nw_force() {   // BDL_GEN_NW = 1..4: weight stages of every plain subgraph (A/B)
+    static const int v = [] { const char *e = getenv("BDL_GEN_NW"); return e ? atoi(e) : 0; }();
+    return v;
+}
 
 // BDL_GEN_STACK=0: no depth stacking (A/B runs)
 static bool gen_stack_ok() {
@@ -1594,6 +1642,11 @@ static bool gen_tma_ok() {
     static const int v = [] { const char *e = getenv("BDL_GEN_TMA"); return e ? atoi(e) : 1; }();
     return v != 0;
 }
+// 3x3 stride-2 layers by element-strided TMA rows (BDL_GEN_TMA3=0: cp.async, for A/B runs)
+static bool gen_tma3_ok() {
+    static const int v = [] { const char *e = getenv("BDL_GEN_TMA3"); return e ? atoi(e) : 1; }();
+    return v != 0;
+}
 // Padded-mode first layer eligible for TMA rows (stride 1, swizzled A layout, 2-D or SW64 3-D)?
 static bool gen_pad_tma_ok(const gen::LayerP &G, int nsp, int Bw) {
     if (!gen_tma_ok() || G.s[0] != 1 || G.s[1] != 1 || G.s[2] != 1 || Bw > 256) return false;
@@ -1697,9 +1750,10 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
     }
     const bool shallow = f > 0 && kf / f < kGenShallowK;
     const bool nw2 = !stk_geo && !fused && (gen_nw2() < 0 ? shallow : gen_nw2() == 1);
+    const int nwp = (!stk_geo && !fused && gen_nw_force() >= 1 && gen_nw_force() <= gen::kMaxW) ? gen_nw_force()
+                    : nw2 ? kGenW - 1 : kGenW;   // weight stages of a plain subgraph
     const int in_budget = stk_geo ? kGenInBudget + (kGenW - stk_nw_env) * kGenWStage
-                          : nw2   ? kGenInBudget + kGenWStage
-                                  : kGenInBudget;
+                                  : kGenInBudget + (kGenW - nwp) * kGenWStage;
     if (fused) {   // the pool's output is the last conv's task grid
         gen::LayerP &G = g.layer[nconv - 1];
         const Layer &pl = p->layers[sg.last];
@@ -1797,7 +1851,7 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
     g.in_stride = in_stride;
     g.w_stride = (w_stride + 1023) / 1024 * 1024;
     g.nin = std::min(gen::kMaxIn, in_budget / in_stride);
-    g.nw = g.pool_bytes ? kGenW - 1 : stk_geo ? stk_nw_env : nw2 ? kGenW - 1 : kGenW;
+    g.nw = g.pool_bytes ? kGenW - 1 : stk_geo ? stk_nw_env : nwp;
     if (g.pool_bytes > kGenWStage) return false;
     g.acc_stride = acc;
     g.nacc = 2 * acc <= 512 ? 2 : 1;
@@ -2050,6 +2104,11 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
                  G.Tw % p->in_layout.Bw == 0 && 2 * G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
                  gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, 2 * G.Tw / p->in_layout.Bw, 2))
             G.tma = 2;
+        else if (!padded && G.amode == gen::AM_SW128 && G.k[0] == 1 && G.ke[1] == 3 && G.ke[2] == 3 && G.s[1] == 2 &&
+                 G.s[2] == 2 && G.pd[1] == 1 && G.pd[2] == 1 && nsp == 2 && !G.src.bmap && G.Tw % p->in_layout.Bw == 0 &&
+                 2 * G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 && gen_tma_ok() && gen_tma3_ok() &&
+                 gen_encode_row_map(&P.tm_row[j], G.src, 2 * G.Tw / p->in_layout.Bw, 2))
+            G.tma = 3;   // 3x3 stride-2 rows: two element-strided TMA boxes (even / odd columns) per input row
         G.has_res = sg.res_tensor[j] >= 0 || G.resl >= 0;
         if (getenv("BDL_GEN_GEOM"))
             fprintf(stderr, "gen sg[%d..%d] layer %d: tma %d amode %d s %d,%d k %d,%d Tb %d Tw %d nkb %d\n", sg.first, sg.last, j,
