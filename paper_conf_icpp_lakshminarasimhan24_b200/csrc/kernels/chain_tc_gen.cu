@@ -209,6 +209,14 @@ __device__ __forceinline__ long long pix(const TView &v, int n, int d, int y, in
 }
 
 // First conv-output row / column of tile (ty, tx) (pooled layers: under its first pool window; may be < 0).
+// Fused pool: channel batches staged together in the epilogue -- a power of two (the staging tile's XOR swizzle
+// masks with the chunk count), <= 4 / M tiles so the 4 warp ranks share ntl x gcb items
+__host__ __device__ __forceinline__ int pool_gcb(int ncb, int ntl) {
+    int g = ncb < 4 / ntl ? ncb : 4 / ntl;
+    if (g < 1) g = 1;
+    while (g & (g - 1)) g &= g - 1;
+    return g;
+}
 __host__ __device__ __forceinline__ int tile_y0(const LayerP &L, int ty) {
     return L.pool ? ty * L.Tpb * L.ps[0] - L.ppd[0] : ty * L.Tb;
 }
@@ -1229,7 +1237,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 const int nck = CB / 8;
                 // channel batches staged together: the 4 warp ranks share ntl x gcb (tile, batch) items, so every
                 // epilogue warp reads TMEM even when a task has a single M tile; staging <= ntl*128 x 128 ch
-                const int gcb = min(ncb, max(1, 4 / L.ntl));
+                const int gcb = pool_gcb(ncb, L.ntl);
                 const int nchk = gcb * nck;   // 16-B chunks per staged position (a power of two)
                 for (int cb0 = 0; cb0 < ncb; cb0 += gcb) {
                     const int ng = min(gcb, ncb - cb0);
@@ -1262,11 +1270,13 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                         }
                     }
                     asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");
-                    const int nc_g = ng * nck;
+                    const int nc_g = ng * nck;                // (a power of two unless the last, partial group)
+                    const int lnc = 31 - __clz(nc_g);
                     const int nout = L.Tpb * L.Tpw * nc_g;
                     for (int q = ew * 32 + lane; q < nout; q += 32 * kEpiW) {
-                        const int ck = q % nc_g, o = q / nc_g;
-                        const int ox = o % L.Tpw, oy = o / L.Tpw;
+                        const int ck = (nc_g & (nc_g - 1)) ? q % nc_g : q & (nc_g - 1);
+                        const int o = (nc_g & (nc_g - 1)) ? q / nc_g : q >> lnc;
+                        const int oy = o / L.Tpw, ox = o - oy * L.Tpw;
                         const int py = T.py0 + oy, px = T.px0 + ox;
                         if (d >= T.hi[0] || py >= T.hi[1] || px >= T.hi[2]) continue;
                         if (p.padded && (py < T.dlo[1] || px < T.dlo[2])) continue;
@@ -1276,24 +1286,22 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                             *dst = make_uint4(0, 0, 0, 0);
                             continue;
                         }
-                        __nv_bfloat162 mx[4];
-                        bool any = false;
-                        for (int rr = 0; rr < L.pk[0]; rr++) {
-                            const int i = oy * L.ps[0] + rr, y = T.y0 + i;
-                            if (y < 0 || y >= L.out_ext[1]) continue;
-                            for (int cc = 0; cc < L.pk[1]; cc++) {
-                                const int j = ox * L.ps[1] + cc, x = T.x0 + j;
-                                if (x < 0 || x >= L.out_ext[2]) continue;
-                                const int m = i * L.Wp + j;
+                        // the window's taps inside the conv output (out-of-range taps ignored; pad < k keeps
+                        // at least one): bounds hoisted out of the tap loops, the max starts from -inf
+                        const int i0 = oy * L.ps[0], j0 = ox * L.ps[1];
+                        const int rlo = max(0, -(T.y0 + i0)), rhi = min(L.pk[0], L.out_ext[1] - (T.y0 + i0));
+                        const int clo = max(0, -(T.x0 + j0)), chi = min(L.pk[1], L.out_ext[2] - (T.x0 + j0));
+                        const __nv_bfloat162 ninf = __halves2bfloat162(__ushort_as_bfloat16((unsigned short)0xFF80),
+                                                                       __ushort_as_bfloat16((unsigned short)0xFF80));
+                        __nv_bfloat162 mx[4] = {ninf, ninf, ninf, ninf};
+                        for (int rr = rlo; rr < rhi; rr++) {
+                            const int mrow = (i0 + rr) * L.Wp + j0;
+                            for (int cc = clo; cc < chi; cc++) {
+                                const int m = mrow + cc;
                                 const uint4 u = stg[m * nchk + (ck ^ (m & (nchk - 1)))];
                                 const __nv_bfloat162 *h = reinterpret_cast<const __nv_bfloat162 *>(&u);
-                                if (!any) {
-                                    mx[0] = h[0]; mx[1] = h[1]; mx[2] = h[2]; mx[3] = h[3];
-                                    any = true;
-                                } else {
-                                    mx[0] = __hmax2(mx[0], h[0]); mx[1] = __hmax2(mx[1], h[1]);
-                                    mx[2] = __hmax2(mx[2], h[2]); mx[3] = __hmax2(mx[3], h[3]);
-                                }
+                                mx[0] = __hmax2(mx[0], h[0]); mx[1] = __hmax2(mx[1], h[1]);
+                                mx[2] = __hmax2(mx[2], h[2]); mx[3] = __hmax2(mx[3], h[3]);
                             }
                         }
                         *dst = *reinterpret_cast<const uint4 *>(mx);
@@ -1558,7 +1566,7 @@ static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out,
 // Fused pool: epilogue staging tile, every M row of the conv tile x the channel batches staged together, bf16.
 static int gen_pool_stage_bytes(const gen::LayerP &G) {
     const int CB = G.Nc >= 32 ? 32 : 16, ncb = G.Nc / CB;
-    const int gcb = std::min(ncb, std::max(1, 4 / G.ntl));   // channel batches staged together (epilogue)
+    const int gcb = gen::pool_gcb(ncb, G.ntl);   // channel batches staged together (epilogue)
     return G.ntl * 128 * gcb * CB * 2;
 }
 
