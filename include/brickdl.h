@@ -97,11 +97,12 @@ typedef struct bdl_layer {
                                     [cout][kd][kh][kw][cin/g]; runs on the CUDA-core brick kernels (not a dense contraction) */
 } bdl_layer;
 
-/* Static-analysis knobs (§3.3); bdl_plan_opts_default gives the paper's values. */
+/* Static-analysis knobs (§3.3); bdl_plan_opts_default gives the paper's values, except delta_threshold. */
 typedef struct bdl_plan_opts {
-    double delta_threshold;      /* 0.15: memoized when padding data growth Delta > 15% (L644).  On B200 our
-                                    memoized kernels measured faster than padded on every subgraph tried
-                                    (DESIGN.md §7); a negative value selects memoized everywhere. */
+    double delta_threshold;      /* 0.10: memoized when padding data growth Delta > 10%.  The paper uses 15%
+                                    (L644, "validated on multiple NVIDIA and AMD GPU architectures"); on B200 our
+                                    padded mode lost at Delta = 0.13 (VGG-16 conv1 block: 2.47 vs 2.10 ms) and tied
+                                    at 0.074 and 0.  A negative value selects memoized everywhere. */
     int64_t tau;                 /* 4096: rho threshold, "tau = 2^12" (L656, printed "212") */
     int32_t bcand[4];            /* {4, 8, 16, 32} brick edge candidates (L654) */
     int64_t onchip_budget;       /* bytes a merged subgraph's footprint may use; 0 = device L2 size (L611-614) */

@@ -1712,6 +1712,11 @@ bool gen_pool_fused(const bdl_plan *p, const Subgraph &sg, int nconv, bool padde
     const int mode = p->opts.fuse_pool;   // 0 measured rule, 1 always, 2 never
     if (mode == 2 || nconv < 1 || nconv != sg.last - sg.first) return false;
     if (mode != 1 && (padded || p->layers[sg.first + nconv - 1].L.cout > 128)) return false;
+    // large maps: the staging tile takes the input ring's shallow-K extra stage, and the smaller conv tiles cost more
+    // than the separate pool pass (B200, VGG-16 conv1 block at 224^2: fused 2.10 vs 1.91 ms; at 112^2 fusing wins:
+    // ResNet-50 stem 0.72 -> 0.62 ms, VGG-16 conv2 block 1.10 -> 0.95 ms)
+    const Layer &cl = p->layers[sg.first + nconv - 1];
+    if (mode != 1 && (long long)cl.out_ext[2] * cl.out_ext[3] > 112LL * 112) return false;
     const bdl_layer &pl = p->layers[sg.last].L;
     const int ci = sg.first + nconv - 1;
     if (pl.kind != BDL_OP_MAXPOOL || pl.input != ci) return false;

@@ -47,7 +47,7 @@ const char *bdl_version(void) { return "brickdl-b200 0.1 (sm_100a)"; }
 void bdl_plan_opts_default(bdl_plan_opts *o) {
     if (!o) return;
     std::memset(o, 0, sizeof(*o));
-    o->delta_threshold = 0.15;   // L644
+    o->delta_threshold = 0.10;   // L644's 15 %, recalibrated for these B200 kernels (brickdl.h)
     o->tau = 4096;               // L656, "tau = 2^12"
     o->bcand[0] = 4; o->bcand[1] = 8; o->bcand[2] = 16; o->bcand[3] = 32;  // L654
     o->onchip_budget = 0;

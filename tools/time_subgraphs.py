@@ -19,10 +19,15 @@ def main():
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--N", type=int, default=None)
     ap.add_argument("--max-layers", type=int, default=0)
+    ap.add_argument("--fuse-pool", type=int, default=None)
     a = ap.parse_args()
     wl = workloads.make_workload(a.cfg, N=a.N)
-    plan = engine.plan_from_workload(wl, max_subgraph_layers=a.max_layers) if a.max_layers else \
-        engine.plan_from_workload(wl)
+    kw = {}
+    if a.max_layers:
+        kw["max_subgraph_layers"] = a.max_layers
+    if a.fuse_pool is not None:
+        kw["fuse_pool"] = a.fuse_pool
+    plan = engine.plan_from_workload(wl, **kw)
     if a.mode != "auto":
         plan.set_mode(a.mode)
     xb = plan.brickify(wl["x"])
