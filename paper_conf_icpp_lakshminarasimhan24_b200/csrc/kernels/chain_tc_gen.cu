@@ -739,6 +739,21 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
         ptx::fence_proxy_async_smem();   // zero-filled rows (generic stores) -> tcgen05 operand reads
         return;
     }
+    if (L.tma == 4 && !T.src_scr) {
+        // 1x1 stride-1 layer whose tiles start on a brick row (Tb % Bh == 0, no halo: Wp == Tw): the Bh rows of a brick
+        // row of bricks land as Bh consecutive tile rows of Tw pixels, one TMA box each; rows past the bricked grid are
+        // zero-filled by TMA's out-of-bounds fill
+        const int l = (int)(&L - p.layer);
+        const int Bh = 1 << lBh;
+        for (int b = w; b < (L.Tb >> lBh); b += kLW) {
+            if (lane == 0) {
+                ptx::mbar_expect_tx(bar, (uint32_t)(Bh * L.Tw) * 128u);
+                ptx::tma_load_5d(buf + (size_t)(b * Bh * L.Wp) * 128, &p.tm_row[l], kb * 64, 0, T.x0 >> lBw, 0,
+                                 T.n * v.nb[2] + (y0 >> lBh) + b, bar);
+            }
+        }
+        return;
+    }
     if (L.tma && !T.src_scr) {
         // stride-1 swizzled rows (SW128: 64-channel K-block rows of 128 B; SW64: 32-channel rows of 64 B): the
         // Tw in-tile columns of an in-image row by one TMA box (completion on `bar` by transaction count), halo
@@ -1655,6 +1670,11 @@ static bool gen_tma3_ok() {
     static const int v = [] { const char *e = getenv("BDL_GEN_TMA3"); return e ? atoi(e) : 1; }();
     return v != 0;
 }
+// 1x1 layers by one TMA box per brick row of bricks (BDL_GEN_TMA4=0: one box per pixel row, for A/B runs)
+static bool gen_tma4_ok() {
+    static const int v = [] { const char *e = getenv("BDL_GEN_TMA4"); return e ? atoi(e) : 1; }();
+    return v != 0;
+}
 // Padded-mode first layer eligible for TMA rows (stride 1, swizzled A layout, 2-D or SW64 3-D)?
 static bool gen_pad_tma_ok(const gen::LayerP &G, int nsp, int Bw) {
     if (!gen_tma_ok() || G.s[0] != 1 || G.s[1] != 1 || G.s[2] != 1 || Bw > 256) return false;
@@ -1664,7 +1684,8 @@ static bool gen_pad_tma_ok(const gen::LayerP &G, int nsp, int Bw) {
 
 // 5-D view of a 2-D bricked bf16 tensor (identity BrickMap): (channel, x in brick, brick column, y in brick,
 // brick row over (n, by)); box = 64 channels x Bw x nseg bricks x 1 x 1, 128-B swizzled (the SW128 A layout).
-static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int xstride = 1, int box_ch = 64) {
+static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int xstride = 1, int box_ch = 64,
+                               int rows = 1) {
     static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
     if (!enc) {
         cudaDriverEntryPointQueryResult qr;
@@ -1678,7 +1699,7 @@ static bool gen_encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int xs
     cuuint64_t dims[5] = {(cuuint64_t)v.Cp, (cuuint64_t)v.B[3], (cuuint64_t)v.nb[3], (cuuint64_t)v.B[1] * v.B[2],
                           (cuuint64_t)v.nb[0] * v.nb[1] * v.nb[2]};
     cuuint64_t strides[4] = {px, brick, px * v.B[3], brick * v.nb[3]};
-    cuuint32_t box[5] = {(cuuint32_t)box_ch, (cuuint32_t)v.B[3], (cuuint32_t)nseg, 1, 1};
+    cuuint32_t box[5] = {(cuuint32_t)box_ch, (cuuint32_t)v.B[3], (cuuint32_t)nseg, (cuuint32_t)rows, 1};
     cuuint32_t es[5] = {1, (cuuint32_t)xstride, 1, 1, 1};   // xstride 2: every other pixel of a brick row
     return enc(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, v.ptr, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                box_ch == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
@@ -2098,7 +2119,14 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
         // pooled tiles start at tx * Tpw * ps - pad: TMA rows need that brick-aligned and non-negative
         const bool pool_al = !G.pool || (G.ppd[0] == 0 && G.ppd[1] == 0 && (G.Tpw * G.ps[1]) % p->in_layout.Bw == 0);
         // (padded mode: only the first layer, whose tiles are brick-aligned (xal); later layers read CTA scratch)
+        const int Bh = p->in_layout.Bh;
         if (!pool_al) {
+        } else if (!padded && G.amode == gen::AM_SW128 && G.k[0] == 1 && G.k[1] == 1 && G.k[2] == 1 && G.s[1] == 1 &&
+                   G.s[2] == 1 && G.pd[1] == 0 && G.pd[2] == 0 && nsp == 2 && !G.pool && !G.src.bmap &&
+                   G.Wp == G.Tw && G.Tb % Bh == 0 && G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 &&
+                   Bh <= 256 && G.src.Cp % 64 == 0 && gen_tma_ok() && gen_tma4_ok() &&
+                   gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw, 1, 64, Bh)) {
+            G.tma = 4;   // 1x1 stride-1 layer, brick-row-aligned tiles: one TMA box per Bh rows (the brick's rows)
         } else if ((!padded || G.xal) && G.amode == gen::AM_SW128 && G.s[1] == 1 && G.s[2] == 1 && G.k[0] == 1 && nsp == 2 &&
             !G.src.bmap && G.Tw % p->in_layout.Bw == 0 && G.Tw / p->in_layout.Bw <= 256 && G.src.Cp % 64 == 0 &&
             gen_tma_ok() && gen_encode_row_map(&P.tm_row[j], G.src, G.Tw / p->in_layout.Bw))
