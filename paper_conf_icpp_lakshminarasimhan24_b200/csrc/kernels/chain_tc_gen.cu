@@ -1591,8 +1591,14 @@ static int gen_pool_stage_bytes(const gen::LayerP &G) {
 // the conv tile is the region under their windows, Tb = (Tpb-1)*ps + pk (likewise Tw).
 constexpr int kGenPoolStageMax = 32 * 1024;   // fused pool: largest epilogue staging tile
 
+// Loader cost of a 1x1 stride-1 layer's stage in the tile model (MMA units per TMA box): one box per pixel row, or one
+// per brick row of bricks when the tile height is a multiple of the brick height Bh (the multi-row TMA path).
+static double gen_row_cost() {   // BDL_GEN_ROWC: A/B knob
+    static const double v = [] { const char *e = getenv("BDL_GEN_ROWC"); return e ? atof(e) : 4.0; }();
+    return v;
+}
 static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign, int in_budget = kGenInBudget,
-                            int max_td = 1) {
+                            int max_td = 1, int bh = 0) {
     double best = -1e30;
     bool found = false;
     gen::LayerP cand = G;
@@ -1647,8 +1653,14 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
                 }
                 mmas = (double)cand.ntl * (G.nks / 3) * w;
             }
+            // 1x1 stride-1 layers: TMA boxes per task (see gen_row_cost)
+            double boxes = 0;
+            if (bh > 0 && G.amode == gen::AM_SW128 && G.k[0] == 1 && G.k[1] == 1 && G.k[2] == 1 && G.s[1] == 1 &&
+                G.s[2] == 1 && !G.pool)
+                boxes = (double)G.nkb * (Tb % bh == 0 ? Tb / bh : Tb);
             // per output plane: tasks / Td
-            const double cost = (double)nty * ntx / Td * (mmas + gen_task_overhead()) * (1.0 + 0.1 * (halo - 1.0));
+            const double cost = (double)nty * ntx / Td * (mmas + gen_task_overhead() + gen_row_cost() * boxes) *
+                                (1.0 + 0.1 * (halo - 1.0));
             const double score = -cost + 1e-6 * Ub * Uw * Td;
             if (score > best) {
                 best = score;
@@ -1864,7 +1876,9 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
             // pooled tiles: brick-aligned conv columns (TMA rows) when the windows tile the map (k = s, no padding)
             int walign = p->in_layout.Bw;
             if (G.pool) walign = (G.pk[1] == G.ps[1] && G.ppd[1] == 0 && p->in_layout.Bw % G.ps[1] == 0) ? p->in_layout.Bw / G.ps[1] : 1;
-            if (!gen_layer_tiles(G, G.grid[1], G.grid[2], walign, in_budget, stk_geo ? max_td_env : 1)) return false;
+            if (!gen_layer_tiles(G, G.grid[1], G.grid[2], walign, in_budget, stk_geo ? max_td_env : 1,
+                                 nsp == 2 && gen_tma4_ok() ? p->in_layout.Bh : 0))
+                return false;
             G.ntd = (G.grid[0] + G.Td - 1) / G.Td;   // plane blocks of Td output planes
             const int tb = G.pool ? G.Tpb : G.Tb, tw = G.pool ? G.Tpw : G.Tw;   // pooled: tiles of pool outputs
             G.nty = (G.grid[1] + tb - 1) / tb;
