@@ -855,6 +855,17 @@ __device__ __forceinline__ void load_stage(const Params &p, const LayerP &L, con
     }
 }
 
+// 256-bit global accesses (sm_100): one full 32-B sector per lane
+__device__ __forceinline__ void ld_cg_v8(const uint4 *p, uint32_t (&r)[8]) {
+    asm volatile("ld.global.cg.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+                 : "l"(p));
+}
+__device__ __forceinline__ void st_v8(uint4 *p, const uint32_t (&w)[8]) {
+    asm volatile("st.global.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(w[0]), "r"(w[1]), "r"(w[2]),
+                 "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7])
+                 : "memory");
+}
 __device__ __forceinline__ uint32_t pack2(float a, float b) {
     __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
     return *reinterpret_cast<uint32_t *>(&v);
@@ -1361,34 +1372,37 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                     T.dst_scr ? scr + ((((long long)(d - T.dlo[0]) * L.pR[1] + (y - T.dlo[1])) * L.pR[2] + (x - T.dlo[2])) *
                                            L.cout + ch0)
                               : outp + pix_pow2(L.out, L.lB, T.n, d, y, x) + ch0);
+                // 16 channels (32 B: one full sector) per 256-bit store (kind 1: zeros)
 #pragma unroll
-                for (int k = 0; k < 4; k++) {
-                    if (k >= CB / 8) break;
-                    float v[8];
+                for (int k2 = 0; k2 < 2; k2++) {
+                    if (k2 >= CB / 16) break;
+                    uint32_t w8[8];
 #pragma unroll
-                    for (int e = 0; e < 8; e++)
-                        v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]) + __shfl_sync(0xffffffffu, bl, k * 8 + e);
-                    if (kind != 2) {
-                        if (kind == 1) dst[k] = make_uint4(0, 0, 0, 0);
-                        continue;
-                    }
-                    if (has_rs) {
-                        const uint4 rr = rnext;
-                        if (k + 1 < CB / 8) rnext = __ldcg(rsp + k + 1);
-                        const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr);
+                    for (int h = 0; h < 2; h++) {   // 16-B chunk k = 2 k2 + h: channels 8k .. 8k + 7
+                        const int k = 2 * k2 + h;
+                        float v[8];
 #pragma unroll
-                        for (int e = 0; e < 4; e++) {
-                            const float2 f = __bfloat1622float2(h2[e]);
-                            v[2 * e] += f.x;
-                            v[2 * e + 1] += f.y;
+                        for (int e = 0; e < 8; e++)
+                            v[e] = __uint_as_float(r[k2][h * 8 + e]) + __shfl_sync(0xffffffffu, bl, k * 8 + e);
+                        if (has_rs) {
+                            const uint4 rr = rnext;
+                            if (k + 1 < CB / 8) rnext = __ldcg(rsp + k + 1);
+                            const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr);
+#pragma unroll
+                            for (int e = 0; e < 4; e++) {
+                                const float2 f = __bfloat1622float2(h2[e]);
+                                v[2 * e] += f.x;
+                                v[2 * e + 1] += f.y;
+                            }
                         }
-                    }
-                    if (L.relu) {
+                        if (L.relu) {
 #pragma unroll
-                        for (int e = 0; e < 8; e++) v[e] = fmaxf(v[e], 0.f);
+                            for (int e = 0; e < 8; e++) v[e] = fmaxf(v[e], 0.f);
+                        }
+#pragma unroll
+                        for (int e = 0; e < 4; e++) w8[h * 4 + e] = kind == 2 ? pack2(v[2 * e], v[2 * e + 1]) : 0u;
                     }
-                    if (!DBG(p, 4))
-                        dst[k] = make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
+                    if (kind && !DBG(p, 4)) st_v8(dst + 2 * k2, w8);
                 }
             }
             PT(if (p.prof) { wit += clock64() - ti0; ntask++; })
