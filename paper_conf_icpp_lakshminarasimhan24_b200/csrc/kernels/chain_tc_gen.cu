@@ -1355,8 +1355,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 const float bl = DBG(p, 8) ? 0.f : __ldg(L.bias + ch0 + (lane & (CB - 1)));
                 const bool has_rs = L.has_res && kind == 2 && !DBG(p, 16);
                 const uint4 *rsp = has_rs ? reinterpret_cast<const uint4 *>(resp + pix_pow2(L.res, L.lB, T.n, d, y, x) + ch0) : nullptr;
-                uint4 rnext = make_uint4(0, 0, 0, 0);
-                if (has_rs) rnext = __ldcg(rsp);
+                uint32_t rnext[8] = {0, 0, 0, 0, 0, 0, 0, 0};   // residual: 16 channels per 256-bit load, one pair ahead
+                if (has_rs) ld_cg_v8(rsp, rnext);
                 uint32_t r[2][16];
                 const uint32_t taddr = tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) +
                                        tl * (Tdv * L.Nc) + (Tdv - 1 - o) * L.Nc + cb * CB;
@@ -1377,6 +1377,8 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 for (int k2 = 0; k2 < 2; k2++) {
                     if (k2 >= CB / 16) break;
                     uint32_t w8[8];
+                    if (has_rs && k2 > 0) ld_cg_v8(rsp + 2 * k2, rnext);   // (pair 0: issued before the TMEM load)
+                    const uint32_t *rr = rnext;
 #pragma unroll
                     for (int h = 0; h < 2; h++) {   // 16-B chunk k = 2 k2 + h: channels 8k .. 8k + 7
                         const int k = 2 * k2 + h;
@@ -1385,9 +1387,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                         for (int e = 0; e < 8; e++)
                             v[e] = __uint_as_float(r[k2][h * 8 + e]) + __shfl_sync(0xffffffffu, bl, k * 8 + e);
                         if (has_rs) {
-                            const uint4 rr = rnext;
-                            if (k + 1 < CB / 8) rnext = __ldcg(rsp + k + 1);
-                            const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr);
+                            const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr[h * 4]);
 #pragma unroll
                             for (int e = 0; e < 4; e++) {
                                 const float2 f = __bfloat1622float2(h2[e]);
