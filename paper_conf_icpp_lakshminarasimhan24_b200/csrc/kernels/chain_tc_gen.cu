@@ -2038,7 +2038,10 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
     // images per group: the group's first layer holds `group_waves` waves of tasks (enough ready work at every
     // dependency level; measured on B200, cfg4: 2 waves 13.3 ms, 4 waves 11.6 ms, 8 waves 11.2 ms)
     const double gw = p->opts.group_waves > 0 ? p->opts.group_waves : 8.0;
-    static const double lw = [] { const char *e = getenv("BDL_GEN_LAGWAVES"); return e ? atof(e) : 2.0; }();
+    // lag of a consumer layer behind its producers, in waves of its tasks (BDL_GEN_LAGWAVES: A/B knob); measured on
+    // B200 (r02e build): 1 / 2 / 3 / 4 / 6 waves: VGG-16 7.72 / 6.18 / 6.06 / 6.01 / 6.00 ms, ResNet-50 7.67 / 7.59 /
+    // 7.59 / 7.58 / 7.56 ms, 3-D 1.37 / 1.25 / 1.25 / 1.25 / 1.25 ms
+    static const double lw = [] { const char *e = getenv("BDL_GEN_LAGWAVES"); return e ? atof(e) : 4.0; }();
     int G = (int)std::max<long long>(1, (long long)std::ceil(gw * p->num_sms / std::max<long long>(1, per_img0)));
     G = std::min(G, N);
     std::vector<double> key(total, 0.0);
