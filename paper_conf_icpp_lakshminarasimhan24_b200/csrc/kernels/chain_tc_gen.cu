@@ -41,7 +41,11 @@ namespace bdl {
 
 namespace gen {
 
-constexpr int kSched = 0, kLoad0 = 1, kLW = 4, kWProd = 5, kMma = 6, kEpi0 = 7, kEpiW = 16;
+#ifndef BDL_GEN_EPIW
+#define BDL_GEN_EPIW 12
+#endif
+constexpr int kSched = 0, kLoad0 = 1, kLW = 4, kWProd = 5, kMma = 6, kEpi0 = 7, kEpiW = BDL_GEN_EPIW;
+constexpr int kEpiR = kEpiW / 4;   // epilogue warps per TMEM lane quadrant
 constexpr int kThreads = 32 * (kEpi0 + kEpiW);
 constexpr int kLoadT = 32 * kLW;
 constexpr int kQ = 4, kRing = 16, kStack = 128;
@@ -212,7 +216,7 @@ __device__ __forceinline__ long long pix(const TView &v, int n, int d, int y, in
 // Fused pool: channel batches staged together in the epilogue -- a power of two (the staging tile's XOR swizzle
 // masks with the chunk count), <= 4 / M tiles so the 4 warp ranks share ntl x gcb items
 __host__ __device__ __forceinline__ int pool_gcb(int ncb, int ntl) {
-    int g = ncb < 4 / ntl ? ncb : 4 / ntl;
+    int g = ncb < kEpiR / ntl ? ncb : kEpiR / ntl;
     if (g < 1) g = 1;
     while (g & (g - 1)) g &= g - 1;
     return g;
@@ -1233,7 +1237,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         unsigned long long wed = 0, wea = 0, web = 0, wtm = 0, wit = 0, wpub = 0, ntask = 0, ncomp = 0;
         const unsigned long long t_start = clock64();
         const int quad = warp % 4;        // TMEM lane quadrant this warp may access
-        const int rank = ew / 4;          // 4 warps per quadrant split the (tile, column batch) items
+        const int rank = ew / 4;          // kEpiR warps per quadrant split the (tile, column batch) items
         const uint32_t tmem_base = sh.tmem_base;
         for (uint32_t seq = 0;; seq++) {
             pwait(p, &sh.desc_full[seq % kRing], (seq / kRing) & 1, wed);
@@ -1267,7 +1271,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 const int nchk = gcb * nck;   // 16-B chunks per staged position (a power of two)
                 for (int cb0 = 0; cb0 < ncb; cb0 += gcb) {
                     const int ng = min(gcb, ncb - cb0);
-                    for (int it = rank; it < L.ntl * ng; it += 4) {
+                    for (int it = rank; it < L.ntl * ng; it += kEpiR) {
                         const int tl = it / ng, cbl = it - tl * ng;
                         const int ch0 = T.nc * L.Nc + (cb0 + cbl) * CB;
                         const int m = tl * 128 + quad * 32 + lane;
@@ -1336,7 +1340,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 }
             }
             PT(const unsigned long long ti0 = p.prof ? clock64() : 0;)
-            for (int it = rank; it < (L.pool ? 0 : items); it += 4) {
+            for (int it = rank; it < (L.pool ? 0 : items); it += kEpiR) {
                 const int o = STK ? it / (L.ntl * ncb) : 0, itr = it - o * (L.ntl * ncb);   // output plane of the task
                 const int tl = itr / ncb, cb = itr - tl * ncb;
                 const int m = tl * 128 + quad * 32 + lane;
