@@ -41,12 +41,9 @@ namespace bdl {
 
 namespace gen {
 
-#ifndef BDL_GEN_EPIW
-#define BDL_GEN_EPIW 12
-#endif
-constexpr int kSched = 0, kLoad0 = 1, kLW = 4, kWProd = 5, kMma = 6, kEpi0 = 7, kEpiW = BDL_GEN_EPIW;
-constexpr int kEpiR = kEpiW / 4;   // epilogue warps per TMEM lane quadrant
-constexpr int kThreads = 32 * (kEpi0 + kEpiW);
+// Warp roles; the epilogue has EPIW warps (a template parameter: 8 or 12, EPIW / 4 per TMEM lane quadrant).  Fewer
+// warps leave more registers per thread (19 warps: 96, 15 warps: 128; 23 warps were capped at 80 and spilled).
+constexpr int kSched = 0, kLoad0 = 1, kLW = 4, kWProd = 5, kMma = 6, kEpi0 = 7;
 constexpr int kLoadT = 32 * kLW;
 constexpr int kQ = 4, kRing = 16, kStack = 128;
 constexpr int kPendDraw = 32, kPend = kPendDraw + kStack;   // pending (deferred) tasks: draw tickets below kPendDraw
@@ -215,8 +212,8 @@ __device__ __forceinline__ long long pix(const TView &v, int n, int d, int y, in
 // First conv-output row / column of tile (ty, tx) (pooled layers: under its first pool window; may be < 0).
 // Fused pool: channel batches staged together in the epilogue -- a power of two (the staging tile's XOR swizzle
 // masks with the chunk count), <= 4 / M tiles so the 4 warp ranks share ntl x gcb items
-__host__ __device__ __forceinline__ int pool_gcb(int ncb, int ntl) {
-    int g = ncb < kEpiR / ntl ? ncb : kEpiR / ntl;
+__host__ __device__ __forceinline__ int pool_gcb(int ncb, int ntl, int er) {
+    int g = ncb < er / ntl ? ncb : er / ntl;
     if (g < 1) g = 1;
     while (g & (g - 1)) g &= g - 1;
     return g;
@@ -905,8 +902,8 @@ __device__ __forceinline__ void issue_ksteps(const uint32_t *ksl, int q0, int q1
 
 // STK: the subgraph has depth-stacked layers.  Two instantiations, so the stacked issue path is absent from the kernel
 // that 2-D subgraphs run (present, it cost 2-D layers ~15 % through the MMA warp's register allocation; B200 A/B).
-template <bool STK>
-__global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant__ Params p) {
+template <bool STK, int EPIW>
+__global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __grid_constant__ Params p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     __shared__ Shared sh;
     const int warp = __shfl_sync(0xffffffff, (int)threadIdx.x / 32, 0), lane = threadIdx.x % 32;
@@ -915,7 +912,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
     if (ptx::smem_u32(smem) & 1023) __trap();   // 128-B swizzle atoms need 1024-B alignment
 
     // k-step descriptor-offset tables
-    for (int i = threadIdx.x; i < p.L * kMaxKs; i += kThreads) {
+    for (int i = threadIdx.x; i < p.L * kMaxKs; i += (32 * (kEpi0 + EPIW))) {
         const int l = i / kMaxKs, q = i % kMaxKs;
         const LayerP &L = p.layer[l];
         if (q >= (L.stk ? L.nks / L.k[0] : L.nks)) continue;
@@ -960,7 +957,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         }
         for (int i = 0; i < 2; i++) {
             ptx::mbar_init(&sh.acc_full[i], 1);
-            ptx::mbar_init(&sh.acc_empty[i], kEpiW);
+            ptx::mbar_init(&sh.acc_empty[i], EPIW);
         }
         for (int i = 0; i < kRing; i++) ptx::mbar_init(&sh.desc_full[i], 1);
         sh.done_seq = 0;
@@ -1237,7 +1234,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
         unsigned long long wed = 0, wea = 0, web = 0, wtm = 0, wit = 0, wpub = 0, ntask = 0, ncomp = 0;
         const unsigned long long t_start = clock64();
         const int quad = warp % 4;        // TMEM lane quadrant this warp may access
-        const int rank = ew / 4;          // kEpiR warps per quadrant split the (tile, column batch) items
+        const int rank = ew / 4;          // (EPIW / 4) warps per quadrant split the (tile, column batch) items
         const uint32_t tmem_base = sh.tmem_base;
         for (uint32_t seq = 0;; seq++) {
             pwait(p, &sh.desc_full[seq % kRing], (seq / kRing) & 1, wed);
@@ -1267,11 +1264,11 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                 const int nck = CB / 8;
                 // channel batches staged together: the 4 warp ranks share ntl x gcb (tile, batch) items, so every
                 // epilogue warp reads TMEM even when a task has a single M tile; staging <= ntl*128 x 128 ch
-                const int gcb = pool_gcb(ncb, L.ntl);
+                const int gcb = pool_gcb(ncb, L.ntl, EPIW / 4);
                 const int nchk = gcb * nck;   // 16-B chunks per staged position (a power of two)
                 for (int cb0 = 0; cb0 < ncb; cb0 += gcb) {
                     const int ng = min(gcb, ncb - cb0);
-                    for (int it = rank; it < L.ntl * ng; it += kEpiR) {
+                    for (int it = rank; it < L.ntl * ng; it += (EPIW / 4)) {
                         const int tl = it / ng, cbl = it - tl * ng;
                         const int ch0 = T.nc * L.Nc + (cb0 + cbl) * CB;
                         const int m = tl * 128 + quad * 32 + lane;
@@ -1299,11 +1296,11 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                                 make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
                         }
                     }
-                    asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");
+                    asm volatile("bar.sync 2, %0;" ::"n"(32 * EPIW) : "memory");
                     const int nc_g = ng * nck;                // (a power of two unless the last, partial group)
                     const int lnc = 31 - __clz(nc_g);
                     const int nout = L.Tpb * L.Tpw * nc_g;
-                    for (int q = ew * 32 + lane; q < nout; q += 32 * kEpiW) {
+                    for (int q = ew * 32 + lane; q < nout; q += 32 * EPIW) {
                         const int ck = (nc_g & (nc_g - 1)) ? q % nc_g : q & (nc_g - 1);
                         const int o = (nc_g & (nc_g - 1)) ? q / nc_g : q >> lnc;
                         const int oy = o / L.Tpw, ox = o - oy * L.Tpw;
@@ -1336,11 +1333,11 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
                         }
                         *dst = *reinterpret_cast<const uint4 *>(mx);
                     }
-                    asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");   // staging reused by the next group
+                    asm volatile("bar.sync 2, %0;" ::"n"(32 * EPIW) : "memory");   // staging reused by the next group
                 }
             }
             PT(const unsigned long long ti0 = p.prof ? clock64() : 0;)
-            for (int it = rank; it < (L.pool ? 0 : items); it += kEpiR) {
+            for (int it = rank; it < (L.pool ? 0 : items); it += (EPIW / 4)) {
                 const int o = STK ? it / (L.ntl * ncb) : 0, itr = it - o * (L.ntl * ncb);   // output plane of the task
                 const int tl = itr / ncb, cb = itr - tl * ncb;
                 const int m = tl * 128 + quad * 32 + lane;
@@ -1415,7 +1412,7 @@ __global__ void __launch_bounds__(kThreads, 1) gen_kernel(const __grid_constant_
             if (lane == 0) mbar_arrive(&sh.acc_empty[a]);
             // every epilogue warp's stores of this tile precede the publication
             const unsigned long long tb0 = p.prof ? clock64() : 0;
-            asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiW) : "memory");
+            asm volatile("bar.sync 2, %0;" ::"n"(32 * EPIW) : "memory");
             if (p.prof) web += clock64() - tb0;
             if (ew == 0 && lane == 0) {
                 PT(const unsigned long long tp0 = p.prof ? clock64() : 0;)
@@ -1597,9 +1594,9 @@ static bool gen_layer_static(const Layer &ly, int nsp, const bdl_layout &lo_out,
 }
 
 // Fused pool: epilogue staging tile, every M row of the conv tile x the channel batches staged together, bf16.
-static int gen_pool_stage_bytes(const gen::LayerP &G) {
+static int gen_pool_stage_bytes(const gen::LayerP &G, int er) {
     const int CB = G.Nc >= 32 ? 32 : 16, ncb = G.Nc / CB;
-    const int gcb = gen::pool_gcb(ncb, G.ntl);   // channel batches staged together (epilogue)
+    const int gcb = gen::pool_gcb(ncb, G.ntl, er);   // channel batches staged together (epilogue)
     return G.ntl * 128 * gcb * CB * 2;
 }
 
@@ -1652,7 +1649,7 @@ static bool gen_layer_tiles(gen::LayerP &G, int cover_h, int cover_w, int walign
                                : (G.amode == gen::AM_PLANES ? G.kc * rows * 16 : rows * 16);
             cand.stage_bytes = (cand.stage_bytes + 1023) / 1024 * 1024;
             if (cand.stage_bytes * 2 > in_budget) continue;   // two input stages at least
-            if (G.pool && gen_pool_stage_bytes(cand) > kGenPoolStageMax) continue;
+            if (G.pool && gen_pool_stage_bytes(cand, 3) > kGenPoolStageMax) continue;   // (fused pools: 12 warps)
             const int nty = (cover_h + Ub - 1) / Ub, ntx = (cover_w + Uw - 1) / Uw;
             // time model per plane: tasks x (MMAs per task + a fixed per-task cost), times a penalty for loaded
             // halo pixels.  The fixed cost (claim, dependency acquire, barriers, epilogue hand-off, publication)
@@ -1749,7 +1746,7 @@ static unsigned long long *gen_prof_buffer(cudaStream_t s) {
 struct GenGeom {
     gen::LayerP layer[kMaxLayers];
     int L;
-    int nin, in_stride, nw, w_stride, acc_stride, nacc, tmem_cols, smem, pool_bytes;
+    int nin, in_stride, nw, w_stride, acc_stride, nacc, tmem_cols, smem, pool_bytes, epiw;
     int PB[3], npb[3];
     long long scr_slot;
 };
@@ -1813,6 +1810,15 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
         f += F;
     }
     const bool shallow = f > 0 && kf / f < kGenShallowK;
+    // epilogue warps: 12 where the epilogue carries more per output (residual adds, depth-stacked planes), else 8 (the
+    // 128 registers per thread of a 15-warp CTA).  Measured on B200 per subgraph, same box, 12 vs 8 warps: VGG-16
+    // stages 1.61 / 1.55, 0.85 / 0.81, 1.21 / 1.20 ms, ResNet-50 stem 0.56 / 0.53 ms; ResNet-50 bottleneck subgraphs
+    // 1.43 / 1.49, 1.62 / 1.72, 1.16 / 1.21, 0.64 / 0.69 ms; 3-D chain 1.16 / 1.25 ms.
+    static const int epiw_env = [] { const char *e = getenv("BDL_GEN_EPIW"); return e ? atoi(e) : 0; }();
+    bool any_res = false;
+    for (int j = 0; j < nconv; j++)
+        any_res = any_res || (j < (int)sg.res_tensor.size() && sg.res_tensor[j] >= 0) || g.layer[j].resl >= 0;
+    g.epiw = epiw_env == 8 || epiw_env == 12 ? epiw_env : (any_res || any_stk) ? 12 : 8;
     const bool nw2 = !stk_geo && !fused && (gen_nw2() < 0 ? shallow : gen_nw2() == 1);
     const int nwp = (!stk_geo && !fused && gen_nw_force() >= 1 && gen_nw_force() <= gen::kMaxW) ? gen_nw_force()
                     : nw2 ? kGenW - 1 : kGenW;   // weight stages of a plain subgraph
@@ -1912,7 +1918,7 @@ static bool gen_geometry(const bdl_plan *p, const Subgraph &sg, int nconv, bool 
         in_stride = std::max(in_stride, G.stage_bytes);
         w_stride = std::max(w_stride, G.kpw * 2 * (G.stk ? 3 : 1) * G.Nc * 16);
         acc = std::max(acc, G.ntl * G.Td * G.Nc);
-        if (G.pool) g.pool_bytes = (gen_pool_stage_bytes(G) + 1023) / 1024 * 1024;
+        if (G.pool) g.pool_bytes = (gen_pool_stage_bytes(G, g.epiw / 4) + 1023) / 1024 * 1024;
     }
     g.in_stride = in_stride;
     g.w_stride = (w_stride + 1023) / 1024 * 1024;
@@ -2209,7 +2215,9 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
     P.counters = (unsigned long long *)(wsp + sg.counter_off);
     bool any_stk = false;
     for (int j = 0; j < L; j++) any_stk = any_stk || P.layer[j].stk;
-    auto kern = any_stk ? gen::gen_kernel<true> : gen::gen_kernel<false>;
+    auto kern = any_stk ? (g.epiw == 8 ? gen::gen_kernel<true, 8> : gen::gen_kernel<true, 12>)
+                        : (g.epiw == 8 ? gen::gen_kernel<false, 8> : gen::gen_kernel<false, 12>);
+    const int nthreads = 32 * (gen::kEpi0 + g.epiw);
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
     const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;
     if (padded) {
@@ -2223,14 +2231,14 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
         P.scr_slot = g.scr_slot;
         P.norder = (long long)p->layers[sg.first].in_ext[0] * g.npb[0] * g.npb[1] * g.npb[2];
         const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-        launch_pdl(kern, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+        launch_pdl(kern, dim3(grid), dim3(nthreads), g.smem, s, P);
         *launches += 1;
     } else if (!unmerged) {
         P.only_layer = -1;
         P.order = (const int *)(wsp + sg.order_off);
         P.norder = sg.norder;
         const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-        launch_pdl(kern, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+        launch_pdl(kern, dim3(grid), dim3(nthreads), g.smem, s, P);
         *launches += 1;
     } else {
         P.order = nullptr;
@@ -2238,7 +2246,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
             P.only_layer = j;
             P.norder = P.layer[j].ntasks;
             const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-            launch_pdl(kern, dim3(grid), dim3(gen::kThreads), g.smem, s, P);
+            launch_pdl(kern, dim3(grid), dim3(nthreads), g.smem, s, P);
             *launches += 1;
         }
     }
