@@ -1377,9 +1377,10 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
 #pragma unroll
                 for (int k2 = 0; k2 < 2; k2++) {
                     if (k2 >= CB / 16) break;
-                    uint32_t w8[8];
-                    if (has_rs && k2 > 0) ld_cg_v8(rsp + 2 * k2, rnext);   // (pair 0: issued before the TMEM load)
-                    const uint32_t *rr = rnext;
+                    uint32_t w8[8], rr[8];
+#pragma unroll
+                    for (int e = 0; e < 8; e++) rr[e] = rnext[e];
+                    if (has_rs && k2 + 1 < CB / 16) ld_cg_v8(rsp + 2 * (k2 + 1), rnext);   // next pair in flight
 #pragma unroll
                     for (int h = 0; h < 2; h++) {   // 16-B chunk k = 2 k2 + h: channels 8k .. 8k + 7
                         const int k = 2 * k2 + h;
