@@ -2051,8 +2051,10 @@ std::vector<int> gen_task_order(const bdl_plan *p, const Subgraph &sg) {
     const double gw = p->opts.group_waves > 0 ? p->opts.group_waves : 8.0;
     // lag of a consumer layer behind its producers, in waves of its tasks (BDL_GEN_LAGWAVES: A/B knob); measured on
     // B200 (r02e build): 1 / 2 / 3 / 4 / 6 waves: VGG-16 7.72 / 6.18 / 6.06 / 6.01 / 6.00 ms, ResNet-50 7.67 / 7.59 /
-    // 7.59 / 7.58 / 7.56 ms, 3-D 1.37 / 1.25 / 1.25 / 1.25 / 1.25 ms
-    static const double lw = [] { const char *e = getenv("BDL_GEN_LAGWAVES"); return e ? atof(e) : 4.0; }();
+    // 7.59 / 7.58 / 7.56 ms, 3-D 1.37 / 1.25 / 1.25 / 1.25 / 1.25 ms.  3-D volumes keep 2: their longer lag's footprint
+    // outgrows L2 (ncu, 128^3 x 32: gen_kernel DRAM reads 197 MB at 2 waves, 433 MB at 4, same time)
+    static const double lw_env = [] { const char *e = getenv("BDL_GEN_LAGWAVES"); return e ? atof(e) : 0.0; }();
+    const double lw = lw_env > 0 ? lw_env : p->in_layout.nsp == 3 ? 2.0 : 4.0;
     int G = (int)std::max<long long>(1, (long long)std::ceil(gw * p->num_sms / std::max<long long>(1, per_img0)));
     G = std::min(G, N);
     std::vector<double> key(total, 0.0);
