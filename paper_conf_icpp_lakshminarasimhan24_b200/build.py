@@ -25,6 +25,7 @@ SOURCES = [
     "kernels/chain_brick.cu",
     "kernels/chain_tc.cu",
     "kernels/chain_tc_ws.cu",
+    "kernels/chain_tc_pair.cu",
     "kernels/chain_tc_gen.cu",
 ]
 FLAGS = [

@@ -611,7 +611,7 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
                     if (k < (unsigned long long)p.trace_cap) {
                         unsigned smid;
                         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-                        unsigned long long *rec = p.trace + k * 12;
+                        unsigned long long *rec = p.trace + k * 16;
                         rec[0] = ((unsigned long long)smid << 40) | ((unsigned long long)blockIdx.x << 8) | (unsigned)l;
                         rec[1] = (unsigned long long)t;
                         for (int f = 0; f < 7; f++) rec[2 + f] = sh.tr[sq % kRing][f];
@@ -823,6 +823,28 @@ __global__ void __launch_bounds__(Roles<C>::THREADS, 1) memo_ws_kernel(const __g
 static unsigned long long *ws_trace_buf = nullptr;
 static int ws_trace_cap = 0;
 
+// Debug task trace (BDL_TRACE=<records>): 16 x u64 per task (12 used by the single-CTA kernel), read back by bdl_debug_ws_trace (tools/trace_ws.py).
+unsigned long long *ws_trace_setup(unsigned char *wsp, const Subgraph &sg, cudaStream_t s, int *cap_out) {
+    *cap_out = 0;
+    const char *e = getenv("BDL_TRACE");
+    if (!e) return nullptr;
+    static unsigned long long *tbuf = nullptr;
+    static int tcap = 0;
+    const int cap = atoi(e);
+    if (cap <= 0) return nullptr;
+    if (!tbuf || cap > tcap) {
+        if (tbuf) cudaFree(tbuf);
+        cudaMalloc(&tbuf, (size_t)cap * 16 * 8);
+        tcap = cap;
+    }
+    cudaMemsetAsync(tbuf, 0, (size_t)cap * 16 * 8, s);
+    cudaMemsetAsync(wsp + sg.counter_off + 7 * 8, 0, 8, s);   // trace index
+    ws_trace_buf = tbuf;
+    ws_trace_cap = cap;
+    *cap_out = cap;
+    return tbuf;
+}
+
 struct WsGeom {
     int Tb, Tw, Wt, rowsA, nin, nacc, ntl, tmem_cols, smem;
 };
@@ -905,6 +927,24 @@ std::vector<int> ws_order(const bdl_plan *p, const Subgraph &sg, const WsGeom &g
     return ord;
 }
 
+// Pair kernel order: like ws_order, but per step all images of one layer are consecutive and every (step, layer)
+// run is padded to an even length with -1 entries, so the two entries of a pair ticket share a layer.
+std::vector<int> ws_pair_order(const bdl_plan *p, const Subgraph &sg, const WsGeom &g, int lag) {
+    const Layer &f = p->layers[sg.first];
+    const int L = sg.last - sg.first + 1;
+    const int N = f.in_ext[0], H = f.in_ext[2];
+    const int nty = (H + g.Tb - 1) / g.Tb;
+    std::vector<int> ord;
+    for (int s = 0; s < nty + lag * (L - 1); s++)
+        for (int l = 0; l < L; l++) {
+            const int b = s - lag * l;
+            if (b < 0 || b >= nty) continue;
+            for (int n = 0; n < N; n++) ord.push_back((l << 24) | (n * nty + b));
+            if (ord.size() % 2) ord.push_back(-1);
+        }
+    return ord;
+}
+
 template <int C>
 static bdl_status launch_ws_C(bdl_plan *p, Subgraph &sg, ws::Params &P, const WsGeom &g, bool unmerged, cudaStream_t s,
                               int *launches) {
@@ -955,7 +995,11 @@ static bool encode_pixel_map(CUtensorMap *tm, const TView &v, int box_px) {
 
 // 5-D view of a 2-D bricked bf16 tensor (identity BrickMap): (channel, x in brick, brick column,
 // y in brick, brick row over (n, by)); box = 64 channels x Bw x nseg bricks x 1 x 1 = one tile row.
-static bool encode_row_map(CUtensorMap *tm, const TView &v, int nseg) {
+static bool encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int rows = 1);
+// Like encode_row_map with a box of `rows` pixel rows of one brick row; nseg may exceed the bricks per row (the
+// boxes' extra bricks read outside the map: zero fill).
+bool encode_rows_map_bf16(CUtensorMap *tm, const TView &v, int nseg, int rows) { return encode_row_map(tm, v, nseg, rows); }
+static bool encode_row_map(CUtensorMap *tm, const TView &v, int nseg, int rows) {
     static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
     if (!enc) {
         cudaDriverEntryPointQueryResult qr;
@@ -967,15 +1011,37 @@ static bool encode_row_map(CUtensorMap *tm, const TView &v, int nseg) {
     cuuint64_t dims[5] = {(cuuint64_t)v.Cp, (cuuint64_t)v.B[3], (cuuint64_t)v.nb[3], (cuuint64_t)v.B[2],
                           (cuuint64_t)v.nb[0] * v.nb[1] * v.nb[2]};
     cuuint64_t strides[4] = {px, brick, px * v.B[3], brick * v.nb[3]};
-    cuuint32_t box[5] = {64, (cuuint32_t)v.B[3], (cuuint32_t)nseg, 1, 1};
+    cuuint32_t box[5] = {64, (cuuint32_t)v.B[3], (cuuint32_t)nseg, (cuuint32_t)rows, 1};
     cuuint32_t es[5] = {1, 1, 1, 1, 1};
     CUresult r = enc(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, v.ptr, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                      CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
 
+bool encode_row_map_bf16(CUtensorMap *tm, const TView &v, int nseg) { return encode_row_map(tm, v, nseg); }
+
+bool pair_geometry(int L, int H, int W, int Bw, int N, int num_sms, int &Tb, int &ntl, int &in_bytes, int &smem, int &nin);
+bdl_status launch_pair_subgraph(const bdl_plan *p, const Subgraph &sg, const TView &in, const TView &out, const TView *res,
+                                unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged, void *dense);
+
+// The CTA-pair kernel (chain_tc_pair.cu) runs C = 64 chains over full-width bands when their weights fit resident;
+// returns its band height, or 0.  BDL_NO_PAIR=1 keeps the single-CTA kernel (A/B runs).
+int pair_band_rows(const bdl_plan *p, const Subgraph &sg) {
+    static const bool off = getenv("BDL_NO_PAIR") && atoi(getenv("BDL_NO_PAIR"));
+    const Layer &f = p->layers[sg.first];
+    if (off || f.L.cin != 64 || p->in_layout.nsp != 2 || p->in_layout.brickmap || p->in_layout.Bh > 8) return 0;
+    if (ilog2(p->in_layout.Bh) < 0 || ilog2(p->in_layout.Bw) < 0) return 0;
+    int Tb, ntl, ib, sm, nin;
+    if (!pair_geometry(sg.last - sg.first + 1, f.in_ext[2], f.in_ext[3], p->in_layout.Bw, f.in_ext[0], p->num_sms, Tb, ntl,
+                       ib, sm, nin))
+        return 0;
+    return Tb;
+}
+
 bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const TView &out, const TView *res,
                               unsigned char *wsp, cudaStream_t s, int *launches, bool unmerged, void *dense) {
+    if (pair_band_rows(p, sg) > 0 && !in.bmap && !out.bmap && !(res && res->bmap))
+        return launch_pair_subgraph(p, sg, in, out, res, wsp, s, launches, unmerged, dense);
     WsGeom g;
     if (!ws_geometry(p, sg, g)) return fail(BDL_EUNSUPPORTED, "tcgen05 ws kernel: tile does not fit on chip");
     ws::Params P;
@@ -1043,24 +1109,7 @@ bdl_status launch_ws_subgraph(bdl_plan *p, Subgraph &sg, const TView &in, const 
 #ifdef BDL_DEBUG   // timing knobs that deliberately skip work (wrong results): debug builds only
     if (const char *e = getenv("BDL_WS_DBG")) P.dbg = atoi(e);
 #endif
-    if (const char *e = getenv("BDL_TRACE")) {
-        static unsigned long long *tbuf = nullptr;
-        static int tcap = 0;
-        int cap = atoi(e);
-        if (cap > 0) {
-            if (!tbuf || cap > tcap) {
-                if (tbuf) cudaFree(tbuf);
-                cudaMalloc(&tbuf, (size_t)cap * 12 * 8);
-                tcap = cap;
-            }
-            cudaMemsetAsync(tbuf, 0, (size_t)cap * 12 * 8, s);
-            cudaMemsetAsync(wsp + sg.counter_off + 7 * 8, 0, 8, s);   // trace index
-            P.trace = tbuf;
-            P.trace_cap = cap;
-            ws_trace_buf = tbuf;
-            ws_trace_cap = cap;
-        }
-    }
+    P.trace = ws_trace_setup(wsp, sg, s, &P.trace_cap);
     switch (P.C) {
         case 16: return launch_ws_C<16>(p, sg, P, g, unmerged, s, launches);
         case 32: return launch_ws_C<32>(p, sg, P, g, unmerged, s, launches);
@@ -1076,6 +1125,11 @@ namespace bdl {
 std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg) {
     WsGeom g;
     if (!ws_geometry(p, sg, g)) return {};
+    const bool pair = pair_band_rows(p, sg) > 0;
+    if (pair) {
+        g.Tb = pair_band_rows(p, sg);
+        g.Tw = p->layers[sg.first].in_ext[3];
+    }
     // lag: how many band rows layer l trails layer l-1.  Larger = fewer dependency waits but a larger
     // live intermediate; take the largest lag whose live intermediate (lag band rows of every image of
     // the shard, per merged layer) fits in a quarter of L2, at least 3.
@@ -1086,7 +1140,7 @@ std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg) {
     int lag = (int)std::min<double>(nty, (double)p->l2_bytes / 4.0 / std::max(1, L - 1) / band_bytes);
     lag = std::max(3, lag);
     if (const char *e = getenv("BDL_LAG")) lag = std::max(1, atoi(e));
-    std::vector<int> ord = ws_order(p, sg, g, lag);
+    std::vector<int> ord = pair ? ws_pair_order(p, sg, g, lag) : ws_order(p, sg, g, lag);
     if (p->opts.schedule_seed) {  // any order is valid: the scheduler claims missing dependencies first
         std::mt19937 rng((unsigned)p->opts.schedule_seed);
         std::shuffle(ord.begin(), ord.end(), rng);
@@ -1100,13 +1154,15 @@ extern "C" int bdl_debug_ws_trace(unsigned long long *host, int max_records) {
     if (!bdl::ws_trace_buf) return 0;
     int n = max_records < bdl::ws_trace_cap ? max_records : bdl::ws_trace_cap;
     cudaDeviceSynchronize();
-    cudaMemcpy(host, bdl::ws_trace_buf, (size_t)n * 12 * 8, cudaMemcpyDeviceToHost);
+    cudaMemcpy(host, bdl::ws_trace_buf, (size_t)n * 16 * 8, cudaMemcpyDeviceToHost);
     return n;
 }
 
 namespace bdl {
 // Band height of the warp-specialized kernel for subgraph sg (0 if it cannot run it).
+int pair_band_rows(const bdl_plan *p, const Subgraph &sg);
 int ws_band_rows(const bdl_plan *p, const Subgraph &sg) {
+    if (int tb = pair_band_rows(p, sg)) return tb;
     WsGeom g;
     return ws_geometry(p, sg, g) ? g.Tb : 0;
 }
