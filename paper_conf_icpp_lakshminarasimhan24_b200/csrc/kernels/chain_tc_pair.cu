@@ -167,7 +167,7 @@ __device__ __forceinline__ int ld_relaxed(const int *p) {
     return v;
 }
 
-__device__ void scheduler(const Params &p, Shared &sh) {
+__device__ void scheduler(const Params &p, Shared &sh, int e_first) {
     const int lane = threadIdx.x % 32;
     const unsigned EP = run_epoch(p.counters) << 2;
     const bool unmerged = p.only_layer >= 0;
@@ -262,11 +262,12 @@ __device__ void scheduler(const Params &p, Shared &sh) {
     // entries are claimed (lanes 0-1, CAS) and their dependencies' tags read speculatively (lanes 2-7), ticket k+1's
     // order entries are fetched (lanes 8-9) and ticket k+2 is drawn (lane 0).
     auto entry = [&](long long tk, int w) -> int { return 2 * tk + w < p.norder ? p.order[2 * tk + w] : -1; };
-    unsigned long long tkA = 0, tkB = 0;
-    if (lane == 0) tkA = atomicAdd(&p.counters[4], 1ULL);
-    tkA = __shfl_sync(0xffffffff, tkA, 0);
-    int e = lane < 2 ? entry((long long)tkA, lane) : -1;
-    if (lane == 0) tkB = atomicAdd(&p.counters[4], 1ULL);
+    // the first ticket of cluster c is c (its order entries were fetched before the PDL wait); the shared counter hands
+    // out the rest
+    const unsigned ncl = gridDim.x / 2;
+    unsigned long long tkA = blockIdx.x / 2, tkB = 0;
+    int e = lane < 2 ? e_first : -1;
+    if (lane == 0) tkB = atomicAdd(&p.counters[4], 1ULL) + ncl;
     for (;;) {
         if (2 * (long long)tkA >= p.norder) break;
         if (p.trace) ts_tk = gtime();
@@ -290,7 +291,7 @@ __device__ void scheduler(const Params &p, Shared &sh) {
         int en = -1;
         if (lane >= 8 && lane < 10) en = entry((long long)tkBv, lane - 8);
         unsigned long long tkC = 0;
-        if (lane == 0 && 2 * (long long)tkBv < p.norder) tkC = atomicAdd(&p.counters[4], 1ULL);
+        if (lane == 0 && 2 * (long long)tkBv < p.norder) tkC = atomicAdd(&p.counters[4], 1ULL) + ncl;
         // (2) resolve the claims
         int claimed = 0;
         if (lane < 2 && lr >= 0) {
@@ -342,7 +343,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
     uint8_t *wsm = smem + p.nin * p.in_bytes;                           // resident weights [L][kWLayer]
     float *bias_s = reinterpret_cast<float *>(wsm + p.L * kWLayer);   // [L][C]
     if (ptx::smem_u32(smem) & 1023) __trap();   // 128-B swizzle atoms need 1024-B alignment
-    for (int i = threadIdx.x; i < p.L * C; i += kThreads) bias_s[i] = p.layer[i / C].bias[i % C];
     // the kG guard pixels before row 0 of each band buffer are zero for every task (the left zero pad of the band's first
     // row; every other row's left pad is the previous row's out-of-image brick, zero-filled by TMA)
     for (int i = threadIdx.x; i < p.nin * kG * 8; i += kThreads)
@@ -380,21 +380,30 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
         for (int i = lane; i < p.L * 8; i += 32)
             asm volatile("prefetch.tensormap [%0];" ::"l"(&p.tm_row[i / 8][i % 8]) : "memory");
     }
-    if (warp == kLoadWarp) {
-        // resident weights: this CTA's 32 output channels of every layer (bulk copies of 512 B)
-        if (lane == 0) ptx::mbar_arrive_expect_tx(&sh.wbar, p.L * kWLayer);
-        __syncwarp();
-        for (int i = lane; i < p.L * 72; i += 32) {
+    if (warp >= kEpi0 && warp < kPubWarp) {
+        // resident weights: this CTA's 32 output channels of every layer (bulk copies of 512 B, spread over the idle
+        // epilogue warps so that the loader starts on its first band at once) and the fp32 biases
+        const int et = threadIdx.x - 32 * kEpi0;
+        if (et == 0) ptx::mbar_arrive_expect_tx(&sh.wbar, p.L * (kWLayer + C * 4));
+        asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiWarps) : "memory");
+        for (int i = et; i < p.L * 72; i += 32 * kEpiWarps) {
             const int j = i / 72, r = i % 72;   // r = tap * 8 + k-chunk
             ptx::bulk_g2s(wsm + j * kWLayer + r * 512, p.layer[j].w + ((size_t)r * C + rank * 32) * 8, 512, &sh.wbar);
         }
+        if (et < p.L) ptx::bulk_g2s(bias_s + et * C, p.layer[et].bias, C * 4, &sh.wbar);
     }
+    // the scheduler's first ticket is static (cluster index): fetch its order entries now (written at prepare time)
+    int e_first = -1;
+    if (warp == 0 && leader && p.only_layer < 0 && lane < 2 && (long long)blockIdx.x + lane < p.norder)
+        e_first = p.order[blockIdx.x + lane];   // = order[2 * (blockIdx.x / 2) + lane] (blockIdx.x is even)
+    const unsigned long long t_init = p.trace ? gtime() : 0;
     // PDL: everything below may touch the previous kernel's output (subgraph input) or the memo tags
     pdl_wait();
+    const unsigned long long t_pdl = p.trace ? gtime() : 0;
 
     const unsigned EP = run_epoch(p.counters) << 2;
     if (warp == 0) {
-        if (leader) scheduler(p, sh);
+        if (leader) scheduler(p, sh, e_first);
     } else if (warp == kLoadWarp) {
         // ------------------------------------------------------------------ loader
         const bool unmerged = p.only_layer >= 0;
@@ -430,7 +439,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
             }
             const unsigned long long t_dep = p.trace ? gtime() : 0;
             // the acquired data (generic-proxy stores of other CTAs) is read by TMA (async proxy)
-            if (work && !(p.knob & 4)) asm volatile("fence.proxy.async.global;" ::: "memory");
+            // (layer 0 reads the subgraph input, written by an earlier grid: no proxy fence needed)
+            if (work && l > 0 && !(p.knob & 4)) asm volatile("fence.proxy.async.global;" ::: "memory");
             if (seq >= (uint32_t)p.nin) ptx::mbar_wait(&sh.in_empty[b], ((seq / p.nin) - 1) & 1);
             if (lane == 0) {
                 sh.desc_l[seq % kRing] = l;
@@ -542,6 +552,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
         // ------------------------------------------------------------------ epilogue
         const int ew = warp - kEpi0, g = ew / 4, quad = warp % 4;
         const uint32_t tmem = __shfl_sync(0xffffffff, sh.tmem_base, 0);
+        ptx::mbar_wait(&sh.wbar, 0);   // biases landed (with the weights)
         const int Hg = p.layer[0].out.nb[2] << p.lBh;
         const int mBh = (1 << p.lBh) - 1, mBw = (1 << p.lBw) - 1;
         uint32_t ph = 0;   // phase bit per (accumulator, tile)
@@ -696,6 +707,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
             rec[1] = 0;
             for (int f = 2; f < 11; f++) rec[f] = 0;
             rec[2] = t_entry;
+            rec[3] = t_init;
+            rec[4] = t_pdl;
             rec[11] = gtime();
         }
     }
@@ -730,11 +743,11 @@ bool pair_geometry(int L, int H, int W, int Bw, int N, int num_sms, int &Tb, int
         for (int ni = pr::kMaxNin; ni >= 2; ni--) {
             const int sm = ni * ib + L * (int)pr::kWLayer + L * pr::C * 4;
             if (sm > limit) continue;
-            // time model: pair-task waves x (tiles + per-task overhead of ~0.3 tile); with two band buffers the next
-            // band's load has only one task's MMAs to hide behind (measured on B200: ~30 % bubbles at cfg2)
+            // time model: pair-task waves x (tiles + per-task overhead of ~0.3 tile); the most band buffers that fit
+            // (measured on B200 at cfg2: Tb = 6 with 2 buffers 47 us, Tb = 4 with 3 buffers 51 us)
             const long long tasks = (long long)N * ((H + tb - 1) / tb) * L;
             const long long pairs = (tasks + 1) / 2;
-            const double cost = (double)((pairs + ncl - 1) / ncl) * (nt + 0.3) * (ni >= 3 ? 1.0 : 1.3);
+            const double cost = (double)((pairs + ncl - 1) / ncl) * (nt + 0.3);
             if (cost < best - 1e-9) {
                 best = cost;
                 Tb = tb;

@@ -32,6 +32,8 @@ if len(ctarec):
     print("CTA entry (us rel. first task q): min %.2f max %.2f; CTA exit: min %.2f max %.2f" % (
         (ctarec[:, 2].min() - t0) / 1e3, (ctarec[:, 2].max() - t0) / 1e3, (ctarec[:, 11].min() - t0) / 1e3,
         (ctarec[:, 11].max() - t0) / 1e3))
+    print("CTA init done (rel. entry) mean %.2f, PDL wait done mean %.2f us" % (
+        ((ctarec[:, 3] - ctarec[:, 2]) / 1e3).mean(), ((ctarec[:, 4] - ctarec[:, 2]) / 1e3).mean()))
 names = ["q", "dep", "loaded", "mma0", "mma1", "epi0", "epi1", "sync", "read", "end", "emit", "tk", "claimed", "scanned"]
 rec = []
 for r in a:
