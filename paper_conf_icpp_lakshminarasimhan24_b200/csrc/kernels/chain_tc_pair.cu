@@ -86,6 +86,7 @@ struct Shared {
     uint64_t acc_full[2][kMaxTl];
     uint64_t acc_empty[2];       // leader: 2 x kEpiWarps arrivals
     uint64_t wbar, wpeer;        // own resident weights landed; (leader) the peer's landed
+    uint64_t pf_bar;             // first-band prefetch landed
     uint64_t desc_full[kRing];
     uint64_t epi_done[kRing];    // the CTA's epilogue warps have stored the slot's task (kEpiWarps arrivals)
     uint32_t tmem_base;
@@ -364,6 +365,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
         }
         ptx::mbar_init(&sh.wbar, 1);
         ptx::mbar_init(&sh.wpeer, 1);
+        ptx::mbar_init(&sh.pf_bar, 1);
         for (int i = 0; i < kRing; i++) {
             ptx::mbar_init(&sh.desc_full[i], 1);
             ptx::mbar_init(&sh.epi_done[i], kEpiWarps);
@@ -393,9 +395,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
         if (et < p.L) ptx::bulk_g2s(bias_s + et * C, p.layer[et].bias, C * 4, &sh.wbar);
     }
     // the scheduler's first ticket is static (cluster index): fetch its order entries now (written at prepare time)
-    int e_first = -1;
+    int e_first = -1, e_own = -1;
     if (warp == 0 && leader && p.only_layer < 0 && lane < 2 && (long long)blockIdx.x + lane < p.norder)
         e_first = p.order[blockIdx.x + lane];   // = order[2 * (blockIdx.x / 2) + lane] (blockIdx.x is even)
+    if (warp == kLoadWarp && p.only_layer < 0 && (long long)blockIdx.x < p.norder) e_own = p.order[blockIdx.x];
     const unsigned long long t_init = p.trace ? gtime() : 0;
     // PDL: everything below may touch the previous kernel's output (subgraph input) or the memo tags
     pdl_wait();
@@ -408,6 +411,45 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
         // ------------------------------------------------------------------ loader
         const bool unmerged = p.only_layer >= 0;
         const int R = p.Tb + 2;
+        // Stage the band of task t of layer l: rows y0-1 .. y0+Tb; rows outside the image are zeros (generic proxy,
+        // fenced for the tensor core); in-image rows arrive as one TMA box per run of rows inside one brick row
+        // (Wt = W + Bw pixels per row: the box's last brick is outside the map and zero-filled, it is the row's right
+        // and the next row's left zero pad).
+        auto issue_band = [&](int l, int t, uint8_t *buf, uint64_t *bar) {
+            const int ty = t % p.nty, img = t / p.nty;
+            const int y0 = ty * p.Tb;
+            const TView &src = l == 0 ? p.in : p.layer[l - 1].out;
+            const int ya = max(y0 - 1, 0), yb = min(y0 + p.Tb, p.H - 1);   // in-image rows
+            bool zeros = false;
+            for (int a = 0; a < R; a++) {
+                const int y = y0 - 1 + a;
+                if (y >= 0 && y < p.H) continue;
+                zeros = true;
+                uint4 *d = reinterpret_cast<uint4 *>(buf + (size_t)(kG + a * p.Wt) * 128);
+                for (int q = lane; q < p.Wt * 8; q += 32) d[q] = make_uint4(0, 0, 0, 0);
+            }
+            // (a shared-memory proxy fence costs ~1 us while the tensor core streams operands: only after zero rows)
+            if (zeros) ptx::fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0 && (p.knob & 16)) arrive_local(bar);   // timing experiment: no band loads
+            else if (lane == 0) {
+                ptx::mbar_arrive_expect_tx(bar, (uint32_t)(yb - ya + 1) * p.Wt * 128);
+                const int Bh = 1 << p.lBh;
+                for (int y = ya; y <= yb;) {
+                    const int k = min(yb + 1, (y & ~(Bh - 1)) + Bh) - y;   // rows of this brick row
+                    ptx::tma_load_5d(buf + (size_t)(kG + (y - y0 + 1) * p.Wt) * 128, &p.tm_row[l][k - 1], 0, 0, 0,
+                                     y & (Bh - 1), img * src.nb[2] + (y >> p.lBh), bar);
+                    y += k;
+                }
+            }
+        };
+        // First-band prefetch: the first ticket of cluster c is static (c), so this CTA's first task is order entry
+        // blockIdx.x; if it is a layer-0 task (no dependencies) its band is loaded now, while the scheduler claims it.
+        int pf_task = -1;
+        if (!unmerged && e_own >= 0 && (e_own >> 24) == 0) {
+            pf_task = e_own & 0xFFFFFF;
+            issue_band(0, pf_task, smem, &sh.pf_bar);
+        }
         for (uint32_t seq = 0;; seq++) {
             const int slot = seq % kQ;
             ptx::mbar_wait_cl(&sh.q_full[slot], (seq / kQ) & 1);
@@ -457,38 +499,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
                 }
                 arrive_local(&sh.desc_full[seq % kRing]);
             }
-            if (work) {
-                const int ty = t % p.nty, img = t / p.nty;
-                const int y0 = ty * p.Tb;
-                const TView &src = l == 0 ? p.in : p.layer[l - 1].out;
-                // band rows y0-1 .. y0+Tb: rows outside the image are zeros (generic proxy, fenced for the tensor core);
-                // in-image rows arrive as one TMA box per run of rows inside one brick row (Wt = W + Bw pixels per row:
-                // the box's last brick is outside the map and zero-filled, it is the row's right and the next row's
-                // left zero pad)
-                const int ya = max(y0 - 1, 0), yb = min(y0 + p.Tb, p.H - 1);   // in-image rows
-                bool zeros = false;
-                for (int a = 0; a < R; a++) {
-                    const int y = y0 - 1 + a;
-                    if (y >= 0 && y < p.H) continue;
-                    zeros = true;
-                    uint4 *d = reinterpret_cast<uint4 *>(buf + (size_t)(kG + a * p.Wt) * 128);
-                    for (int q = lane; q < p.Wt * 8; q += 32) d[q] = make_uint4(0, 0, 0, 0);
+            if (work && seq == 0 && pf_task >= 0) {
+                // the first band was prefetched (static first ticket): reuse it if the queue confirms the task
+                ptx::mbar_wait(&sh.pf_bar, 0);
+                if (l == 0 && t == pf_task) {
+                    __syncwarp();
+                    if (lane == 0) arrive_local(bar);
+                } else {
+                    issue_band(l, t, buf, bar);
                 }
-                // (a shared-memory proxy fence costs ~1 us while the tensor core streams operands: only after zero rows)
-                if (zeros) ptx::fence_proxy_async_smem();
-                __syncwarp();
-                if (lane == 0 && (p.knob & 16)) arrive_local(bar);   // timing experiment: no band loads
-                else if (lane == 0) {
-                    ptx::mbar_arrive_expect_tx(bar, (uint32_t)(yb - ya + 1) * p.Wt * 128);
-                    if (p.trace) sh.tr[seq % kRing][7] = gtime();
-                    const int Bh = 1 << p.lBh;
-                    for (int y = ya; y <= yb;) {
-                        const int k = min(yb + 1, (y & ~(Bh - 1)) + Bh) - y;   // rows of this brick row
-                        ptx::tma_load_5d(buf + (size_t)(kG + (y - y0 + 1) * p.Wt) * 128, &p.tm_row[l][k - 1], 0, 0, 0,
-                                         y & (Bh - 1), img * src.nb[2] + (y >> p.lBh), bar);
-                        y += k;
-                    }
-                }
+                if (p.trace && lane == 0) sh.tr[seq % kRing][2] = gtime();
+            } else if (work) {
+                issue_band(l, t, buf, bar);
                 if (p.trace && lane == 0) sh.tr[seq % kRing][2] = gtime();
             } else {
                 __syncwarp();
