@@ -4,12 +4,10 @@
 //   brickify:   TMA load of the NCHW box (64 px, 64 ch, R rows) through a 5-D view that splits the
 //               channel c = 8g + k so the box lands as smem [xb][row][k][g][128 B] (128-B swizzled);
 //               a thread owns 8 channels (group g) x 8 pixels: for each k the 8 lanes of a group read 8
-//               consecutive swizzled rows (conflict-free), transpose 8x8 in registers, and write the 8
-//               pixel chunks g of 8 pixel rows (the 8 lanes fill one 128-B row: conflict-free) of
-//               smem [row][px][128 B]; one TMA store per brick row through the 5-D row map.
+//               consecutive swizzled rows (conflict-free), transpose 8x8 in registers, and store the 8
+//               pixel chunks g straight to the bricked tensor (the 8 lanes of a group fill one pixel's 128 B).
 //   unbrickify: the reverse (TMA row load of bricks, transpose, TMA store of NCHW boxes).
-// No L1 traffic on either global side: both move through the TMA engine; shared-memory accesses are
-// 16-byte and conflict-free.
+// Dense-side traffic moves through the TMA engine; shared-memory accesses are 16-byte and conflict-free.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -30,6 +28,9 @@ struct TmaConvParams {
     int nbx, nbh;         // bricks along w, h
     int nxb;              // 64-pixel boxes along w
     int ncb;              // 64-channel blocks
+    void *out;            // brickify: the bricked tensor (direct stores)
+    int Cp;               // padded channels
+    long long brick_elems;
 };
 
 // 128-B swizzle: 16-B chunk j of the 128-B row at shared address `row` lives at chunk j ^ (row bits 7..9)
@@ -50,7 +51,9 @@ __device__ __forceinline__ void transpose8(const uint4 (&in)[8], uint4 (&out)[8]
     }
 }
 
-// smem: A = dense tile [nxb][R][64 ch][128 B], B = brick tile [R][nbx*Bw px][128 B]
+// smem: A = dense tile [nxb][R][64 ch][128 B].  The transposed 8-channel pixel chunks go straight to the bricked
+// tensor: the 8 lanes of a group write the 8 chunks of one pixel (one 128-B line), so the stores are coalesced and no
+// staging tile is needed -- 16 KB of shared memory per CTA (R = 2) lets the whole grid run in one wave.
 __global__ void __launch_bounds__(128) brickify_tma_kernel(const __grid_constant__ TmaConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     __shared__ uint64_t bar;
@@ -61,7 +64,6 @@ __global__ void __launch_bounds__(128) brickify_tma_kernel(const __grid_constant
     const int y0 = rb * p.R;
     const int Wg = p.nbx * p.Bw;
     uint8_t *A = smem;
-    uint8_t *B = smem + (size_t)p.nxb * p.R * 64 * 128;
     if (threadIdx.x == 0) {
         ptx::mbar_init(&bar, 1);
         ptx::fence_barrier_init();
@@ -77,10 +79,13 @@ __global__ void __launch_bounds__(128) brickify_tma_kernel(const __grid_constant
     // each item: one row, 8 channels (group g), 8 pixels (group q) -> 8 pixel chunks
     const int nq = Wg / 8;
     const int items = p.R * 8 * nq;
+    uint8_t *out_base = reinterpret_cast<uint8_t *>(p.out);
     for (int it = threadIdx.x; it < items; it += blockDim.x) {
         const int g = it % 8;
         const int q = (it / 8) % nq;
         const int r = it / 8 / nq;
+        const int y = y0 + r;
+        if (y >= p.nbh * p.Bh) break;
         const int xb = q / 8, j = q % 8;
         uint4 in[8], out[8];
 #pragma unroll
@@ -89,22 +94,15 @@ __global__ void __launch_bounds__(128) brickify_tma_kernel(const __grid_constant
             in[k] = *reinterpret_cast<const uint4 *>(swz(row, j));
         }
         transpose8(in, out);
+        // pixels x = 8q .. 8q+7 lie in one brick (Bw is a multiple of 8 or 8 a multiple of Bw: per-pixel brick index)
 #pragma unroll
         for (int i = 0; i < 8; i++) {
-            uint8_t *row = B + ((size_t)r * Wg + q * 8 + i) * 128;
-            *reinterpret_cast<uint4 *>(swz(row, g)) = out[i];
+            const int x = q * 8 + i;
+            const long long brick = ((long long)n * p.nbh + (y >> p.lBh)) * p.nbx + (x >> p.lBw);
+            const long long off = brick * p.brick_elems +
+                                  (long long)(((y & (p.Bh - 1)) << p.lBw) + (x & (p.Bw - 1))) * p.Cp + cb * 64 + g * 8;
+            *reinterpret_cast<uint4 *>(out_base + off * 2) = out[i];
         }
-    }
-    ptx::fence_proxy_async_smem();
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int r = 0; r < p.R; r++) {
-            const int y = y0 + r;
-            if (y >= p.nbh * p.Bh) break;
-            ptx::tma_store_5d(&p.bricks, B + (size_t)r * Wg * 128, cb * 64, 0, 0, y & (p.Bh - 1), n * p.nbh + (y >> p.lBh));
-        }
-        ptx::bulk_commit();
-        ptx::bulk_wait_read0();   // shared memory must stay valid until the store has read it
     }
 }
 
@@ -228,9 +226,13 @@ bool launch_convert_tma(const bdl_layout *l, const void *dense, void *bricked, c
     const size_t smem = (size_t)P.nxb * P.R * 64 * 128 + (size_t)P.R * Wg * 128;
     if (smem > 200 * 1024) return false;
     if (to_bricks) {
+        P.out = bricked;
+        P.Cp = (int)l->c_pad;
+        P.brick_elems = l->brick_elems;
+        const size_t smem_b = (size_t)P.nxb * P.R * 64 * 128;   // no staging tile: direct stores
         const long long grid = (long long)N * (nbh * l->Bh / P.R) * P.ncb;
-        cudaFuncSetAttribute(brickify_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        brickify_tma_kernel<<<(unsigned)grid, 128, smem, s>>>(P);
+        cudaFuncSetAttribute(brickify_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_b);
+        brickify_tma_kernel<<<(unsigned)grid, 128, smem_b, s>>>(P);
     } else {
         const long long grid = (long long)N * ((H + P.R - 1) / P.R) * P.ncb;
         cudaFuncSetAttribute(unbrickify_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
