@@ -224,6 +224,11 @@ void bdl_plan_destroy(bdl_plan *p);
 bdl_status bdl_plan_subgraph_model(const bdl_plan *p, int32_t i, double *delta_first, int64_t *rho,
                                    int32_t *mode_model, int32_t *tc_band);
 
+/* 1 if subgraph i's memoized / unmerged execution runs on the CTA-pair tcgen05 kernel (C = 64 3x3 chains over
+ * full-width bands: two CTAs of a cluster share one M = 256 MMA, each holding half of the output channels' weights;
+ * DESIGN.md §6), 0 otherwise (or on a bad index).  Host only. */
+int32_t bdl_plan_subgraph_cta_pair(const bdl_plan *p, int32_t i);
+
 /* Region analysis (Fig 4): input-region extent of each layer of layers[first..last] for
  * one interior output brick of edge b along spatial dim `dim` (1 = d, 2 = h, 3 = w), by reverse
  * traversal I = s*(O-1) + k.  layers: HOST; ext_out: HOST [last-first+1]. */

@@ -73,6 +73,7 @@ _SIGS = {
     "bdl_last_error": (ctypes.c_char_p, []),
     "bdl_version": (ctypes.c_char_p, []),
     "bdl_plan_subgraph_model": (_i32, [_vp, _i32, _P(_f64), _P(_i64), _P(_i32), _P(_i32)]),
+    "bdl_plan_subgraph_cta_pair": (_i32, [_vp, _i32]),
     "bdl_region_extents": (_i32, [_P(bdl_layer), _i32, _i32, _i32, _i32, _P(_i64)]),
     "bdl_model_brick": (_i32, [_P(bdl_plan_opts), _i32, _i64, _i64, _i64, _i64, _P(_i64)]),
 }

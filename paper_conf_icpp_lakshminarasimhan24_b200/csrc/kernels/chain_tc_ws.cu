@@ -1027,7 +1027,8 @@ bdl_status launch_pair_subgraph(const bdl_plan *p, const Subgraph &sg, const TVi
 // The CTA-pair kernel (chain_tc_pair.cu) runs C = 64 chains over full-width bands when their weights fit resident;
 // returns its band height, or 0.  BDL_NO_PAIR=1 keeps the single-CTA kernel (A/B runs).
 int pair_band_rows(const bdl_plan *p, const Subgraph &sg) {
-    static const bool off = getenv("BDL_NO_PAIR") && atoi(getenv("BDL_NO_PAIR"));
+    const char *np = getenv("BDL_NO_PAIR");
+    const bool off = np && atoi(np);
     const Layer &f = p->layers[sg.first];
     if (off || f.L.cin != 64 || p->in_layout.nsp != 2 || p->in_layout.brickmap || p->in_layout.Bh > 8) return 0;
     if (ilog2(p->in_layout.Bh) < 0 || ilog2(p->in_layout.Bw) < 0) return 0;
@@ -1148,6 +1149,12 @@ std::vector<int> ws_task_order(const bdl_plan *p, const Subgraph &sg) {
     return ord;
 }
 }  // namespace bdl
+
+extern "C" int32_t bdl_plan_subgraph_cta_pair(const bdl_plan *p, int32_t i) {
+    if (!p || i < 0 || i >= (int)p->sgs.size()) return 0;
+    const bdl::Subgraph &sg = p->sgs[i];
+    return bdl::effective_kernel(sg) == bdl::KERNEL_TC_BAND && bdl::pair_band_rows(p, sg) > 0 ? 1 : 0;
+}
 
 // Debug: copy the warp-specialized kernel's task trace (8 x u64 per task) to host.
 extern "C" int bdl_debug_ws_trace(unsigned long long *host, int max_records) {

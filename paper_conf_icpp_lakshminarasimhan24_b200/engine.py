@@ -122,7 +122,8 @@ class Plan:
             out.append(dict(first=f.value, last=la.value, mode=MODE_NAMES.get(m.value, m.value),
                             mode_id=m.value, model_brick=b.value, delta=d.value, delta_first=df.value,
                             rho=rho.value, mode_model=MODE_NAMES.get(mm.value, mm.value),
-                            kernel=KERNEL_NAMES[k.value], tc_band=tb.value))
+                            kernel=KERNEL_NAMES[k.value], tc_band=tb.value,
+                            cta_pair=bool(lib().bdl_plan_subgraph_cta_pair(self.h, i))))
         return out
 
     def set_mode(self, mode, i=None):
