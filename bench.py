@@ -454,6 +454,8 @@ def main():
         peak_src = f"{peak_src} bf16_tflops (burst, cuBLAS 8192^3)"
     achieved = flops / (kernel_ms / 1e3) / 1e12
     kname = sg[0]["kernel"] if len(sg) == 1 else f"{len(sg)} subgraph launches ({', '.join(sorted(kinds))})"
+    if len(sg) == 1 and sg[0].get("cta_pair") and sg[0]["mode"] != "padded":
+        kname += ", CTA pair (cta_group::2, memo_pair_kernel)"
     roofline = {"bound": bound, "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                 "traffic": traffic if len(sg) == 1 and kinds == {"tcgen05 band"} else None,
                 "traffic_source": traffic_src if len(sg) == 1 and kinds == {"tcgen05 band"} else None,
@@ -499,7 +501,8 @@ def main():
             "data": "synthetic (seeded N(0,1) inputs, He-normal weights; workloads.py)",
             "config": {"workload": workload_desc(wl), "images_per_gpu": wl["N"], "global_batch": wl["N"] * world,
                        "mode": sg[0]["mode"], "mode_model": sg[0]["mode_model"], "delta": round(sg[0]["delta"], 4),
-                       "kernel": sg[0]["kernel"], "subgraphs": len(sg), "step": "brickify + merged subgraph with unbrickify fused into its last epilogue (bdl_run_dense)",
+                       "kernel": sg[0]["kernel"] + (", CTA pair (cta_group::2)" if sg[0].get("cta_pair") else ""),
+                       "subgraphs": len(sg), "step": "brickify + merged subgraph with unbrickify fused into its last epilogue (bdl_run_dense)",
                        "l2": "flushed between timed steps (256 MiB write + 256 MiB read, outside the events)",
                        "timing": "value/ms_per_step: K steps with events only around each step; breakdown_ms and "
                                  "roofline: a second K-step pass with events between the kernels",

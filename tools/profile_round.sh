@@ -9,8 +9,8 @@ timeout 900 python bench.py > gpurun_out/${R}_bench.json 2> gpurun_out/${R}_benc
 timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --csv \
     --log-file gpurun_out/${R}_launches.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-cudnn --no-extra > /dev/null 2>&1
 echo launches=$?
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:memo_ws -s 3 -c 1 \
-    -o gpurun_out/${R}_memo_ws python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn --no-extra > /dev/null 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:memo_pair -s 3 -c 1 \
+    -o gpurun_out/${R}_memo_pair python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn --no-extra > /dev/null 2>&1
 echo memo=$?
 timeout 600 ncu --set full --clock-control none -k regex:brickify -s 2 -c 2 \
     -o gpurun_out/${R}_brickify python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-cudnn --no-extra > /dev/null 2>&1
@@ -36,4 +36,10 @@ for tool in memcheck synccheck racecheck; do
   eval timeout 1200 compute-sanitizer --tool $tool --print-limit 20 --target-processes all \
       python -m pytest $CASES -q -p no:cacheprovider > gpurun_out/${R}_sanitize_gen_$tool.log 2>&1
   echo "sanitize $tool rc=$?"; grep -E "ERROR SUMMARY|passed|failed|RACECHECK SUMMARY" gpurun_out/${R}_sanitize_gen_$tool.log | tail -3
+done
+# the CTA-pair band kernel (cfg2 path): memcheck / synccheck / racecheck on its GPU tests
+for tool in memcheck synccheck racecheck; do
+  timeout 1200 compute-sanitizer --tool $tool --print-limit 20 --target-processes all \
+      python -m pytest tests/test_gpu_pair.py -q -p no:cacheprovider -k "shape1 or shape2" > gpurun_out/${R}_sanitize_pair_$tool.log 2>&1
+  echo "sanitize pair $tool rc=$?"; grep -E "ERROR SUMMARY|passed|failed|RACECHECK SUMMARY" gpurun_out/${R}_sanitize_pair_$tool.log | tail -3
 done

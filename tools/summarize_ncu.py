@@ -10,7 +10,7 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "l1tex__throughput.avg.pct_of_peak_sustained_elapsed", "launch__registers_per_thread", "launch__grid_size",
         "launch__block_size", "launch__shared_mem_per_block_dynamic", "sm__cycles_elapsed.avg.per_second"]
 summary = {"round": R, "kernels": {}}
-for tag in ["memo_ws", "brickify", "padded", "gen_cfg5", "gen_cfg4"]:
+for tag in ["memo_pair", "memo_ws", "brickify", "padded", "gen_cfg5", "gen_cfg4"]:
     rep = os.path.join(OUT, f"{R}_{tag}.ncu-rep")
     if not os.path.exists(rep):
         continue
@@ -43,9 +43,8 @@ if os.path.exists(lc):
         key = k.split("(")[0]
         tot.setdefault(key, []).append(v)
     summary["launch_list"] = {k: {"count": len(v), "mean_ns": sum(v) / len(v)} for k, v in tot.items()}
-    step = [v for k, v in launches if "brickify" in k or "memo_ws" in k]
     ours = {k: sum(v) for k, v in tot.items()
-            if any(t in k for t in ("bdl::", "memo_ws", "gen_kernel", "brickify", "pool_vec")) and "pack" not in k}
+            if any(t in k for t in ("bdl::", "memo_ws", "memo_pair", "gen_kernel", "brickify", "pool_vec")) and "pack" not in k}
     s = sum(ours.values())
     summary["launch_share_of_step"] = {k: v / s for k, v in ours.items()}
     with open(f"profiles/{R}_launches.csv", "w") as f:
@@ -55,7 +54,7 @@ if os.path.exists(lc):
 # dram bytes per launch of the dominant kernel (for bench.py's roofline.traffic)
 dram = None
 for name, lst in summary["kernels"].items():
-    if "memo_ws" in name:
+    if "memo_pair" in name or ("memo_ws" in name and dram is None):
         d = lst[0]
         rb = float(d["dram__bytes_read.sum"]["value"]) * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[d["dram__bytes_read.sum"]["unit"]]
         wb = float(d["dram__bytes_write.sum"]["value"]) * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[d["dram__bytes_write.sum"]["unit"]]
