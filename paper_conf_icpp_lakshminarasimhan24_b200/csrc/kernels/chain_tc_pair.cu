@@ -63,6 +63,7 @@ struct Params {
     __nv_bfloat16 *dense;        // non-null: the LAST layer writes dense NCHW here (unbrickify fused, bdl_run_dense)
     int L, H, W, Tb, Wt, nty, lBh, lBw, ntl;
     int nin;                     // input band buffers (2 or 3)
+    int qd;                      // scheduler queue depth (<= kQ): how far claims may run ahead of the loader
     uint32_t in_bytes;           // one input buffer (1024-B multiple)
     Layer layer[kMaxL];
     TView in, res;
@@ -176,8 +177,8 @@ __device__ void scheduler(const Params &p, Shared &sh, int e_first) {
     uint32_t qseq = 0;
     unsigned long long ts_tk = 0, ts_cl = 0, ts_dp = 0;   // debug trace
     auto emit = [&](int l, int t0, int t1) {
-        const int slot = qseq % kQ;
-        if (qseq >= (uint32_t)kQ) ptx::mbar_wait_cl(&sh.q_empty[slot], ((qseq / kQ) - 1) & 1);
+        const int slot = qseq % p.qd;
+        if (qseq >= (uint32_t)p.qd) ptx::mbar_wait_cl(&sh.q_empty[slot], ((qseq / p.qd) - 1) & 1);
         if (lane == 0) {
             const int n = l < 0 ? 0 : max(tiles_of(p, t0), tiles_of(p, t1));
             sh.q_l[slot] = l;
@@ -451,8 +452,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
             issue_band(0, pf_task, smem, &sh.pf_bar);
         }
         for (uint32_t seq = 0;; seq++) {
-            const int slot = seq % kQ;
-            ptx::mbar_wait_cl(&sh.q_full[slot], (seq / kQ) & 1);
+            const int slot = seq % p.qd;
+            ptx::mbar_wait_cl(&sh.q_full[slot], (seq / p.qd) & 1);
             const int l = sh.q_l[slot], t = sh.q_t[slot], n = sh.q_n[slot];
             __syncwarp();
             if (lane == 0) arrive_leader(&sh.q_empty[slot]);
@@ -810,6 +811,8 @@ bdl_status launch_pair_subgraph(const bdl_plan *p, const Subgraph &sg, const TVi
     P.ntl = ntl;
     P.in_bytes = (uint32_t)in_bytes;
     P.nin = nin;
+    P.qd = pr::kQ;
+    if (const char *e = getenv("BDL_PAIR_QD")) P.qd = std::max(1, std::min(pr::kQ, atoi(e)));
     P.in = in;
     if (res) P.res = *res;
     for (int j = 0; j < L; j++) {
