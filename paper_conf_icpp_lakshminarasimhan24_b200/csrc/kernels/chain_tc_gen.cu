@@ -91,6 +91,8 @@ struct LayerP {
     long long task_base, ntasks;
     int pR[3];                // padded: largest region of this layer's output (scratch pitches)
     long long scr_off;        // padded: byte offset of the layer's region buffer in a scratch slot
+    int l2hint;               // epilogue stores' L2 policy: 1 evict_last (a later layer of the subgraph reads this
+                              // output: keep it resident), 2 evict_first (leaves the subgraph: stream it), 0 none
 };
 
 struct Params {
@@ -867,6 +869,13 @@ __device__ __forceinline__ void st_v8(uint4 *p, const uint32_t (&w)[8]) {
                  "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7])
                  : "memory");
 }
+// the same with an L2 eviction-priority policy (createpolicy): locality-aware memoization keeps the memo buffers
+// that later layers of the subgraph read resident and streams the subgraph's outputs
+__device__ __forceinline__ void st_v8_pol(uint4 *p, const uint32_t (&w)[8], uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8}, %9;" ::"l"(p), "r"(w[0]), "r"(w[1]),
+                 "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7]), "l"(pol)
+                 : "memory");
+}
 __device__ __forceinline__ uint32_t pack2(float a, float b) {
     __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
     return *reinterpret_cast<uint32_t *>(&v);
@@ -1252,6 +1261,9 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
             const int items = L.ntl * ncb * Tdv;
             const __nv_bfloat16 *resp = reinterpret_cast<const __nv_bfloat16 *>(L.res.ptr);
             __nv_bfloat16 *outp = reinterpret_cast<__nv_bfloat16 *>(L.out.ptr);
+            uint64_t pol_keep, pol_stream;
+            asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
+            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_stream));
             const int d = T.d;
             __nv_bfloat16 *scr = T.dst_scr ? reinterpret_cast<__nv_bfloat16 *>(scr_slot(p, T.slot) + L.scr_off) : nullptr;
             if (L.pool) {
@@ -1404,7 +1416,10 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
 #pragma unroll
                         for (int e = 0; e < 4; e++) w8[h * 4 + e] = kind == 2 ? pack2(v[2 * e], v[2 * e + 1]) : 0u;
                     }
-                    if (kind && !DBG(p, 4)) st_v8(dst + 2 * k2, w8);
+                    if (kind && !DBG(p, 4)) {
+                        if (L.l2hint) st_v8_pol(dst + 2 * k2, w8, L.l2hint == 1 ? pol_keep : pol_stream);
+                        else st_v8(dst + 2 * k2, w8);
+                    }
                 }
             }
             PT(if (p.prof) { wit += clock64() - ti0; ntask++; })
@@ -2158,6 +2173,14 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
         }
         G.src = G.srcl >= 0 ? outs[G.srcl] : srcv[j];
         G.out = outs[j];
+        {   // L2 policy of the epilogue stores (locality-aware memoization; BDL_GEN_L2HINT=0 turns it off)
+            static const int hint = [] { const char *e = getenv("BDL_GEN_L2HINT"); return e ? atoi(e) : 1; }();
+            bool read_inside = false;
+            for (int q = j + 1; q < L; q++)
+                read_inside = read_inside || (q < (int)sg.src_local.size() ? sg.src_local[q] : q - 1) == j ||
+                              (q < (int)sg.res_local.size() && sg.res_local[q] == j);
+            G.l2hint = !hint || padded ? 0 : read_inside ? 1 : 2;
+        }
         G.tma = 0;
         G.pxo = 0;
         // pooled tiles start at tx * Tpw * ps - pad: TMA rows need that brick-aligned and non-negative
