@@ -49,6 +49,8 @@ def lib():
             L.oracle_round_bf16.argtypes = [ctypes.c_double]
             L.oracle_conv.restype = None
             L.oracle_conv.argtypes = [_dp, _i, _i, _i, _i, _i, _dp, _dp, _i] + [_i] * 12 + [_dp, _i, _i, _i]
+            L.oracle_conv_transpose.restype = None
+            L.oracle_conv_transpose.argtypes = [_dp, _i, _i, _i, _i, _i, _dp, _dp, _i] + [_i] * 12 + [_dp, _i, _i, _i]
             L.oracle_maxpool.restype = None
             L.oracle_maxpool.argtypes = [_dp, _i, _i, _i, _i, _i] + [_i] * 9 + [_dp, _i, _i, _i]
             L.oracle_epilogue.restype = None
@@ -117,6 +119,31 @@ def conv(x, w, bias=None, stride=(1, 1, 1), pad=(0, 0, 0), dil=(1, 1, 1), groups
     b = None if bias is None else np.ascontiguousarray(np.asarray(bias, dtype=np.float64))
     lib().oracle_conv(_d(x), N, Ci, D, H, W, _d(w), None if b is None else _d(b), Co,
                       kd, kh, kw, *stride, *pad, *dil, _d(y), Do, Ho, Wo)
+    return y[:, :, 0] if four else y
+
+
+def conv_transpose(x, w, bias=None, stride=(1, 1, 1), pad=(0, 0, 0), dil=(1, 1, 1)):
+    """Transposed convolution, fp64 (oracle_conv_transpose: every input element scattered through the kernel).
+    x [N,Ci,D,H,W] (or 4-D), w [Co,Ci,kd,kh,kw]: w[co,ci,t] carries input channel ci to output channel co.
+    Output extent (I-1)s - 2p + d(k-1) + 1."""
+    four = np.asarray(x).ndim == 4
+    x = _as5(x)
+    w = np.asarray(w, dtype=np.float64)
+    if w.ndim == 4:
+        w = w[:, :, None]
+    w = np.ascontiguousarray(w)
+    N, Ci, D, H, W = x.shape
+    Co, Ci2, kd, kh, kw = w.shape
+    assert Ci == Ci2
+    if four:
+        stride, pad, dil = (1,) + tuple(stride[-2:]), (0,) + tuple(pad[-2:]), (1,) + tuple(dil[-2:])
+    Do = (D - 1) * stride[0] - 2 * pad[0] + dil[0] * (kd - 1) + 1
+    Ho = (H - 1) * stride[1] - 2 * pad[1] + dil[1] * (kh - 1) + 1
+    Wo = (W - 1) * stride[2] - 2 * pad[2] + dil[2] * (kw - 1) + 1
+    y = np.empty((N, Co, Do, Ho, Wo), dtype=np.float64)
+    b = None if bias is None else np.ascontiguousarray(np.asarray(bias, dtype=np.float64))
+    lib().oracle_conv_transpose(_d(x), N, Ci, D, H, W, _d(w), None if b is None else _d(b), Co,
+                                kd, kh, kw, *stride, *pad, *dil, _d(y), Do, Ho, Wo)
     return y[:, :, 0] if four else y
 
 
@@ -200,7 +227,10 @@ def run_graph(layers, x, weights, biases, dtype="bf16", keep_all=False):
     outs = []
     for l, w, b in zip(layers, weights, biases):
         src = x if l["input"] == -1 else outs[l["input"]]
-        if l["kind"] == "conv":
+        if l["kind"] == "conv" and l.get("transposed"):
+            y = conv_transpose(src, np.asarray(w, dtype=np.float64), None if b is None else np.asarray(b, np.float64),
+                               stride=l["stride"], pad=l["pad"], dil=l.get("dil", (1, 1, 1)))
+        elif l["kind"] == "conv":
             y = conv(src, np.asarray(w, dtype=np.float64), None if b is None else np.asarray(b, np.float64),
                      stride=l["stride"], pad=l["pad"], dil=l.get("dil", (1, 1, 1)), groups=l.get("groups", 1))
         else:

@@ -18,6 +18,10 @@
  *                     (SURVEY Q9), stride s, padding p, dilation d:
  *                       y[n,co,o] = sum_{ci,t} w[co,ci,t] * x[n,ci, s*o - p + d*t]   (x = 0 outside)
  *                     output extent floor((I + 2p - d(k-1) - 1)/s) + 1.
+ *   oracle_conv_transpose : transposed convolution (of the mergeable set, L378-385), the adjoint of the
+ *                     convolution's map from x to y: every input element is scattered through the kernel,
+ *                       y[n,co,s*i - p + d*t] += w[co,ci,t] * x[n,ci,i]   (positions outside the output ignored)
+ *                     output extent (I-1)s - 2p + d(k-1) + 1.
  *   oracle_maxpool  : max over the window, out-of-range positions ignored,
  *                     padding factor = pool stride (L456-458).
  *   oracle_epilogue : bias -> residual add -> ReLU -> storage rounding.
@@ -82,6 +86,42 @@ void oracle_conv(const double *x, int N, int Ci, int D, int H, int W,
                     }
                 }
                 y[IDX5(n, co, od, oh, ow, Co, Do, Ho, Wo)] = acc;
+            }
+        }
+    }
+}
+
+/* N-d transposed convolution (scatter form).  x: [N][Ci][D][H][W], w: [Co][Ci][kd][kh][kw] (w[co][ci][t] carries
+ * input channel ci to output channel co through tap t), bias: [Co] or NULL, y: [N][Co][Do][Ho][Wo]. */
+void oracle_conv_transpose(const double *x, int N, int Ci, int D, int H, int W,
+                           const double *w, const double *bias, int Co,
+                           int kd, int kh, int kw, int sd, int sh, int sw,
+                           int pd, int ph, int pw, int dd, int dh, int dw,
+                           double *y, int Do, int Ho, int Wo) {
+#pragma omp parallel for collapse(2) schedule(static)
+    for (int n = 0; n < N; n++) {
+        for (int co = 0; co < Co; co++) {
+            for (size_t q = 0; q < (size_t)Do * Ho * Wo; q++)
+                y[IDX5(n, co, 0, 0, 0, Co, Do, Ho, Wo) + q] = bias ? bias[co] : 0.0;
+            for (int ci = 0; ci < Ci; ci++)
+            for (int id = 0; id < D; id++)
+            for (int ih = 0; ih < H; ih++)
+            for (int iw = 0; iw < W; iw++) {
+                double xv = x[IDX5(n, ci, id, ih, iw, Ci, D, H, W)];
+                for (int td = 0; td < kd; td++) {
+                    int od = sd * id - pd + dd * td;
+                    if (od < 0 || od >= Do) continue;
+                    for (int th = 0; th < kh; th++) {
+                        int oh = sh * ih - ph + dh * th;
+                        if (oh < 0 || oh >= Ho) continue;
+                        for (int tw = 0; tw < kw; tw++) {
+                            int ow = sw * iw - pw + dw * tw;
+                            if (ow < 0 || ow >= Wo) continue;
+                            y[IDX5(n, co, od, oh, ow, Co, Do, Ho, Wo)] +=
+                                w[IDX5(co, ci, td, th, tw, Ci, kd, kh, kw)] * xv;
+                        }
+                    }
+                }
             }
         }
     }

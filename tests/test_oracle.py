@@ -384,3 +384,56 @@ def test_depthwise_is_per_channel():
     y = oracle.conv(x, w, pad=(1, 1), groups=3)
     for c in range(3):
         np.testing.assert_array_equal(y[:, c:c + 1], oracle.conv(x[:, c:c + 1], w[c:c + 1], pad=(1, 1)))
+
+
+# ---------------------------------------------------------------- transposed convolution (N2)
+@pytest.mark.parametrize("k,s,p,d", [(4, 2, 1, 1), (2, 2, 0, 1), (3, 2, 1, 1), (3, 1, 1, 1), (3, 1, 2, 2), (5, 3, 2, 1)])
+def test_p6_torch_conv_transpose2d(k, s, p, d):
+    """Transposed conv against torch fp64 (torch's weight is [Ci, Co, k]: ours, w[co, ci], transposed)."""
+    x = rng.standard_normal((2, 6, 7, 9))
+    w = rng.standard_normal((5, 6, k, k))
+    b = rng.standard_normal(5)
+    y = oracle.conv_transpose(x, w, bias=b, stride=(s, s), pad=(p, p), dil=(d, d))
+    ref = torch.nn.functional.conv_transpose2d(torch.from_numpy(x), torch.from_numpy(w).transpose(0, 1).contiguous(),
+                                               torch.from_numpy(b), stride=s, padding=p, dilation=d).numpy()
+    assert y.shape == ref.shape
+    np.testing.assert_allclose(y, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_p6_torch_conv_transpose3d():
+    x = rng.standard_normal((1, 3, 4, 5, 6))
+    w = rng.standard_normal((4, 3, 4, 4, 4))
+    y = oracle.conv_transpose(x, w, stride=(2, 2, 2), pad=(1, 1, 1))
+    ref = torch.nn.functional.conv_transpose3d(torch.from_numpy(x), torch.from_numpy(w).transpose(0, 1).contiguous(),
+                                               stride=2, padding=1).numpy()
+    np.testing.assert_allclose(y, ref, rtol=1e-12, atol=1e-12)
+
+
+@pytest.mark.parametrize("k,s,p,d", [(3, 2, 1, 1), (4, 2, 1, 1), (3, 1, 2, 2), (5, 3, 1, 1)])
+def test_conv_transpose_is_the_adjoint(k, s, p, d):
+    """The defining identity, independent of any library: <conv(x; w), y> = <x, conv_transpose(y; w^T)> with
+    w^T[ci, co] = w[co, ci], whenever the transposed extent returns to the conv's input extent."""
+    I = s * 7 + d * (k - 1) + 1 - 2 * p        # (I + 2p - d(k-1) - 1) divisible by s
+    x = rng.standard_normal((1, 3, I, I))
+    w = rng.standard_normal((4, 3, k, k))
+    yc = oracle.conv(x, w, stride=(s, s), pad=(p, p), dil=(d, d))
+    y = rng.standard_normal(yc.shape)
+    xt = oracle.conv_transpose(y, np.ascontiguousarray(w.transpose(1, 0, 2, 3)), stride=(s, s), pad=(p, p), dil=(d, d))
+    assert xt.shape == x.shape
+    lhs, rhs = float(np.sum(yc * y)), float(np.sum(x * xt))
+    assert abs(lhs - rhs) <= 1e-10 * max(1.0, abs(lhs))
+
+
+def test_p1_delta_input_transposed():
+    """Delta input: one input element at i spreads the kernel to outputs s*i - p + d*t."""
+    x = np.zeros((1, 1, 5, 5))
+    x[0, 0, 2, 3] = 1.0
+    w = rng.standard_normal((2, 1, 4, 4))
+    y = oracle.conv_transpose(x, w, stride=(2, 2), pad=(1, 1))
+    expect = np.zeros_like(y)
+    for r in range(4):
+        for c in range(4):
+            oh, ow = 2 * 2 - 1 + r, 2 * 3 - 1 + c
+            if 0 <= oh < y.shape[2] and 0 <= ow < y.shape[3]:
+                expect[0, :, oh, ow] = w[:, 0, r, c]
+    np.testing.assert_array_equal(y, expect)
