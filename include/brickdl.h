@@ -95,6 +95,10 @@ typedef struct bdl_layer {
                                     the mergeable set of L378-385).  Tensor-core kernels: stride 1 when dilated. */
     int32_t groups;              /* <= 1: dense conv; g > 1: grouped / depthwise (g = cin) conv, weights
                                     [cout][kd][kh][kw][cin/g]; runs on the CUDA-core brick kernels (not a dense contraction) */
+    int32_t transposed;          /* conv only: 1 = transposed convolution (the mergeable set of L378-385): input element
+                                    i reaches outputs s*i - p + d*t through tap t (weights [cout][kd][kh][kw][cin] as above,
+                                    w[co][t][ci] carrying ci to co); output extent (I-1)s - 2p + d(k-1) + 1.  groups = 1;
+                                    runs on the CUDA-core brick kernels.  0 = ordinary (cross-correlation) conv. */
 } bdl_layer;
 
 /* Static-analysis knobs (§3.3); bdl_plan_opts_default gives the paper's values, except delta_threshold. */

@@ -34,7 +34,7 @@ class bdl_layout(ctypes.Structure):
 class bdl_layer(ctypes.Structure):
     _fields_ = [("kind", _i32), ("cin", _i32), ("cout", _i32), ("k", _i32 * 3), ("stride", _i32 * 3),
                 ("pad", _i32 * 3), ("relu", _i32), ("input", _i32), ("residual", _i32), ("w", _vp),
-                ("bias", _vp), ("dil", _i32 * 3), ("groups", _i32)]
+                ("bias", _vp), ("dil", _i32 * 3), ("groups", _i32), ("transposed", _i32)]
 
 
 class bdl_plan_opts(ctypes.Structure):

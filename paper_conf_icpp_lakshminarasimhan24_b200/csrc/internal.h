@@ -29,6 +29,7 @@ struct GLayer {
     int k[4], s[4], p[4];   // index 0 (batch) always k=1, s=1, p=0
     int dl[4];              // dilation (index 0 = 1)
     int groups;             // grouped conv: output channel co reads input channels of group co / (cout/groups)
+    int tr;                 // transposed conv: output o gathers input i = (o + p - d*t) / s where divisible
     int in_ext[4], out_ext[4];
     int relu;
     int res_ext;         // 1: add the external residual view `res` (same extents as output)

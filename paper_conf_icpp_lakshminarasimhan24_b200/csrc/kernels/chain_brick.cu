@@ -55,6 +55,20 @@ __device__ __forceinline__ bool inside4(const int *e, int n, int d, int h, int w
     return n >= 0 && n < e[0] && d >= 0 && d < e[1] && h >= 0 && h < e[2] && w >= 0 && w < e[3];
 }
 
+// Input range [lo_in, lo_in + ext_in) of layer ly along dim i that its output range [lo, lo + ext) reads (Fig 4 reverse
+// traversal): I = s(O-1) + d(k-1) + 1 for a conv / pool; a transposed conv's outputs [lo, lo+ext) gather the inputs
+// i in [ceil((lo + p - d(k-1)) / s), floor((lo + ext - 1 + p) / s)].
+__device__ __forceinline__ int fdiv_d(int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
+__device__ __forceinline__ void in_range(const GLayer &ly, int i, int lo, int ext, int &lo_in, int &ext_in) {
+    if (ly.tr && i > 0) {
+        lo_in = -fdiv_d(-(lo + ly.p[i] - ly.dl[i] * (ly.k[i] - 1)), ly.s[i]);
+        ext_in = max(0, fdiv_d(lo + ext - 1 + ly.p[i], ly.s[i]) + 1 - lo_in);
+    } else {
+        lo_in = lo * ly.s[i] - ly.p[i];
+        ext_in = (ext - 1) * ly.s[i] + ly.dl[i] * (ly.k[i] - 1) + 1;
+    }
+}
+
 // Evaluate one output element (position pos, channel co) of layer `ly`.
 template <typename T, bool FromRegion>
 __device__ __forceinline__ float eval_elem(const GLayer &ly, const BrickSrc<T> &bs, const RegionBuf &rs,
@@ -67,9 +81,19 @@ __device__ __forceinline__ float eval_elem(const GLayer &ly, const BrickSrc<T> &
     for (int td = 0; td < ly.k[1]; td++)
         for (int th = 0; th < ly.k[2]; th++)
             for (int tw = 0; tw < ly.k[3]; tw++, tap++) {
-                int id = d * ly.s[1] - ly.p[1] + td * ly.dl[1];
-                int ih = h * ly.s[2] - ly.p[2] + th * ly.dl[2];
-                int iw = w * ly.s[3] - ly.p[3] + tw * ly.dl[3];
+                int id, ih, iw;
+                if (ly.tr) {   // transposed conv (L378-385): input i reaches output s*i - p + d*t
+                    const int nd = d + ly.p[1] - td * ly.dl[1], nh = h + ly.p[2] - th * ly.dl[2];
+                    const int nw = w + ly.p[3] - tw * ly.dl[3];
+                    if (nd < 0 || nh < 0 || nw < 0 || nd % ly.s[1] || nh % ly.s[2] || nw % ly.s[3]) continue;
+                    id = nd / ly.s[1];
+                    ih = nh / ly.s[2];
+                    iw = nw / ly.s[3];
+                } else {
+                    id = d * ly.s[1] - ly.p[1] + td * ly.dl[1];
+                    ih = h * ly.s[2] - ly.p[2] + th * ly.dl[2];
+                    iw = w * ly.s[3] - ly.p[3] + tw * ly.dl[3];
+                }
                 if (!inside4(ly.in_ext, n, id, ih, iw)) continue;
                 if (pool) {
                     float v = FromRegion ? rs.p[rs.idx(n, id, ih, iw) + co] : to_f(bs.base(n, id, ih, iw)[co]);
@@ -158,8 +182,8 @@ __global__ void __launch_bounds__(256) padded_chain_kernel(GChain g) {
                 for (int i = 0; i < 4; i++) { s_lo[j][i] = lo[i]; s_ext[j][i] = ext[i]; }
                 const GLayer &ly = g.layer[j];
                 for (int i = 0; i < 4; i++) {
-                    int nlo = lo[i] * ly.s[i] - ly.p[i];
-                    int next = (ext[i] - 1) * ly.s[i] + ly.dl[i] * (ly.k[i] - 1) + 1;
+                    int nlo, next;
+                    in_range(ly, i, lo[i], ext[i], nlo, next);
                     lo[i] = nlo;
                     ext[i] = next;
                 }
@@ -203,8 +227,9 @@ __device__ __forceinline__ DepBox dep_box(const GChain &g, int l, long long b) {
     brick_region(ly.out, b, lo, ext);
     DepBox box;
     for (int i = 0; i < 4; i++) {
-        int a = lo[i] * ly.s[i] - ly.p[i];
-        int e = (lo[i] + ext[i] - 1) * ly.s[i] - ly.p[i] + ly.dl[i] * (ly.k[i] - 1) + 1;  // exclusive
+        int a, e;
+        in_range(ly, i, lo[i], ext[i], a, e);
+        e += a;   // exclusive
         a = max(a, 0);
         e = min(e, ly.in_ext[i]);
         box.lo[i] = a / src.B[i];
@@ -472,6 +497,7 @@ bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &i
             G.k[d + 1] = ly.L.k[d]; G.s[d + 1] = ly.L.stride[d]; G.p[d + 1] = ly.L.pad[d]; G.dl[d + 1] = ly.L.dil[d];
         }
         G.groups = ly.L.groups;
+        G.tr = ly.L.transposed;
         for (int d = 0; d < 4; d++) { G.in_ext[d] = ly.in_ext[d]; G.out_ext[d] = ly.out_ext[d]; }
         G.relu = ly.L.relu;
         G.w = ly.L.kind == BDL_OP_CONV ? (const float *)(ws + ly.w_off) : nullptr;

@@ -1957,7 +1957,7 @@ int gen_conv_layers(const bdl_plan *p, const Subgraph &sg) {
     if (p->layers[sg.last].L.kind == BDL_OP_MAXPOOL) L--;
     if (L < 1 || L > kMaxLayers) return 0;
     for (int j = 0; j < L; j++) {
-        if (p->layers[sg.first + j].L.kind != BDL_OP_CONV) return 0;
+        if (p->layers[sg.first + j].L.kind != BDL_OP_CONV || p->layers[sg.first + j].L.transposed) return 0;
         const bool res = p->layers[sg.first + j].L.residual != BDL_NO_RESIDUAL;
         if (res && sg.res_tensor[j] < 0 && sg.res_local[j] < 0) return 0;
     }
@@ -1972,6 +1972,7 @@ int gen_conv_layers(const bdl_plan *p, const Subgraph &sg) {
 bool gen_layer_supported(const bdl_plan *p, int li) {
     if (p->in_layout.dtype != BDL_BF16 || p->in_layout.Bn != 1) return false;
     const Layer &ly = p->layers[li];
+    if (ly.L.transposed) return false;   // transposed convs: CUDA-core brick kernels
     bdl_layout lo;
     bdl_layout_init(&lo, p->in_layout.nsp, ly.out_ext[0], ly.L.cout, ly.out_ext[1], ly.out_ext[2], ly.out_ext[3],
                     p->in_layout.Bn, p->in_layout.Bd, p->in_layout.Bh, p->in_layout.Bw, BDL_BF16);

@@ -13,8 +13,12 @@
 
 namespace bdl {
 
-// Output extent of a layer along one dim: floor((I + 2p - (k-1) - 1)/s) + 1.
-static int out_extent(int I, int k, int s, int p, int d) { return (I + 2 * p - d * (k - 1) - 1) / s + 1; }
+// Output extent of a layer along one dim: floor((I + 2p - (k-1) - 1)/s) + 1; transposed conv (I-1)s - 2p + d(k-1) + 1.
+static int out_extent(int I, int k, int s, int p, int d, int tr = 0) {
+    return tr ? (I - 1) * s - 2 * p + d * (k - 1) + 1 : (I + 2 * p - d * (k - 1) - 1) / s + 1;
+}
+static int64_t fdiv(int64_t a, int64_t b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }   // floor(a / b), b > 0
+static int64_t cdiv(int64_t a, int64_t b) { return -fdiv(-a, b); }                            // ceil(a / b)
 // Input extent of one window, d(k-1) + 1.  Layers are normalized at partition time (dil >= 1).
 static int keff(const bdl_layer &l, int dim) { return (l.dil[dim] > 1 ? l.dil[dim] : 1) * (l.k[dim] - 1) + 1; }
 
@@ -42,7 +46,12 @@ static void regions_dag(const std::vector<Layer> &ly, int first, int last, int d
         const bdl_layer &l = ly[first + j].L;
         int k = dim == 0 ? 1 : keff(l, dim - 1), s = dim == 0 ? 1 : l.stride[dim - 1], p = dim == 0 ? 0 : l.pad[dim - 1];
         int64_t lo, hi;
-        if (halo) {
+        if (dim > 0 && l.kind == BDL_OP_CONV && l.transposed) {
+            // transposed conv: input i reaches outputs s*i - p + d*t, t < k: the inputs reaching [olo, ohi)
+            const int kk = halo ? k : std::min(k, s), pp = halo ? p : 0;
+            lo = cdiv(olo[j] + pp - (kk - 1), s);
+            hi = fdiv(ohi[j] - 1 + pp, s) + 1;
+        } else if (halo) {
             lo = olo[j] * s - p;               // input extent I = s(O-1) + k (Q19)
             hi = (ohi[j] - 1) * s - p + k;
         } else {                               // halo-free: non-overlapping windows of the same stride
@@ -164,7 +173,7 @@ static bool tc_eligible(const bdl_plan *p, const Subgraph &sg) {
     int nsp = p->in_layout.nsp;
     for (int j = sg.first; j <= sg.last; j++) {
         const bdl_layer &l = p->layers[j].L;
-        if (l.kind != BDL_OP_CONV || l.cin != C || l.cout != C || l.groups != 1) return false;
+        if (l.kind != BDL_OP_CONV || l.cin != C || l.cout != C || l.groups != 1 || l.transposed) return false;
         if (l.dil[0] != 1 || l.dil[1] != 1 || l.dil[2] != 1) return false;
         for (int d = 0; d < 3; d++) {
             bool spatial = (nsp == 3) || d > 0;
@@ -221,6 +230,10 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             bdl_plan_destroy(p);
             return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": groups must divide cin and cout (convs only)");
         }
+        if (l.transposed && (l.kind != BDL_OP_CONV || l.groups != 1)) {
+            bdl_plan_destroy(p);
+            return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": transposed convs only (groups = 1)");
+        }
         if (l.kind == BDL_OP_MAXPOOL && (l.dil[0] != 1 || l.dil[1] != 1 || l.dil[2] != 1)) {
             bdl_plan_destroy(p);
             return fail(BDL_EUNSUPPORTED, "layer " + std::to_string(i) + ": dilated pooling");
@@ -252,7 +265,7 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
                 bdl_plan_destroy(p);
                 return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": bad kernel/stride/pad");
             }
-            L.out_ext[d + 1] = out_extent(L.in_ext[d + 1], l.k[d], l.stride[d], l.pad[d], l.dil[d]);
+            L.out_ext[d + 1] = out_extent(L.in_ext[d + 1], l.k[d], l.stride[d], l.pad[d], l.dil[d], l.transposed);
             if (L.out_ext[d + 1] <= 0) {
                 bdl_plan_destroy(p);
                 return fail(BDL_EINVAL, "layer " + std::to_string(i) + ": empty output");
@@ -303,8 +316,10 @@ bdl_status bdl_graph_partition(const bdl_layer *layers, int32_t nlayers, const b
             if (!(j == end && is_pool(p->layers[j]))) all_gen = all_gen && gen_layer_supported(p, j);
             // bf16: grouped (depthwise) convs run on the CUDA-core kernels, dense ones on the tensor cores: the two
             // do not share a subgraph (the whole subgraph runs on one kernel)
+            // (transposed convs too: CUDA-core only)
+            auto cc = [&](int q) { return p->layers[q].L.groups > 1 || p->layers[q].L.transposed; };
             if (in->dtype == BDL_BF16 && j > first && p->layers[j].L.kind == BDL_OP_CONV &&
-                p->layers[j - 1].L.kind == BDL_OP_CONV && (p->layers[j].L.groups > 1) != (p->layers[j - 1].L.groups > 1))
+                p->layers[j - 1].L.kind == BDL_OP_CONV && cc(j) != cc(j - 1))
                 return false;
         }
         if (branch && !(dag_ok && all_gen)) return false;

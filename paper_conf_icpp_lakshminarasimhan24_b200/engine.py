@@ -66,6 +66,7 @@ class Plan:
                 a.k[d], a.stride[d], a.pad[d] = l["k"][d], l["stride"][d], l["pad"][d]
                 a.dil[d] = l.get("dil", (1, 1, 1))[d]
             a.groups = l.get("groups", 1)
+            a.transposed = 1 if l.get("transposed") else 0
             a.relu = int(l["relu"])
             a.input = l["input"]
             a.residual = BDL_NO_RESIDUAL if l["residual"] is None else l["residual"]

@@ -43,15 +43,16 @@ CONFIGS = {
 _CFG_NUM = {"cfg1": 1, "cfg2": 2, "cfg3": 3, "cfg4": 4, "cfg5": 5}
 
 
-def _conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2, dil=1, groups=1):
+def _conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2, dil=1, groups=1,
+          transposed=False):
     if p is None:
-        p = dil * (k - 1) // 2
+        p = dil * (k - 1) // 2 if not transposed else (dil * (k - 1) + 1 - s) // 2   # transposed: output = s * input
     if nsp == 3:
         kk, ss, pp, dd = (k, k, k), (s, s, s), (p, p, p), (dil, dil, dil)
     else:
         kk, ss, pp, dd = (1, k, k), (1, s, s), (0, p, p), (1, dil, dil)
     return dict(kind="conv", cin=cin, cout=cout, k=kk, stride=ss, pad=pp, relu=relu,
-                input=inp, residual=res, wscale=wscale, dil=dd, groups=groups)
+                input=inp, residual=res, wscale=wscale, dil=dd, groups=groups, transposed=bool(transposed))
 
 
 def _pool(c, k, s, p):
@@ -106,10 +107,14 @@ def make_layers(cfg: str, C: int | None = None, nlayers: int | None = None):
 
 
 def layer_out_shape(layer, D, H, W):
-    """Output spatial extent of one layer: floor((I + 2p - d(k-1) - 1)/s) + 1 per dim."""
+    """Output spatial extent of one layer: floor((I + 2p - d(k-1) - 1)/s) + 1 per dim (transposed conv:
+    (I-1)s - 2p + d(k-1) + 1)."""
     out = []
     for I, k, s, p, d in zip((D, H, W), layer["k"], layer["stride"], layer["pad"], layer.get("dil", (1, 1, 1))):
-        out.append((I + 2 * p - d * (k - 1) - 1) // s + 1)
+        if layer.get("transposed"):
+            out.append((I - 1) * s - 2 * p + d * (k - 1) + 1)
+        else:
+            out.append((I + 2 * p - d * (k - 1) - 1) // s + 1)
     return tuple(out)
 
 
@@ -134,10 +139,12 @@ def make_workload(cfg: str, N=None, C=None, D=None, H=None, W=None, nlayers=None
     return wl
 
 
-def conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2, dil=1, groups=1):
+def conv(cin, cout, k=3, s=1, p=None, relu=True, inp=None, res=None, wscale=1.0, nsp=2, dil=1, groups=1,
+         transposed=False):
     """Layer dict of a conv (public form of the graph builder used by the configurations).  dil: dilation;
-    groups: grouped conv (groups = cin: depthwise), weights [cout, cin/groups, k...]."""
-    return _conv(cin, cout, k, s, p, relu, inp, res, wscale, nsp, dil, groups)
+    groups: grouped conv (groups = cin: depthwise), weights [cout, cin/groups, k...]; transposed: transposed conv
+    (weights [cout, cin, k...], w[co, ci] carrying ci to co; default padding makes the output s x the input)."""
+    return _conv(cin, cout, k, s, p, relu, inp, res, wscale, nsp, dil, groups, transposed)
 
 
 def pool(c, k, s, p):

@@ -242,3 +242,28 @@ def test_grouped_and_depthwise(dtype):
         assert rel_err(outs[mode], ref) <= (TOL if dtype == "bf16" else 1e-5), (mode, rel_err(outs[mode], ref))
     np.testing.assert_array_equal(outs["memoized"], outs["unmerged"])
     np.testing.assert_array_equal(outs["memoized"], outs["padded"])
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_transposed_conv_chain(dtype):
+    """Transposed convs (the last of the L378-385 mergeable ops): an encoder-decoder chain -- 3x3 stride-2 conv down,
+    2x upsampling transposed conv (k 4, s 2, p 1), a dilated stride-1 transposed conv, a 3x3 conv with the graph input
+    as residual -- runs on the CUDA-core brick kernels (bf16: the dense convs stay on the tensor cores); every mode
+    against the oracle, the merged modes bit-equal to unmerged."""
+    layers = [W.conv(16, 32, 3, s=2), W.conv(32, 16, 4, s=2, transposed=True), W.conv(16, 16, 3, dil=2, transposed=True),
+              W.conv(16, 16, 3, res=-1, wscale=0.5)]
+    wl = W.make_graph_workload(layers, 2, 16, 1, 20, 24, 2, (1, 1, 8, 8), dtype, seed=31)
+    assert tuple(wl["x"].shape[-2:]) == (20, 24)
+    ref = oracle.run_graph(wl["layers"], wl["x"].numpy(), wl["weights"], wl["biases"], dtype=dtype)
+    assert ref.shape[-2:] == (20, 24)
+    plan = engine.plan_from_workload(wl, force_mode=2)
+    if dtype == "bf16":
+        kinds = {s["kernel"] for s in plan.subgraphs()}
+        assert "cuda-core brick" in kinds and "tcgen05 generic" in kinds, kinds
+    outs = {}
+    for mode in ("memoized", "padded", "unmerged"):
+        plan.set_mode(mode)
+        outs[mode] = plan.forward(wl["x"]).float().cpu().numpy()
+        assert rel_err(outs[mode], ref) <= (TOL if dtype == "bf16" else 1e-5), (mode, rel_err(outs[mode], ref))
+    np.testing.assert_array_equal(outs["memoized"], outs["unmerged"])
+    np.testing.assert_array_equal(outs["memoized"], outs["padded"])

@@ -284,3 +284,42 @@ def test_gloo_two_ranks_cover_batch_once():
     for p in procs:
         p.join(timeout=60)
     assert got == list(range(37)) and tmax == 2.0
+
+
+# ------------------------------------------------------------------------------ transposed convolution regions
+def _tlayers(specs):
+    """specs: (k, s, p, d, transposed) per layer, 8 channels, a chain along the listing."""
+    arr = (bdl.bdl_layer * len(specs))()
+    for i, (k, s, p, d, tr) in enumerate(specs):
+        a = arr[i]
+        a.kind = bdl.BDL_OP_CONV
+        a.cin = a.cout = 8
+        a.k[:] = [1, k, k]
+        a.stride[:] = [1, s, s]
+        a.pad[:] = [0, p, p]
+        a.dil[:] = [1, d, d]
+        a.input = i - 1
+        a.residual = bdl.BDL_NO_RESIDUAL
+        a.transposed = tr
+    return arr
+
+
+def _tregions(specs, b):
+    out = (ctypes.c_int64 * len(specs))()
+    bdl.check(bdl.lib().bdl_region_extents(_tlayers(specs), 0, len(specs) - 1, 2, b, out))
+    return list(out)
+
+
+@pytest.mark.parametrize("k,s,p,d", [(4, 2, 1, 1), (2, 2, 0, 1), (3, 2, 1, 1), (3, 1, 1, 2), (5, 3, 2, 1)])
+def test_region_transposed_brute_force(k, s, p, d):
+    """Reverse traversal through a transposed conv: the input region of an output brick [0, b) is the hull of the
+    inputs i with s*i - p + d*t in [0, b) for some tap t (enumerated here)."""
+    for b in (4, 8, 16):
+        reach = [i for i in range(-4 * b, 4 * b) if any(0 <= s * i - p + d * t < b for t in range(k))]
+        assert _tregions([(k, s, p, d, 1)], b) == [max(reach) - min(reach) + 1]
+
+
+def test_region_chain_through_transposed():
+    # 3x3 conv (p = 1) then a 2x upsampling transposed conv (k 4, s 2, p 1): brick 8 of the output needs inputs
+    # [-1, 4] of the transposed conv (6) and 6 + 2 of the first conv
+    assert _tregions([(3, 1, 1, 1, 0), (4, 2, 1, 1, 1)], 8) == [8, 6]
