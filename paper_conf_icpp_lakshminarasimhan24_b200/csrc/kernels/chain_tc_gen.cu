@@ -1033,7 +1033,9 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
             PT(const unsigned long long tlb = p.prof ? clock64() : 0;)
             asm volatile("bar.sync 1, %0;" ::"n"(kLoadT) : "memory");
             PT(if (p.prof) wbar += clock64() - tlb;)
-            if (l >= 0 && p.layer[l].tma) ptx::fence_proxy_async();   // acquired data is read by TMA (async proxy)
+            // acquired data (generic-proxy stores of other CTAs) is read by TMA (async proxy); a source written by an earlier
+            // grid needs no fence, and the global-memory proxy fence is the one needed (the full fence: ~1 us per task)
+            if (l >= 0 && p.layer[l].tma && p.layer[l].srcl >= 0 && !p.padded) asm volatile("fence.proxy.async.global;" ::: "memory");
             if (tid == 0) {
                 sh.desc_l[seq % kRing] = l;
                 sh.desc_t[seq % kRing] = t;
