@@ -76,3 +76,23 @@ def test_pair_three_layer_chain():
     c = plan.counters(0)
     tasks = 3 * N * -(-H // sg[0]["tc_band"])   # every (layer, band) task computed exactly once
     assert c["computed"] == tasks and c["cas_ok"] == tasks, c
+
+
+@pytest.mark.parametrize("brick,H,W", [((1, 1, 4, 4), 36, 52), ((1, 1, 8, 16), 30, 48), ((1, 1, 2, 8), 17, 40)])
+def test_pair_other_bricks(brick, H, W):
+    """Other brick shapes: the band row is W + Bw pixels (the out-of-map brick is the zero pad) and TMA boxes never
+    cross a brick row, so the pair kernel must match the single-CTA kernel bit for bit and the oracle."""
+    layers = workloads.make_layers("cfg2")
+    wl = workloads.make_graph_workload(layers, 3, 64, 1, H, W, 2, brick, "bf16", seed=7)
+    plan, pair = run_modes(wl)
+    assert plan.subgraphs()[0]["cta_pair"]
+
+    def single_cta():
+        plan1, outs = run_modes(wl)
+        assert not plan1.subgraphs()[0]["cta_pair"]
+        return outs
+
+    single = with_env("BDL_NO_PAIR", "1", single_cta)
+    for m in pair:
+        np.testing.assert_array_equal(pair[m], single[m])
+    assert rel_err(pair["memoized"], oracle_out(wl)) <= TOL["bf16"]
