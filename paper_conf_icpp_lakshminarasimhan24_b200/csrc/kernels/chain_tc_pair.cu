@@ -761,6 +761,7 @@ bool pair_geometry(int L, int H, int W, int Bw, int N, int num_sms, int &Tb, int
         const int m = (tb - 1) * Wt + W;
         const int nt = (m + 127) / 128;
         if (nt > pr::kMaxTl) continue;
+        if ((long long)N * ((H + tb - 1) / tb) >= (1LL << 24)) continue;   // order entries: (layer << 24) | task
         const int rows = std::max(pr::kG + nt * 128 + 2 * Wt + 1, pr::kG + (tb + 2) * Wt);
         const int ib = (rows * 128 + 1023) / 1024 * 1024;
         for (int ni = pr::kMaxNin; ni >= 2; ni--) {
