@@ -166,3 +166,20 @@ def test_gloo_batch_gather_equals_unsharded(world):
     for p in procs:
         p.join(timeout=60)
     assert res == {r: True for r in range(world)}
+
+
+def test_torchrun_batch_gather():
+    """The multi-process launch the driver uses (python -m torch.distributed.run, env:// rendezvous on 127.0.0.1,
+    one process per rank), here with 2 CPU ranks over gloo: the batch runner's all-gather equals the unsharded batch."""
+    import subprocess
+    import sys
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_torchrun_gather.py")
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+                        "--master-addr", "127.0.0.1", "--master-port", str(port), script],
+                       capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    assert "GATHER_OK" in r.stdout, r.stdout[-2000:]
