@@ -90,6 +90,7 @@ struct Shared {
     uint64_t pf_bar;             // first-band prefetch landed
     uint64_t desc_full[kRing];
     uint64_t epi_done[kRing];    // the CTA's epilogue warps have stored the slot's task (kEpiWarps arrivals)
+    uint64_t pub_free[kRing];    // the publisher is done with the slot (the loader may reuse it)
     uint32_t tmem_base;
     int q_l[kQ], q_t[kQ], q_n[kQ];
     unsigned long long q_ts[kQ][4];   // debug trace (leader): ticket drawn, claimed, dependencies scanned, emitted
@@ -370,6 +371,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
         for (int i = 0; i < kRing; i++) {
             ptx::mbar_init(&sh.desc_full[i], 1);
             ptx::mbar_init(&sh.epi_done[i], kEpiWarps);
+            ptx::mbar_init(&sh.pub_free[i], 1);
         }
         ptx::fence_barrier_init();
     }
@@ -485,6 +487,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
             // (layer 0 reads the subgraph input, written by an earlier grid: no proxy fence needed)
             if (work && l > 0 && !(p.knob & 4)) asm volatile("fence.proxy.async.global;" ::: "memory");
             if (seq >= (uint32_t)p.nin) ptx::mbar_wait(&sh.in_empty[b], ((seq / p.nin) - 1) & 1);
+            // the descriptor slot's previous task is published (the epilogue may run ahead of the publisher: without
+            // this, a slot's epi_done could complete two phases before the publisher waits on the first)
+            if (seq >= (uint32_t)kRing) ptx::mbar_wait(&sh.pub_free[seq % kRing], ((seq / kRing) - 1) & 1);
             if (lane == 0) {
                 sh.desc_l[seq % kRing] = l;
                 sh.desc_t[seq % kRing] = t;
@@ -687,7 +692,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
             ptx::mbar_wait(&sh.desc_full[slot], (seq / kRing) & 1);
             const int l = sh.desc_l[slot], t = sh.desc_t[slot];
             if (l < 0) break;
-            if (t < 0) continue;
+            if (t < 0) {
+                __syncwarp();
+                if (lane == 0) arrive_local(&sh.pub_free[slot]);
+                continue;
+            }
             ptx::mbar_wait(&sh.epi_done[slot], (ph >> slot) & 1);
             ph ^= 1u << slot;
             if (lane == 0) {
@@ -711,7 +720,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
                         rec[15] = sh.tr[slot][12];  // scheduler: dependencies scanned
                     }
                 }
+                arrive_local(&sh.pub_free[slot]);
             }
+            __syncwarp();
         }
         if (computed) atomicAdd(&p.counters[0], computed);
     }
