@@ -203,11 +203,13 @@ __device__ void scheduler(const Params &p, Shared &sh, int e_first) {
     // Claim the not-started dependencies of one or two same-layer roots (Fig 2d), breadth first, so every stack entry
     // sits below its dependencies; emit from the top (dependencies first), pairing neighbours of one layer.
     auto expand = [&](int rl, int ra, int rb) {
+        // (with two roots ra sits on top of rb, so the pair is emitted as (ra, rb): the leader gets ra -- the order entry
+        // it prefetched the band of, for the static first ticket)
         if (lane == 0) {
             sh.stk_l[0] = rl;
-            sh.stk_t[0] = ra;
+            sh.stk_t[0] = rb >= 0 ? rb : ra;
             sh.stk_l[1] = rl;
-            sh.stk_t[1] = rb;
+            sh.stk_t[1] = ra;
         }
         int sp = rb >= 0 ? 2 : 1;
         for (int s = 0; s < sp; s++) {
