@@ -370,7 +370,9 @@ __device__ __forceinline__ long long tv_off_p2(const TView &v, const int *lB, in
     return tv_phys(v, logical) * v.brick_elems + (long long)in * v.Cp;
 }
 
-template <typename T, bool P2>
+// K > 0: a 2-D K x K window, unrolled so that all its loads are in flight at once (the generic loop waits for each tap's
+// load before the next: ~3 TB/s on VGG-16's pools)
+template <typename T, bool P2, int K>
 __global__ void __launch_bounds__(256) pool_vec_kernel(GLayer ly, TView in, unsigned long long *counter, int4 lb4) {
     const int lB[4] = {lb4.x, lb4.y, lb4.z, lb4.w};
     constexpr int V = 16 / sizeof(T);
@@ -415,7 +417,29 @@ __global__ void __launch_bounds__(256) pool_vec_kernel(GLayer ly, TView in, unsi
 #pragma unroll
         for (int j = 0; j < V; j++) m[j] = -INFINITY;
         bool any = false;
-        if (inside4(ly.out_ext, n, d, h, w)) {
+        if (K > 0 && inside4(ly.out_ext, n, d, h, w)) {
+            constexpr int KK = K > 0 ? K * K : 1;
+            uint4 q[KK];
+            bool ok[KK];
+#pragma unroll
+            for (int th = 0; th < K; th++)
+#pragma unroll
+                for (int tw = 0; tw < K; tw++) {
+                    const int ih = h * ly.s[2] - ly.p[2] + th, iw = w * ly.s[3] - ly.p[3] + tw;
+                    const int id = d * ly.s[1] - ly.p[1];
+                    ok[th * K + tw] = inside4(ly.in_ext, n, id, ih, iw);
+                    const long long eo = ok[th * K + tw] ? (P2 ? tv_off_p2(in, lB, n, id, ih, iw) : tv_off(in, n, id, ih, iw)) : 0;
+                    q[th * K + tw] = __ldg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(in.ptr) + eo + cv * V));
+                }
+#pragma unroll
+            for (int t = 0; t < K * K; t++) {
+                if (!ok[t]) continue;
+                const T *e = reinterpret_cast<const T *>(&q[t]);
+#pragma unroll
+                for (int j = 0; j < V; j++) m[j] = fmaxf(m[j], to_f(e[j]));
+                any = true;
+            }
+        } else if (K == 0 && inside4(ly.out_ext, n, d, h, w)) {
             for (int td = 0; td < ly.k[1]; td++) {
                 const int id = d * ly.s[1] - ly.p[1] + td;
                 for (int th = 0; th < ly.k[2]; th++) {
@@ -544,13 +568,21 @@ bdl_status launch_brick_subgraph(bdl_plan *p, const Subgraph &sg, const TView &i
                 auto lg = [](int v) { int r = 0; while ((1 << r) < v) r++; return (1 << r) == v ? r : -1; };
                 const int4 lb4 = make_int4(lg(src.B[0]), lg(src.B[1]), lg(src.B[2]), lg(src.B[3]));
                 const bool p2 = lb4.x >= 0 && lb4.y >= 0 && lb4.z >= 0 && lb4.w >= 0;
+                const int kk = G.k[1] == 1 && G.k[2] == G.k[3] && (G.k[2] == 2 || G.k[2] == 3) ? G.k[2] : 0;
+#define BDL_POOL_LAUNCH(TT, PP)                                                                            \
+    do {                                                                                                  \
+        if (kk == 2) pool_vec_kernel<TT, PP, 2><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);              \
+        else if (kk == 3) pool_vec_kernel<TT, PP, 3><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);         \
+        else pool_vec_kernel<TT, PP, 0><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);                       \
+    } while (0)
                 if (g.bf16) {
-                    if (p2) pool_vec_kernel<__nv_bfloat16, true><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);
-                    else pool_vec_kernel<__nv_bfloat16, false><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);
+                    if (p2) BDL_POOL_LAUNCH(__nv_bfloat16, true);
+                    else BDL_POOL_LAUNCH(__nv_bfloat16, false);
                 } else {
-                    if (p2) pool_vec_kernel<float, true><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);
-                    else pool_vec_kernel<float, false><<<gp, 256, 0, s>>>(G, src, g.counters, lb4);
+                    if (p2) BDL_POOL_LAUNCH(float, true);
+                    else BDL_POOL_LAUNCH(float, false);
                 }
+#undef BDL_POOL_LAUNCH
                 *launches += 1;
                 continue;
             }
