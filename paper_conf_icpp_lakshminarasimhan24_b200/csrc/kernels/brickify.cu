@@ -125,6 +125,46 @@ __global__ void __launch_bounds__(256) unbrickify_kernel(TView v, T *__restrict_
     }
 }
 
+// Unbrickify of maps whose rows are not whole 16-B vectors (W % V != 0: ResNet-50's and VGG-16's 7 x 7 outputs):
+// a CTA takes kSmallPx pixels of one sample's (D, H, W) volume x 128 bytes of channels, reads each pixel's channel
+// run (coalesced: channels are innermost in a brick) into shared memory, and writes every channel's pixel run
+// contiguously (consecutive threads -> consecutive pixels of one channel plane).  The register-transpose kernel
+// wrote 2-byte scattered stores there (0.47 TB/s on ResNet-50's output).
+constexpr int kSmallPx = 256;
+template <typename T>
+__global__ void __launch_bounds__(256) unbrickify_small_kernel(TView v, T *__restrict__ dstd) {
+    constexpr int CB = 128 / sizeof(T);   // channels per block (128 B per pixel)
+    __shared__ T tile[kSmallPx][CB + 2];  // (+2: consecutive pixels in different banks)
+    pdl_wait();
+    const long long vol = (long long)v.ext[1] * v.ext[2] * v.ext[3];
+    const int nchunk = (int)((vol + kSmallPx - 1) / kSmallPx), ncb = (v.Cp + CB - 1) / CB;
+    long long bid = blockIdx.x;
+    const int cb = (int)(bid % ncb);
+    bid /= ncb;
+    const int chunk = (int)(bid % nchunk);
+    const int n = (int)(bid / nchunk);
+    const long long p0 = (long long)chunk * kSmallPx;
+    const int np = (int)std::min<long long>(kSmallPx, vol - p0);
+    const T *src = reinterpret_cast<const T *>(v.ptr);
+    constexpr int V = 16 / sizeof(T);
+    for (int i = threadIdx.x; i < np * (CB / V); i += blockDim.x) {   // 16-B chunks of each pixel's channel run
+        const int px = i / (CB / V), q = i % (CB / V);
+        const long long p = p0 + px;
+        const int w = (int)(p % v.ext[3]), h = (int)((p / v.ext[3]) % v.ext[2]), d = (int)(p / ((long long)v.ext[3] * v.ext[2]));
+        const int c = cb * CB + q * V;
+        Vec<T> val;
+        val.u = c < v.Cp ? __ldg(reinterpret_cast<const uint4 *>(src + brick_px(v, n, d, h, w) + c)) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+        for (int e = 0; e < V; e++) tile[px][q * V + e] = val.e[e];
+    }
+    __syncthreads();
+    const int nc = min(CB, v.C - cb * CB);
+    for (int i = threadIdx.x; i < nc * np; i += blockDim.x) {
+        const int c = i / np, px = i % np;
+        dstd[((long long)n * v.C + cb * CB + c) * vol + p0 + px] = tile[px][c];
+    }
+}
+
 bool launch_convert_tma(const bdl_layout *l, const void *dense, void *bricked, cudaStream_t s, bool to_bricks,
                         bdl_status *st);
 
@@ -150,6 +190,17 @@ static bdl_status launch_convert(const bdl_layout *l, const void *src, void *dst
     const int threads = 256;
     const long long blocks = std::max<long long>(1, std::min<long long>((units + threads - 1) / threads, 148LL * 16));
     cudaStream_t s = (cudaStream_t)stream;
+    if (!to_bricks && !cg.vec_ok && l->Bn == 1) {   // rows that are not whole 16-B vectors: shared-memory transpose
+        const long long vol = l->D * l->H * l->W;
+        const int CB = 128 / E;
+        const long long nb = l->N * ((vol + kSmallPx - 1) / kSmallPx) * ((l->c_pad + CB - 1) / CB);
+        if (l->dtype == BDL_F32)
+            launch_pdl(unbrickify_small_kernel<float>, dim3((unsigned)nb), dim3(threads), 0, s, v, (float *)dst);
+        else
+            launch_pdl(unbrickify_small_kernel<__nv_bfloat16>, dim3((unsigned)nb), dim3(threads), 0, s, v, (__nv_bfloat16 *)dst);
+        BDL_CUDA_CHECK_LAUNCH("bdl_unbrickify");
+        return BDL_OK;
+    }
     if (l->dtype == BDL_F32) {
         if (to_bricks) brickify_kernel<float><<<(unsigned)blocks, threads, 0, s>>>(v, (const float *)src, cg);
         else launch_pdl(unbrickify_kernel<float>, dim3((unsigned)blocks), dim3(threads), 0, s, v, (float *)dst, cg);
