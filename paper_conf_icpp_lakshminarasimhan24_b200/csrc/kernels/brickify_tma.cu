@@ -12,6 +12,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <string>
 
 #include "common.cuh"
@@ -94,14 +95,24 @@ __global__ void __launch_bounds__(128) brickify_tma_kernel(const __grid_constant
             in[k] = *reinterpret_cast<const uint4 *>(swz(row, j));
         }
         transpose8(in, out);
-        // pixels x = 8q .. 8q+7 lie in one brick (Bw is a multiple of 8 or 8 a multiple of Bw: per-pixel brick index)
+        // pixels x = 8q .. 8q+7: one brick when Bw >= 8 (consecutive pixels Cp channels apart), else Bw-pixel runs
+        const long long brow = ((long long)n * p.nbh + (y >> p.lBh)) * p.nbx;
+        const int yin = (y & (p.Bh - 1)) << p.lBw;
+        if (p.Bw >= 8) {
+            const long long off = (brow + ((q * 8) >> p.lBw)) * p.brick_elems +
+                                  (long long)(yin + ((q * 8) & (p.Bw - 1))) * p.Cp + cb * 64 + g * 8;
+            uint4 *dst = reinterpret_cast<uint4 *>(out_base + off * 2);
+            const int step = p.Cp / 8;   // 16-B vectors per pixel
 #pragma unroll
-        for (int i = 0; i < 8; i++) {
-            const int x = q * 8 + i;
-            const long long brick = ((long long)n * p.nbh + (y >> p.lBh)) * p.nbx + (x >> p.lBw);
-            const long long off = brick * p.brick_elems +
-                                  (long long)(((y & (p.Bh - 1)) << p.lBw) + (x & (p.Bw - 1))) * p.Cp + cb * 64 + g * 8;
-            *reinterpret_cast<uint4 *>(out_base + off * 2) = out[i];
+            for (int i = 0; i < 8; i++) dst[i * step] = out[i];
+        } else {
+#pragma unroll
+            for (int i = 0; i < 8; i++) {
+                const int x = q * 8 + i;
+                const long long off = (brow + (x >> p.lBw)) * p.brick_elems +
+                                      (long long)(yin + (x & (p.Bw - 1))) * p.Cp + cb * 64 + g * 8;
+                *reinterpret_cast<uint4 *>(out_base + off * 2) = out[i];
+            }
         }
     }
 }
@@ -198,6 +209,7 @@ bool launch_convert_tma(const bdl_layout *l, const void *dense, void *bricked, c
     P.nxb = (Wg + 63) / 64;
     P.ncb = C / 64;
     P.R = std::min(l->Bh, 2);   // small tiles: many CTAs per SM keep enough TMA traffic in flight
+    if (const char *e = getenv("BDL_BRICKIFY_R")) P.R = std::max(1, std::min(l->Bh, atoi(e)));   // A/B knob
     while ((nbh * l->Bh) % P.R) P.R--;
     // dense NCHW viewed as (W, C/8, 8, H, N) with c = 8g + k: the box lands as [row][k][g][x]
     {
@@ -232,6 +244,7 @@ bool launch_convert_tma(const bdl_layout *l, const void *dense, void *bricked, c
         const size_t smem_b = (size_t)P.nxb * P.R * 64 * 128;   // no staging tile: direct stores
         const long long grid = (long long)N * (nbh * l->Bh / P.R) * P.ncb;
         cudaFuncSetAttribute(brickify_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_b);
+        cudaFuncSetAttribute(brickify_tma_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
         brickify_tma_kernel<<<(unsigned)grid, 128, smem_b, s>>>(P);
     } else {
         const long long grid = (long long)N * ((H + P.R - 1) / P.R) * P.ncb;
