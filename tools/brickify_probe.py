@@ -8,12 +8,17 @@ plan = engine.plan_from_workload(wl)
 x = wl["x"].to(device="cuda", dtype=plan.tdtype).contiguous()
 xb = plan.alloc_bricked(plan.in_layout)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+flush_rd = torch.ones(64 << 20, dtype=torch.float32, device="cuda")   # bench.py's flush: write, then read
+MODE = os.environ.get("PROBE_FLUSH", "bench")
+def do_flush(it):
+    flush.fill_(it & 0xFF)
+    if MODE == "bench": flush_rd.sum()
 ref = None
 for R in sys.argv[1:] or ["1", "2", "4", "8", "2"]:
     os.environ["BDL_BRICKIFY_R"] = R
     ts = []
     for it in range(30):
-        flush.fill_(it & 0xFF)
+        do_flush(it)
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(); plan.brickify(x, out=xb); b.record(); b.synchronize()
         if it >= 5: ts.append(a.elapsed_time(b) * 1e3)
@@ -27,7 +32,7 @@ for R in sys.argv[1:] or ["1", "2", "4", "8", "2"]:
 dst = torch.empty_like(x)
 ts = []
 for it in range(30):
-    flush.fill_(it & 0xFF)
+    do_flush(it)
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     a.record(); dst.copy_(x); b.record(); b.synchronize()
     if it >= 5: ts.append(a.elapsed_time(b) * 1e3)
