@@ -65,6 +65,7 @@ struct LayerP {
     int pout[3];              // pooled output extents (d, h, w); out_ext stays the conv's
     int Tpb, Tpw;
     const float *bias;        // [cout]
+    int bofs;                 // float offset of this layer's bias in the shared bias table (Params::bias_off)
     int relu, has_res;
     int cin, cout;
     int k[3], s[3], pd[3];    // (d, h, w)
@@ -101,6 +102,8 @@ struct Params {
     int L;
     int nin, nw, in_stride, w_stride;    // ring depths and slot strides (bytes)
     int pool_off;                        // fused pool: byte offset of the epilogue staging tile in dynamic smem
+    int bias_off;                        // byte offset of the fp32 bias table (every layer's cout) in dynamic smem, or
+                                         // -1: the epilogue then reads each item's biases by one global load + shuffles
     int nacc, acc_stride, tmem_cols;
     int *status;
     int defer;                           // bdl_plan_opts.memo_defer: 1 = hand over only ready tasks (revisit the others)
@@ -951,6 +954,11 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
         else { aoff = tap_px(tap); lbo = t1 >= 0 ? (uint32_t)(tap_px(t1) - tap_px(tap)) : 0u; }
         sh.ks[l][q] = (aoff & 0xFFFF) | (lbo << 16);
     }
+    if (p.bias_off >= 0) {   // the biases are weights (not the previous kernel's output): staged before the PDL wait
+        float *bt = reinterpret_cast<float *>(smem + p.bias_off);
+        for (int l = 0; l < p.L; l++)
+            for (int c = threadIdx.x; c < p.layer[l].cout; c += 32 * (kEpi0 + EPIW)) bt[p.layer[l].bofs + c] = p.layer[l].bias[c];
+    }
     if (threadIdx.x == 0) {
         for (int i = 0; i < kQ; i++) {
             ptx::mbar_init(&sh.q_full[i], 1);
@@ -1288,7 +1296,9 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
                         const int m = tl * 128 + quad * 32 + lane;
                         // one coalesced bias load per item (lane c holds channel ch0 + c), issued before the TMEM load;
                         // lanes take their channels' values by shuffle
-                        const float bl = __ldg(L.bias + ch0 + (lane & (CB - 1)));
+                        const bool bsm = p.bias_off >= 0;   // shared bias table (warp-uniform)
+                        const float bl = bsm ? 0.f : __ldg(L.bias + ch0 + (lane & (CB - 1)));
+                        const float4 *bsv = reinterpret_cast<const float4 *>(smem + p.bias_off) + ((L.bofs + ch0) >> 2);
                         uint32_t r[2][16];
                         const uint32_t taddr =
                             tmem_base + a * p.acc_stride + ((uint32_t)(quad * 32) << 16) + tl * L.Nc + (cb0 + cbl) * CB;
@@ -1302,10 +1312,18 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
                             if (k >= nck) break;
                             float v[8];
 #pragma unroll
-                            for (int e = 0; e < 8; e++) {
-                                v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]) + __shfl_sync(0xffffffffu, bl, k * 8 + e);
-                                if (L.relu) v[e] = fmaxf(v[e], 0.f);
+                            for (int e = 0; e < 8; e++) v[e] = __uint_as_float(r[k / 2][(k % 2) * 8 + e]);
+                            if (bsm) {
+                                const float4 b0 = bsv[2 * k], b1 = bsv[2 * k + 1];
+                                v[0] += b0.x; v[1] += b0.y; v[2] += b0.z; v[3] += b0.w;
+                                v[4] += b1.x; v[5] += b1.y; v[6] += b1.z; v[7] += b1.w;
+                            } else {
+#pragma unroll
+                                for (int e = 0; e < 8; e++) v[e] += __shfl_sync(0xffffffffu, bl, k * 8 + e);
                             }
+#pragma unroll
+                            for (int e = 0; e < 8; e++)
+                                if (L.relu) v[e] = fmaxf(v[e], 0.f);
                             stg[m * nchk + ((cbl * nck + k) ^ (m & (nchk - 1)))] =
                                 make_uint4(pack2(v[0], v[1]), pack2(v[2], v[3]), pack2(v[4], v[5]), pack2(v[6], v[7]));
                         }
@@ -1367,7 +1385,9 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
                 // chunk, which the compiler may not move it past).  Measured on B200 against per-chunk bias loads and
                 // in-order residual loads: cfg4 11.46 -> 11.25 ms, cfg3 7.28 -> 7.16 ms; all four residual chunks up
                 // front (registers), two chunks ahead, or 16-channel items with the next item's reads in flight were slower.
-                const float bl = DBG(p, 8) ? 0.f : __ldg(L.bias + ch0 + (lane & (CB - 1)));
+                const bool bsm = p.bias_off >= 0;   // (warp-uniform)
+                const float bl = DBG(p, 8) || bsm ? 0.f : __ldg(L.bias + ch0 + (lane & (CB - 1)));
+                const float4 *bsv = reinterpret_cast<const float4 *>(smem + p.bias_off) + ((L.bofs + ch0) >> 2);
                 const bool has_rs = L.has_res && kind == 2 && !DBG(p, 16);
                 const uint4 *rsp = has_rs ? reinterpret_cast<const uint4 *>(resp + pix_pow2(L.res, L.lB, T.n, d, y, x) + ch0) : nullptr;
                 uint32_t rnext[8] = {0, 0, 0, 0, 0, 0, 0, 0};   // residual: 16 channels per 256-bit load, one pair ahead
@@ -1400,8 +1420,15 @@ __global__ void __launch_bounds__(32 * (kEpi0 + EPIW), 1) gen_kernel(const __gri
                         const int k = 2 * k2 + h;
                         float v[8];
 #pragma unroll
-                        for (int e = 0; e < 8; e++)
-                            v[e] = __uint_as_float(r[k2][h * 8 + e]) + __shfl_sync(0xffffffffu, bl, k * 8 + e);
+                        for (int e = 0; e < 8; e++) v[e] = __uint_as_float(r[k2][h * 8 + e]);
+                        if (bsm) {   // shared bias table: two broadcast 16-B reads per 8 channels
+                            const float4 b0 = bsv[2 * k], b1 = bsv[2 * k + 1];
+                            v[0] += b0.x; v[1] += b0.y; v[2] += b0.z; v[3] += b0.w;
+                            v[4] += b1.x; v[5] += b1.y; v[6] += b1.z; v[7] += b1.w;
+                        } else {
+#pragma unroll
+                            for (int e = 0; e < 8; e++) v[e] += __shfl_sync(0xffffffffu, bl, k * 8 + e);
+                        }
                         if (has_rs) {
                             const __nv_bfloat162 *h2 = reinterpret_cast<const __nv_bfloat162 *>(&rr[h * 4]);
 #pragma unroll
@@ -2233,6 +2260,23 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
     }
     P.nin = g.nin;
     P.pool_off = g.nin * g.in_stride + g.nw * g.w_stride;
+    // fp32 bias table in the shared memory left over (BDL_GEN_BIAS_SMEM=0: A/B knob, per-item global loads)
+    int smem_launch = g.smem;
+    {
+        static const int bias_env = [] { const char *e = getenv("BDL_GEN_BIAS_SMEM"); return e ? atoi(e) : 1; }();
+        int bt = 0;
+        for (int j = 0; j < L; j++) {
+            P.layer[j].bofs = bt;
+            bt += (P.layer[j].cout + 3) / 4 * 4;
+        }
+        const int boff = (P.pool_off + g.pool_bytes + 15) / 16 * 16;
+        const int need = boff + bt * 4 + 1024;   // (+ the 1024-B alignment slack of g.smem)
+        P.bias_off = -1;
+        if (bias_env && need <= 227 * 1024 - (int)sizeof(gen::Shared) - 1024) {
+            P.bias_off = boff;
+            smem_launch = std::max(g.smem, need);
+        }
+    }
     P.in_stride = g.in_stride;
     P.nw = g.nw;
     P.w_stride = g.w_stride;
@@ -2247,7 +2291,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
     auto kern = any_stk ? (g.epiw == 8 ? gen::gen_kernel<true, 8> : gen::gen_kernel<true, 12>)
                         : (g.epiw == 8 ? gen::gen_kernel<false, 8> : gen::gen_kernel<false, 12>);
     const int nthreads = 32 * (gen::kEpi0 + g.epiw);
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, g.smem);
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_launch);
     const bool unmerged = sg.mode == BDL_MODE_UNMERGED || L == 1;
     if (padded) {
         P.padded = 1;
@@ -2260,14 +2304,14 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
         P.scr_slot = g.scr_slot;
         P.norder = (long long)p->layers[sg.first].in_ext[0] * g.npb[0] * g.npb[1] * g.npb[2];
         const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-        launch_pdl(kern, dim3(grid), dim3(nthreads), g.smem, s, P);
+        launch_pdl(kern, dim3(grid), dim3(nthreads), smem_launch, s, P);
         *launches += 1;
     } else if (!unmerged) {
         P.only_layer = -1;
         P.order = (const int *)(wsp + sg.order_off);
         P.norder = sg.norder;
         const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-        launch_pdl(kern, dim3(grid), dim3(nthreads), g.smem, s, P);
+        launch_pdl(kern, dim3(grid), dim3(nthreads), smem_launch, s, P);
         *launches += 1;
     } else {
         P.order = nullptr;
@@ -2275,7 +2319,7 @@ bdl_status launch_gen_subgraph(bdl_plan *p, Subgraph &sg, const std::vector<TVie
             P.only_layer = j;
             P.norder = P.layer[j].ntasks;
             const int grid = (int)std::min<long long>(P.norder, p->num_sms);
-            launch_pdl(kern, dim3(grid), dim3(nthreads), g.smem, s, P);
+            launch_pdl(kern, dim3(grid), dim3(nthreads), smem_launch, s, P);
             *launches += 1;
         }
     }
