@@ -3,7 +3,8 @@
 Several choices of `chain_tc_gen.cu` are made per subgraph at launch time, each with an A/B switch read once per
 process from the environment: the epilogue warp count (BDL_GEN_EPIW: 8 or 12, a template instantiation), the TMA box
 per brick row of the 1x1 layers (BDL_GEN_TMA4=0: one box per pixel row), the element-strided TMA rows of 3x3
-stride-2 layers (BDL_GEN_TMA3=0: cp.async), and the shallow-K weight-stage split (BDL_GEN_NW2).  Loads and the
+stride-2 layers (BDL_GEN_TMA3=0: cp.async), the shallow-K weight-stage split (BDL_GEN_NW2), and the epilogue's
+bias source (BDL_GEN_BIAS_SMEM=0: a global load + shuffles per item instead of the shared fp32 table).  Loads and the
 epilogue's partition of work never change an output element's accumulation order, so every setting must give
 bit-identical outputs.  Each setting runs in its own process (the switches are static) on a reduced ResNet-50
 (stem, pools, projection and identity bottlenecks, stride-2 3x3 convs, 1x1 layers at brick-misaligned extents) and
@@ -45,5 +46,5 @@ def digest(cfg, N, H, **env):
 def test_alternative_paths_bit_identical(cfg, N, H):
     base = digest(cfg, N, H)
     for env in (dict(BDL_GEN_EPIW=8), dict(BDL_GEN_EPIW=12), dict(BDL_GEN_TMA4=0), dict(BDL_GEN_TMA3=0),
-                dict(BDL_GEN_NW2=0), dict(BDL_GEN_NW2=1)):
+                dict(BDL_GEN_NW2=0), dict(BDL_GEN_NW2=1), dict(BDL_GEN_BIAS_SMEM=0)):
         assert digest(cfg, N, H, **env) == base, env
