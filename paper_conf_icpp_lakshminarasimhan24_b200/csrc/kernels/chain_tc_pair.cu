@@ -664,7 +664,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1) memo_pa
                                 const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(w8);
                                 __nv_bfloat16 *q = p.dense + (((long long)img * C + c * 16) * p.H + y) * p.W + x;
 #pragma unroll
-                                for (int e = 0; e < 16; e++) q[(long long)e * p.H * p.W] = h[e];
+                                for (int e = 0; e < 16; e++)   // streaming stores: the graph output is not re-read here
+                                    asm volatile("st.global.cs.b16 [%0], %1;" ::"l"(q + (long long)e * p.H * p.W),
+                                                 "h"(__bfloat16_as_ushort(h[e])) : "memory");
                             }
                         } else {
                             st_v8(dst + c * 32, w8);
